@@ -1,0 +1,1065 @@
+// avfs_host.cpp -- host runtime behind include/avfs.h.
+//
+// Native pieces of the flow of Fig. 2:
+//   * .bench parser with full-scan DFF cut
+//   * levelizer: ASAP levels, gates sorted by level
+//   * liveness allocator: interval colouring of waveform buffers over levels
+//     (waveform storage dominates); POs / probes are pinned
+//   * coefficient store: per-cell blocks, or per-gate blocks with the
+//     load capacitance folded in (alpha_i = sum_j beta_ij phi_C(c)^j) when
+//     deg_c > 0
+//   * simulate driver: stimulus expansion, persistent sweep, overflow reruns
+//   * readback (P:L141 step 4)
+// Every arithmetic step of the simulation itself runs in avfs_kernels.cu.
+#include "avfs.h"
+
+#include <algorithm>
+#include <chrono>
+#include <cmath>
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <string>
+#include <unordered_map>
+#include <vector>
+
+#include "avfs_internal.h"
+
+using namespace avfs;
+
+namespace {
+
+struct DevBuf {
+    void* p = nullptr;
+    size_t n = 0;
+    DevBuf() = default;
+    DevBuf(const DevBuf&) = delete;
+    DevBuf& operator=(const DevBuf&) = delete;
+    DevBuf(DevBuf&& o) noexcept : p(o.p), n(o.n) { o.p = nullptr; o.n = 0; }
+    ~DevBuf() { release(); }
+    void release() {
+        if (p) cudaFree(p);
+        p = nullptr;
+        n = 0;
+    }
+    cudaError_t ensure(size_t bytes) {
+        if (bytes <= n && p) return cudaSuccess;
+        release();
+        size_t b = bytes ? bytes : 16;
+        cudaError_t e = cudaMalloc(&p, b);
+        if (e == cudaSuccess) n = b;
+        else p = nullptr;
+        return e;
+    }
+    template <class T> T* as() const { return static_cast<T*>(p); }
+};
+
+struct Round {
+    int64_t n_sw = 0;
+    int64_t sw_first = 0;            // pass 0: contiguous range
+    std::vector<int32_t> sws;        // reruns: explicit list
+    int32_t capacity = 0, W = 0, cstage = 0;
+    int64_t region_bytes = 0;
+    int32_t grid = 0;
+};
+
+}  // namespace
+
+struct avfs_ctx {
+    int dev = -1;
+    int n_sm = 0;
+    bool sticky = false;
+    std::string err;
+    cudaStream_t stream = nullptr;
+
+    // library
+    bool lib_loaded = false;
+    std::vector<std::string> cell_names;
+    std::vector<int32_t> cell_nin;
+    std::vector<uint16_t> cell_tt;
+    int32_t deg_v = 0, deg_c = 0;
+    std::vector<double> beta;
+    double v_min = 0.55, v_max = 1.1, c_min = 0.5, c_max = 128.0;
+
+    // netlist
+    bool net_loaded = false;
+    int32_t n_pi = 0, n_gates = 0;
+    std::vector<int32_t> gate_cell;
+    std::vector<int64_t> fanin_ptr;
+    std::vector<int32_t> fanin_sig;
+    std::vector<double> d_nom, c_load;
+    std::vector<int32_t> po;
+    std::unordered_map<std::string, int32_t> names;
+
+    // levelised view
+    std::vector<int32_t> level;       // per signal
+    std::vector<int32_t> order;       // gates sorted by level
+    std::vector<int32_t> level_ptr;   // [depth+1]
+    std::vector<int32_t> last_read;   // per signal: max level of a reader, -1 none
+    std::vector<int64_t> fanout;      // gate pins reading each signal
+    std::vector<uint8_t> is_po;       // per signal
+    int32_t depth = 0, kmax = 1, n_dangling = 0;
+    std::vector<double> coef;         // coefficient blocks
+    std::vector<uint32_t> coef_off;   // per gate
+
+    // plan (options dependent)
+    bool plan_valid = false;
+    std::vector<uint32_t> loc;        // per signal
+    int32_t n_scratch = 0, n_pinned = 0;
+
+    avfs_options opt{};
+    std::vector<int32_t> probes;
+
+    std::vector<double> vdd;
+    int64_t n_pairs = 0;
+    int32_t words = 0;
+    bool stim_set = false;
+    int64_t slot_first = 0, slot_count = -1;
+
+    // device state
+    bool dev_net_valid = false, dev_vdd_valid = false;
+    DevBuf d_gates, d_coef, d_level_ptr, d_vdd, d_p1, d_p2, d_p1t, d_p2t, d_act, d_latest, d_ovf,
+        d_err, d_list[2], d_count, d_swround, d_swindex, g_loc, g_init, g_count, g_times, g_bad;
+    std::vector<DevBuf> scr, pin;     // per round
+    int32_t* h_pinned = nullptr;      // small pinned host buffer (count, err)
+    cudaEvent_t ev0 = nullptr, ev1 = nullptr;
+
+    // last simulation
+    bool sim_done = false, map_valid = false;
+    std::vector<Round> rounds;
+    int64_t sim_first = 0, sim_end = 0;
+    avfs_stats stats{};
+};
+
+namespace {
+
+avfs_status fail(avfs_ctx* c, avfs_status st, const char* fmt, ...) {
+    char buf[512];
+    va_list ap;
+    va_start(ap, fmt);
+    vsnprintf(buf, sizeof buf, fmt, ap);
+    va_end(ap);
+    if (c) {
+        c->err = buf;
+        if (st == AVFS_ERR_CUDA) c->sticky = true;
+    }
+    return st;
+}
+
+#define CK(call)                                                                                   \
+    do {                                                                                           \
+        cudaError_t e_ = (call);                                                                   \
+        if (e_ != cudaSuccess) {                                                                   \
+            if (e_ == cudaErrorMemoryAllocation) {                                                 \
+                cudaGetLastError();                                                                \
+                return fail(ctx, AVFS_ERR_NOMEM, "%s: %s", #call, cudaGetErrorString(e_));         \
+            }                                                                                      \
+            return fail(ctx, AVFS_ERR_CUDA, "%s: %s", #call, cudaGetErrorString(e_));              \
+        }                                                                                          \
+    } while (0)
+
+#define CHECK_CTX()                                                                                \
+    do {                                                                                           \
+        if (!ctx) return AVFS_ERR_ARG;                                                             \
+        if (ctx->sticky) return AVFS_ERR_CUDA;                                                     \
+        ctx->err.clear();                                                                          \
+    } while (0)
+
+bool has_dev(const avfs_ctx* c) { return c->dev >= 0; }
+
+// ---------------------------------------------------------------- levelizer
+avfs_status levelize(avfs_ctx* ctx) {
+    const int32_t G = ctx->n_gates, S = ctx->n_pi + G;
+    ctx->level.assign(S, 0);
+    ctx->fanout.assign(S, 0);
+    std::vector<int64_t> fo_ptr(S + 1, 0);
+    for (int64_t e = 0; e < ctx->fanin_ptr[G]; ++e) fo_ptr[ctx->fanin_sig[e] + 1]++;
+    for (int32_t s = 0; s < S; ++s) {
+        ctx->fanout[s] = fo_ptr[s + 1];
+        fo_ptr[s + 1] += fo_ptr[s];
+    }
+    std::vector<int32_t> fo_gate(ctx->fanin_ptr[G]);
+    {
+        std::vector<int64_t> fill(fo_ptr.begin(), fo_ptr.end() - 1);
+        for (int32_t g = 0; g < G; ++g)
+            for (int64_t e = ctx->fanin_ptr[g]; e < ctx->fanin_ptr[g + 1]; ++e)
+                fo_gate[fill[ctx->fanin_sig[e]]++] = g;
+    }
+    std::vector<int32_t> indeg(G, 0), queue;
+    queue.reserve(G);
+    for (int32_t g = 0; g < G; ++g) {
+        for (int64_t e = ctx->fanin_ptr[g]; e < ctx->fanin_ptr[g + 1]; ++e)
+            indeg[g] += ctx->fanin_sig[e] >= ctx->n_pi;
+        if (!indeg[g]) queue.push_back(g);
+    }
+    for (size_t h = 0; h < queue.size(); ++h) {
+        const int32_t g = queue[h];
+        int32_t lv = 0;
+        for (int64_t e = ctx->fanin_ptr[g]; e < ctx->fanin_ptr[g + 1]; ++e)
+            lv = std::max(lv, ctx->level[ctx->fanin_sig[e]]);
+        ctx->level[ctx->n_pi + g] = lv + 1;
+        const int32_t s = ctx->n_pi + g;
+        for (int64_t f = fo_ptr[s]; f < fo_ptr[s + 1]; ++f)
+            if (--indeg[fo_gate[f]] == 0) queue.push_back(fo_gate[f]);
+    }
+    if ((int32_t)queue.size() != G) return fail(ctx, AVFS_ERR_PARSE, "netlist has a combinational cycle");
+    ctx->depth = 0;
+    for (int32_t g = 0; g < G; ++g) ctx->depth = std::max(ctx->depth, ctx->level[ctx->n_pi + g]);
+    ctx->order.resize(G);
+    for (int32_t g = 0; g < G; ++g) ctx->order[g] = g;
+    std::stable_sort(ctx->order.begin(), ctx->order.end(), [&](int32_t a, int32_t b) {
+        return ctx->level[ctx->n_pi + a] < ctx->level[ctx->n_pi + b];
+    });
+    ctx->level_ptr.assign(ctx->depth + 1, 0);
+    for (int32_t g = 0; g < G; ++g) ctx->level_ptr[ctx->level[ctx->n_pi + g]]++;
+    for (int32_t L = 1; L <= ctx->depth; ++L) ctx->level_ptr[L] += ctx->level_ptr[L - 1];
+    ctx->last_read.assign(S, -1);
+    for (int32_t g = 0; g < G; ++g)
+        for (int64_t e = ctx->fanin_ptr[g]; e < ctx->fanin_ptr[g + 1]; ++e) {
+            int32_t& lr = ctx->last_read[ctx->fanin_sig[e]];
+            lr = std::max(lr, ctx->level[ctx->n_pi + g]);
+        }
+    ctx->is_po.assign(S, 0);
+    for (int32_t s : ctx->po) ctx->is_po[s] = 1;
+    ctx->n_dangling = 0;
+    for (int32_t g = 0; g < G; ++g)
+        ctx->n_dangling += (ctx->last_read[ctx->n_pi + g] < 0 && !ctx->is_po[ctx->n_pi + g]);
+    ctx->kmax = 1;
+    for (int32_t g = 0; g < G; ++g)
+        ctx->kmax = std::max<int32_t>(ctx->kmax, (int32_t)(ctx->fanin_ptr[g + 1] - ctx->fanin_ptr[g]));
+    return AVFS_OK;
+}
+
+// ---------------------------------------------------------------- coefficient store
+void build_coef(avfs_ctx* ctx) {
+    const int dv = ctx->deg_v, dc = ctx->deg_c;
+    const size_t blk = 8 * (size_t)(dv + 1);
+    auto b = [&](int cell, int pin, int pol, int i, int j) {
+        return ctx->beta[((((size_t)cell * 4 + pin) * 2 + pol) * (dv + 1) + i) * (dc + 1) + j];
+    };
+    ctx->coef_off.assign(ctx->n_gates, 0);
+    if (dc == 0) {
+        const int nc = (int)ctx->cell_nin.size();
+        ctx->coef.assign(nc * blk, 0.0);
+        for (int c = 0; c < nc; ++c)
+            for (int pin = 0; pin < 4; ++pin)
+                for (int pol = 0; pol < 2; ++pol)
+                    for (int i = 0; i <= dv; ++i)
+                        ctx->coef[c * blk + (pin * 2 + pol) * (dv + 1) + i] = b(c, pin, pol, i, 0);
+        for (int32_t g = 0; g < ctx->n_gates; ++g) ctx->coef_off[g] = (uint32_t)(ctx->gate_cell[g] * blk);
+    } else {
+        // Load-time fold of the load capacitance (deg_c > 0): phi_C and
+        // the inner Horner in phi_C with fma, so the kernel's Horner in phi_V
+        // evaluates exactly the nested Horner of Eq. (4).
+        ctx->coef.assign((size_t)ctx->n_gates * blk, 0.0);
+        const double lc0 = std::log2(ctx->c_min), lc1 = std::log2(ctx->c_max);
+        for (int32_t g = 0; g < ctx->n_gates; ++g) {
+            const double z = (std::log2(ctx->c_load[g]) - lc0) / (lc1 - lc0);
+            const int c = ctx->gate_cell[g];
+            for (int pin = 0; pin < 4; ++pin)
+                for (int pol = 0; pol < 2; ++pol)
+                    for (int i = 0; i <= dv; ++i) {
+                        double a = b(c, pin, pol, i, dc);
+                        for (int j = dc - 1; j >= 0; --j) a = std::fma(a, z, b(c, pin, pol, i, j));
+                        ctx->coef[g * blk + (pin * 2 + pol) * (dv + 1) + i] = a;
+                    }
+            ctx->coef_off[g] = (uint32_t)(g * blk);
+        }
+    }
+}
+
+// ---------------------------------------------------------------- liveness allocator
+avfs_status build_plan(avfs_ctx* ctx) {
+    if (ctx->plan_valid) return AVFS_OK;
+    const int32_t G = ctx->n_gates, S = ctx->n_pi + G;
+    std::vector<uint8_t> pinned(S, 0);
+    for (int32_t s = ctx->n_pi; s < S; ++s)
+        if (ctx->opt.keep_all || ctx->is_po[s]) pinned[s] = 1;
+    for (int32_t s : ctx->probes)
+        if (s >= ctx->n_pi) pinned[s] = 1;
+    ctx->loc.assign(S, 0);
+    for (int32_t i = 0; i < ctx->n_pi; ++i) ctx->loc[i] = LOC_PI | (uint32_t)i;
+    int32_t np = 0;
+    for (int32_t s = ctx->n_pi; s < S; ++s)
+        if (pinned[s]) ctx->loc[s] = LOC_PINNED | (uint32_t)np++;
+    ctx->n_pinned = np;
+    // interval colouring: a buffer written at level L and last read at level R
+    // may be rewritten from level max(L, R) + 1 on (the CTA barrier between
+    // levels orders the last read before the rewrite).
+    std::vector<std::vector<int32_t>> release(ctx->depth + 2);
+    std::vector<int32_t> free_list;
+    int32_t n_buf = 0;
+    for (int32_t L = 1; L <= ctx->depth; ++L) {
+        for (int32_t b : release[L]) free_list.push_back(b);
+        for (int32_t i = ctx->level_ptr[L - 1]; i < ctx->level_ptr[L]; ++i) {
+            const int32_t s = ctx->n_pi + ctx->order[i];
+            if (pinned[s]) continue;
+            int32_t b;
+            if (!free_list.empty()) { b = free_list.back(); free_list.pop_back(); }
+            else b = n_buf++;
+            ctx->loc[s] = LOC_SCRATCH | (uint32_t)b;
+            const int32_t until = std::max(L, ctx->last_read[s]);
+            release[until + 1].push_back(b);
+        }
+    }
+    ctx->n_scratch = n_buf;
+    ctx->plan_valid = true;
+    ctx->dev_net_valid = false;
+    return AVFS_OK;
+}
+
+avfs_status upload_netlist(avfs_ctx* ctx) {
+    if (ctx->dev_net_valid) return AVFS_OK;
+    const int32_t G = ctx->n_gates;
+    std::vector<GateDesc> gd(std::max<int32_t>(G, 1));
+    for (int32_t i = 0; i < G; ++i) {
+        const int32_t g = ctx->order[i];
+        GateDesc& d = gd[i];
+        std::memset(&d, 0, sizeof d);
+        const int k = (int)(ctx->fanin_ptr[g + 1] - ctx->fanin_ptr[g]);
+        for (int p = 0; p < KMAX; ++p) d.in_loc[p] = p < k ? ctx->loc[ctx->fanin_sig[ctx->fanin_ptr[g] + p]] : 0u;
+        d.out_loc = ctx->loc[ctx->n_pi + g];
+        d.sig = (uint32_t)(ctx->n_pi + g);
+        d.tt = ctx->cell_tt[ctx->gate_cell[g]];
+        d.k = (uint8_t)k;
+        d.flags = ctx->is_po[ctx->n_pi + g] ? 1 : 0;
+        d.coef_off = ctx->coef_off[g];
+        for (int p = 0; p < k; ++p)
+            for (int pol = 0; pol < 2; ++pol) d.dnom[2 * p + pol] = ctx->d_nom[(ctx->fanin_ptr[g] + p) * 2 + pol];
+        for (int p = k; p < KMAX; ++p) d.dnom[2 * p] = d.dnom[2 * p + 1] = 1.0;
+    }
+    CK(ctx->d_gates.ensure(gd.size() * sizeof(GateDesc)));
+    CK(cudaMemcpy(ctx->d_gates.p, gd.data(), gd.size() * sizeof(GateDesc), cudaMemcpyHostToDevice));
+    CK(ctx->d_coef.ensure(std::max<size_t>(ctx->coef.size(), 1) * sizeof(double)));
+    if (!ctx->coef.empty())
+        CK(cudaMemcpy(ctx->d_coef.p, ctx->coef.data(), ctx->coef.size() * sizeof(double), cudaMemcpyHostToDevice));
+    CK(ctx->d_level_ptr.ensure(ctx->level_ptr.size() * sizeof(int32_t)));
+    CK(cudaMemcpy(ctx->d_level_ptr.p, ctx->level_ptr.data(), ctx->level_ptr.size() * sizeof(int32_t),
+                  cudaMemcpyHostToDevice));
+    ctx->dev_net_valid = true;
+    return AVFS_OK;
+}
+
+void invalidate_sim(avfs_ctx* ctx) {
+    ctx->sim_done = false;
+    ctx->map_valid = false;
+}
+
+// ---------------------------------------------------------------- .bench parser
+std::string trim(const std::string& s) {
+    size_t a = 0, b = s.size();
+    while (a < b && isspace((unsigned char)s[a])) ++a;
+    while (b > a && isspace((unsigned char)s[b - 1])) --b;
+    return s.substr(a, b - a);
+}
+
+std::string upper(std::string s) {
+    for (auto& ch : s) ch = (char)toupper((unsigned char)ch);
+    return s;
+}
+
+}  // namespace
+
+// ============================================================================ C-ABI
+extern "C" {
+
+const char* avfs_version(void) { return "avfs 0.1 sm_100a"; }
+
+const char* avfs_status_string(avfs_status st) {
+    switch (st) {
+        case AVFS_OK: return "AVFS_OK";
+        case AVFS_ERR_ARG: return "AVFS_ERR_ARG";
+        case AVFS_ERR_PARSE: return "AVFS_ERR_PARSE";
+        case AVFS_ERR_STATE: return "AVFS_ERR_STATE";
+        case AVFS_ERR_CUDA: return "AVFS_ERR_CUDA";
+        case AVFS_ERR_NOMEM: return "AVFS_ERR_NOMEM";
+        case AVFS_ERR_DELAY_NONPOS: return "AVFS_ERR_DELAY_NONPOS";
+        case AVFS_ERR_CAPACITY: return "AVFS_ERR_CAPACITY";
+    }
+    return "unknown";
+}
+
+avfs_status avfs_default_options(avfs_options* o) {
+    if (!o) return AVFS_ERR_ARG;
+    std::memset(o, 0, sizeof *o);
+    o->capacity = 8;
+    o->max_rerun_rounds = 3;
+    o->warps_per_cta = 8;
+    return AVFS_OK;
+}
+
+avfs_status avfs_create(int cuda_device, avfs_ctx** out) {
+    if (!out) return AVFS_ERR_ARG;
+    *out = nullptr;
+    avfs_ctx* ctx = new (std::nothrow) avfs_ctx();
+    if (!ctx) return AVFS_ERR_NOMEM;
+    avfs_default_options(&ctx->opt);
+    if (cuda_device >= 0) {
+        int n = 0;
+        cudaError_t e = cudaGetDeviceCount(&n);
+        if (e != cudaSuccess || cuda_device >= n) {
+            cudaGetLastError();
+            delete ctx;
+            return AVFS_ERR_CUDA;
+        }
+        ctx->dev = cuda_device;
+        if (cudaSetDevice(cuda_device) != cudaSuccess ||
+            cudaDeviceGetAttribute(&ctx->n_sm, cudaDevAttrMultiProcessorCount, cuda_device) != cudaSuccess ||
+            cudaMallocHost(&ctx->h_pinned, 64) != cudaSuccess ||
+            cudaEventCreate(&ctx->ev0) != cudaSuccess || cudaEventCreate(&ctx->ev1) != cudaSuccess) {
+            cudaGetLastError();
+            delete ctx;
+            return AVFS_ERR_CUDA;
+        }
+    }
+    *out = ctx;
+    return AVFS_OK;
+}
+
+void avfs_destroy(avfs_ctx* ctx) {
+    if (!ctx) return;
+    if (ctx->dev >= 0) {
+        cudaSetDevice(ctx->dev);
+        if (ctx->h_pinned) cudaFreeHost(ctx->h_pinned);
+        if (ctx->ev0) cudaEventDestroy(ctx->ev0);
+        if (ctx->ev1) cudaEventDestroy(ctx->ev1);
+    }
+    delete ctx;
+}
+
+const char* avfs_last_error(const avfs_ctx* ctx) { return ctx ? ctx->err.c_str() : "null context"; }
+
+avfs_status avfs_load_library(avfs_ctx* ctx, int32_t n_cells, const avfs_cell* cells, int32_t deg_v,
+                              int32_t deg_c, const double* beta, double v_min, double v_max,
+                              double c_min_fF, double c_max_fF) {
+    CHECK_CTX();
+    if (n_cells <= 0 || !cells || !beta) return fail(ctx, AVFS_ERR_ARG, "null library arrays");
+    if (deg_v < 0 || deg_v > MAX_DEG || deg_c < 0 || deg_c > MAX_DEG)
+        return fail(ctx, AVFS_ERR_ARG, "polynomial degree out of range [0,%d]", MAX_DEG);
+    if (!(v_max > v_min) || !(c_max_fF > c_min_fF) || !(c_min_fF > 0))
+        return fail(ctx, AVFS_ERR_ARG, "bad normalisation bounds");
+    ctx->cell_names.clear();
+    ctx->cell_nin.clear();
+    ctx->cell_tt.clear();
+    for (int32_t c = 0; c < n_cells; ++c) {
+        if (cells[c].n_inputs < 1 || cells[c].n_inputs > KMAX)
+            return fail(ctx, AVFS_ERR_ARG, "cell %d: n_inputs must be 1..4", c);
+        ctx->cell_names.push_back(cells[c].name ? upper(cells[c].name) : std::string());
+        ctx->cell_nin.push_back(cells[c].n_inputs);
+        ctx->cell_tt.push_back(cells[c].truth_table);
+    }
+    const size_t nb = (size_t)n_cells * 8 * (deg_v + 1) * (deg_c + 1);
+    ctx->beta.assign(beta, beta + nb);
+    for (double b : ctx->beta)
+        if (!std::isfinite(b)) return fail(ctx, AVFS_ERR_ARG, "non-finite coefficient");
+    ctx->deg_v = deg_v;
+    ctx->deg_c = deg_c;
+    ctx->v_min = v_min;
+    ctx->v_max = v_max;
+    ctx->c_min = c_min_fF;
+    ctx->c_max = c_max_fF;
+    ctx->lib_loaded = true;
+    ctx->net_loaded = false;
+    ctx->plan_valid = false;
+    ctx->dev_net_valid = false;
+    invalidate_sim(ctx);
+    return AVFS_OK;
+}
+
+avfs_status avfs_load_netlist(avfs_ctx* ctx, int32_t n_pi, int32_t n_gates, const int32_t* gate_cell,
+                              const int64_t* fanin_ptr, const int32_t* fanin_sig, const double* d_nom_ps,
+                              const double* c_load_fF, int32_t n_po, const int32_t* po_sig) {
+    CHECK_CTX();
+    if (!ctx->lib_loaded) return fail(ctx, AVFS_ERR_STATE, "load the cell library first");
+    if (n_pi < 0 || n_gates < 1 || !gate_cell || !fanin_ptr || !fanin_sig || !d_nom_ps || n_po < 0 ||
+        (n_po > 0 && !po_sig))
+        return fail(ctx, AVFS_ERR_ARG, "bad netlist arrays");
+    if (ctx->deg_c > 0 && !c_load_fF) return fail(ctx, AVFS_ERR_ARG, "c_load required when deg_c > 0");
+    const int64_t S = (int64_t)n_pi + n_gates;
+    if (S >= (int64_t)LOC_ID) return fail(ctx, AVFS_ERR_ARG, "too many signals");
+    if (fanin_ptr[0] != 0) return fail(ctx, AVFS_ERR_ARG, "fanin_ptr[0] must be 0");
+    for (int32_t g = 0; g < n_gates; ++g) {
+        const int64_t k = fanin_ptr[g + 1] - fanin_ptr[g];
+        if (gate_cell[g] < 0 || gate_cell[g] >= (int32_t)ctx->cell_nin.size())
+            return fail(ctx, AVFS_ERR_ARG, "gate %d: cell index out of range", g);
+        if (k != ctx->cell_nin[gate_cell[g]])
+            return fail(ctx, AVFS_ERR_ARG, "gate %d: %lld fan-ins for a %d-input cell", g, (long long)k,
+                        ctx->cell_nin[gate_cell[g]]);
+        for (int64_t e = fanin_ptr[g]; e < fanin_ptr[g + 1]; ++e) {
+            if (fanin_sig[e] < 0 || fanin_sig[e] >= S) return fail(ctx, AVFS_ERR_ARG, "gate %d: bad fan-in", g);
+            if (fanin_sig[e] == n_pi + g) return fail(ctx, AVFS_ERR_PARSE, "gate %d drives itself", g);
+            for (int pol = 0; pol < 2; ++pol)
+                if (!(d_nom_ps[2 * e + pol] > 0) || !std::isfinite(d_nom_ps[2 * e + pol]))
+                    return fail(ctx, AVFS_ERR_ARG, "gate %d: nominal delay must be finite and > 0", g);
+        }
+        if (c_load_fF && ctx->deg_c > 0 && !(c_load_fF[g] > 0))
+            return fail(ctx, AVFS_ERR_ARG, "gate %d: load must be > 0", g);
+    }
+    for (int32_t i = 0; i < n_po; ++i)
+        if (po_sig[i] < 0 || po_sig[i] >= S) return fail(ctx, AVFS_ERR_ARG, "bad PO signal");
+    const int64_t E = fanin_ptr[n_gates];
+    ctx->n_pi = n_pi;
+    ctx->n_gates = n_gates;
+    ctx->gate_cell.assign(gate_cell, gate_cell + n_gates);
+    ctx->fanin_ptr.assign(fanin_ptr, fanin_ptr + n_gates + 1);
+    ctx->fanin_sig.assign(fanin_sig, fanin_sig + E);
+    ctx->d_nom.assign(d_nom_ps, d_nom_ps + 2 * E);
+    if (c_load_fF) ctx->c_load.assign(c_load_fF, c_load_fF + n_gates);
+    else ctx->c_load.assign(n_gates, 1.0);
+    ctx->po.assign(po_sig, po_sig + n_po);
+    ctx->net_loaded = false;
+    avfs_status st = levelize(ctx);
+    if (st != AVFS_OK) return st;
+    build_coef(ctx);
+    ctx->net_loaded = true;
+    ctx->plan_valid = false;
+    ctx->dev_net_valid = false;
+    ctx->names.clear();
+    invalidate_sim(ctx);
+    return AVFS_OK;
+}
+
+avfs_status avfs_load_bench(avfs_ctx* ctx, const char* text, size_t len, const double* d_nom_ps,
+                            const double* c_load_fF) {
+    CHECK_CTX();
+    if (!ctx->lib_loaded) return fail(ctx, AVFS_ERR_STATE, "load the cell library first");
+    if (!text || !d_nom_ps) return fail(ctx, AVFS_ERR_ARG, "null text or delays");
+    std::vector<std::string> inputs, outputs, dff_q, dff_d;
+    struct GateLine { std::string out, type; std::vector<std::string> ins; int line; };
+    std::vector<GateLine> gates;
+    std::string src(text, len);
+    size_t pos = 0;
+    int lineno = 0;
+    while (pos <= src.size()) {
+        size_t nl = src.find('\n', pos);
+        if (nl == std::string::npos) nl = src.size();
+        std::string line = src.substr(pos, nl - pos);
+        pos = nl + 1;
+        ++lineno;
+        const size_t hash = line.find('#');
+        if (hash != std::string::npos) line = line.substr(0, hash);
+        line = trim(line);
+        if (line.empty()) continue;
+        const size_t lp = line.find('('), rp = line.rfind(')');
+        if (lp == std::string::npos || rp == std::string::npos || rp < lp)
+            return fail(ctx, AVFS_ERR_PARSE, "line %d: expected '(' ... ')'", lineno);
+        const size_t eq = line.find('=');
+        if (eq == std::string::npos || eq > lp) {
+            const std::string kw = upper(trim(line.substr(0, lp)));
+            const std::string arg = trim(line.substr(lp + 1, rp - lp - 1));
+            if (kw == "INPUT") inputs.push_back(arg);
+            else if (kw == "OUTPUT") outputs.push_back(arg);
+            else return fail(ctx, AVFS_ERR_PARSE, "line %d: unknown keyword '%s'", lineno, kw.c_str());
+            continue;
+        }
+        GateLine g;
+        g.line = lineno;
+        g.out = trim(line.substr(0, eq));
+        g.type = upper(trim(line.substr(eq + 1, lp - eq - 1)));
+        std::string args = line.substr(lp + 1, rp - lp - 1);
+        size_t a = 0;
+        while (a <= args.size()) {
+            size_t comma = args.find(',', a);
+            if (comma == std::string::npos) comma = args.size();
+            std::string t = trim(args.substr(a, comma - a));
+            if (!t.empty()) g.ins.push_back(t);
+            a = comma + 1;
+        }
+        if (g.out.empty() || g.ins.empty()) return fail(ctx, AVFS_ERR_PARSE, "line %d: malformed gate", lineno);
+        if (g.type == "DFF") {
+            if (g.ins.size() != 1) return fail(ctx, AVFS_ERR_PARSE, "line %d: DFF takes one input", lineno);
+            dff_q.push_back(g.out);
+            dff_d.push_back(g.ins[0]);
+        } else {
+            gates.push_back(g);
+        }
+    }
+    std::unordered_map<std::string, int32_t> id;
+    int32_t n_pi = 0;
+    for (auto& s : inputs) {
+        if (id.count(s)) return fail(ctx, AVFS_ERR_PARSE, "duplicate input '%s'", s.c_str());
+        id[s] = n_pi++;
+    }
+    for (auto& s : dff_q) {    // full-scan cut: DFF outputs become pseudo PIs
+        if (id.count(s)) return fail(ctx, AVFS_ERR_PARSE, "duplicate net '%s'", s.c_str());
+        id[s] = n_pi++;
+    }
+    const int32_t G = (int32_t)gates.size();
+    for (int32_t g = 0; g < G; ++g) {
+        if (id.count(gates[g].out)) return fail(ctx, AVFS_ERR_PARSE, "line %d: net '%s' driven twice", gates[g].line, gates[g].out.c_str());
+        id[gates[g].out] = n_pi + g;
+    }
+    std::vector<int32_t> cell(G), fsig;
+    std::vector<int64_t> fptr(G + 1, 0);
+    for (int32_t g = 0; g < G; ++g) {
+        const int k = (int)gates[g].ins.size();
+        std::string want = gates[g].type + std::to_string(k);
+        std::vector<std::string> cands = {want, gates[g].type};
+        if (k == 1) {
+            if (gates[g].type == "NOT" || gates[g].type == "INV") cands = {"INV", "NOT"};
+            if (gates[g].type == "BUFF" || gates[g].type == "BUF") cands = {"BUF", "BUFF"};
+        }
+        int32_t ci = -1;
+        for (auto& cn : cands) {
+            for (size_t c = 0; c < ctx->cell_names.size() && ci < 0; ++c)
+                if (ctx->cell_names[c] == cn && ctx->cell_nin[c] == k) ci = (int32_t)c;
+            if (ci >= 0) break;
+        }
+        if (ci < 0) return fail(ctx, AVFS_ERR_PARSE, "line %d: no %d-input library cell for '%s'", gates[g].line, k, gates[g].type.c_str());
+        cell[g] = ci;
+        for (auto& s : gates[g].ins) {
+            auto it = id.find(s);
+            if (it == id.end()) return fail(ctx, AVFS_ERR_PARSE, "line %d: undriven net '%s'", gates[g].line, s.c_str());
+            fsig.push_back(it->second);
+        }
+        fptr[g + 1] = (int64_t)fsig.size();
+    }
+    std::vector<int32_t> po;
+    for (auto& s : outputs) {
+        auto it = id.find(s);
+        if (it == id.end()) return fail(ctx, AVFS_ERR_PARSE, "undriven output '%s'", s.c_str());
+        po.push_back(it->second);
+    }
+    for (auto& s : dff_d) {    // DFF inputs become pseudo POs
+        auto it = id.find(s);
+        if (it == id.end()) return fail(ctx, AVFS_ERR_PARSE, "undriven DFF input '%s'", s.c_str());
+        po.push_back(it->second);
+    }
+    avfs_status st = avfs_load_netlist(ctx, n_pi, G, cell.data(), fptr.data(), fsig.data(), d_nom_ps, c_load_fF,
+                                       (int32_t)po.size(), po.data());
+    if (st != AVFS_OK) return st;
+    ctx->names = std::move(id);
+    return AVFS_OK;
+}
+
+avfs_status avfs_find_signal(avfs_ctx* ctx, const char* name, int32_t* sig) {
+    CHECK_CTX();
+    if (!name || !sig) return fail(ctx, AVFS_ERR_ARG, "null argument");
+    auto it = ctx->names.find(name);
+    if (it == ctx->names.end()) return fail(ctx, AVFS_ERR_ARG, "no net named '%s'", name);
+    *sig = it->second;
+    return AVFS_OK;
+}
+
+avfs_status avfs_get_netlist_info(avfs_ctx* ctx, avfs_netlist_info* info) {
+    CHECK_CTX();
+    if (!info) return fail(ctx, AVFS_ERR_ARG, "null info");
+    if (!ctx->net_loaded) return fail(ctx, AVFS_ERR_STATE, "no netlist");
+    avfs_status st = build_plan(ctx);
+    if (st != AVFS_OK) return st;
+    info->n_pi = ctx->n_pi;
+    info->n_gates = ctx->n_gates;
+    info->n_po = (int32_t)ctx->po.size();
+    info->depth = ctx->depth;
+    info->max_fanin = ctx->kmax;
+    info->n_scratch_buffers = ctx->n_scratch;
+    info->n_pinned = ctx->n_pinned;
+    info->n_dangling = ctx->n_dangling;
+    info->n_edges = ctx->fanin_ptr[ctx->n_gates];
+    return AVFS_OK;
+}
+
+avfs_status avfs_get_levels(avfs_ctx* ctx, int32_t* level) {
+    CHECK_CTX();
+    if (!level) return fail(ctx, AVFS_ERR_ARG, "null output");
+    if (!ctx->net_loaded) return fail(ctx, AVFS_ERR_STATE, "no netlist");
+    std::copy(ctx->level.begin(), ctx->level.end(), level);
+    return AVFS_OK;
+}
+
+avfs_status avfs_get_buffer_map(avfs_ctx* ctx, int32_t* out) {
+    CHECK_CTX();
+    if (!out) return fail(ctx, AVFS_ERR_ARG, "null output");
+    if (!ctx->net_loaded) return fail(ctx, AVFS_ERR_STATE, "no netlist");
+    avfs_status st = build_plan(ctx);
+    if (st != AVFS_OK) return st;
+    for (size_t s = 0; s < ctx->loc.size(); ++s) {
+        const uint32_t l = ctx->loc[s];
+        const uint32_t kind = l & LOC_KIND;
+        out[s] = kind == LOC_PI ? -1 : kind == LOC_SCRATCH ? (int32_t)(l & LOC_ID) : -2 - (int32_t)(l & LOC_ID);
+    }
+    return AVFS_OK;
+}
+
+avfs_status avfs_set_operating_points(avfs_ctx* ctx, int32_t n_vdd, const double* vdd) {
+    CHECK_CTX();
+    if (n_vdd < 1 || !vdd) return fail(ctx, AVFS_ERR_ARG, "need at least one operating point");
+    for (int32_t k = 0; k < n_vdd; ++k)
+        if (!std::isfinite(vdd[k])) return fail(ctx, AVFS_ERR_ARG, "non-finite Vdd");
+    ctx->vdd.assign(vdd, vdd + n_vdd);
+    ctx->dev_vdd_valid = false;
+    if (has_dev(ctx)) {
+        CK(cudaSetDevice(ctx->dev));
+        CK(ctx->d_vdd.ensure(n_vdd * sizeof(double)));
+        CK(cudaMemcpy(ctx->d_vdd.p, vdd, n_vdd * sizeof(double), cudaMemcpyHostToDevice));
+        ctx->dev_vdd_valid = true;
+    }
+    invalidate_sim(ctx);
+    return AVFS_OK;
+}
+
+avfs_status avfs_set_stimuli(avfs_ctx* ctx, int64_t n_pairs, const uint32_t* p1, const uint32_t* p2,
+                             int32_t is_device) {
+    CHECK_CTX();
+    if (!ctx->net_loaded) return fail(ctx, AVFS_ERR_STATE, "load a netlist first");
+    if (n_pairs < 1 || !p1 || !p2) return fail(ctx, AVFS_ERR_ARG, "bad stimuli");
+    if (!has_dev(ctx)) return fail(ctx, AVFS_ERR_STATE, "host-only context");
+    const int32_t words = (ctx->n_pi + 31) / 32;
+    const size_t bytes = (size_t)n_pairs * std::max(words, 1) * sizeof(uint32_t);
+    CK(cudaSetDevice(ctx->dev));
+    CK(ctx->d_p1.ensure(bytes));
+    CK(ctx->d_p2.ensure(bytes));
+    if (words > 0) {
+        const cudaMemcpyKind kind = is_device ? cudaMemcpyDeviceToDevice : cudaMemcpyHostToDevice;
+        CK(cudaMemcpyAsync(ctx->d_p1.p, p1, (size_t)n_pairs * words * 4, kind, ctx->stream));
+        CK(cudaMemcpyAsync(ctx->d_p2.p, p2, (size_t)n_pairs * words * 4, kind, ctx->stream));
+        CK(cudaStreamSynchronize(ctx->stream));
+    }
+    ctx->n_pairs = n_pairs;
+    ctx->words = words;
+    ctx->stim_set = true;
+    invalidate_sim(ctx);
+    return AVFS_OK;
+}
+
+avfs_status avfs_set_slot_range(avfs_ctx* ctx, int64_t first_slot, int64_t n_slots) {
+    CHECK_CTX();
+    if (first_slot < 0) return fail(ctx, AVFS_ERR_ARG, "negative first slot");
+    ctx->slot_first = first_slot;
+    ctx->slot_count = n_slots;
+    invalidate_sim(ctx);
+    return AVFS_OK;
+}
+
+avfs_status avfs_set_options(avfs_ctx* ctx, const avfs_options* o) {
+    CHECK_CTX();
+    if (!o) return fail(ctx, AVFS_ERR_ARG, "null options");
+    if (o->capacity < 1 || o->capacity > 1024) return fail(ctx, AVFS_ERR_ARG, "capacity must be in [1, 1024]");
+    if (o->quantum_ps < 0 || !std::isfinite(o->quantum_ps)) return fail(ctx, AVFS_ERR_ARG, "bad quantum");
+    if (o->n_probe < 0 || (o->n_probe > 0 && !o->probe_sig)) return fail(ctx, AVFS_ERR_ARG, "bad probes");
+    if (o->warps_per_cta < 0 || o->warps_per_cta > 16) return fail(ctx, AVFS_ERR_ARG, "warps_per_cta in [0,16]");
+    if (o->max_rerun_rounds < 0 || o->max_rerun_rounds > 6) return fail(ctx, AVFS_ERR_ARG, "max_rerun_rounds in [0,6]");
+    std::vector<int32_t> pr(o->probe_sig, o->probe_sig + o->n_probe);
+    if (ctx->net_loaded)
+        for (int32_t s : pr)
+            if (s < 0 || s >= ctx->n_pi + ctx->n_gates) return fail(ctx, AVFS_ERR_ARG, "probe %d out of range", s);
+    const bool plan_change = !ctx->plan_valid || o->keep_all != ctx->opt.keep_all || pr != ctx->probes;
+    ctx->opt = *o;
+    ctx->opt.probe_sig = nullptr;
+    ctx->probes = pr;
+    if (plan_change) ctx->plan_valid = false;
+    invalidate_sim(ctx);
+    return AVFS_OK;
+}
+
+avfs_status avfs_sync(avfs_ctx* ctx) {
+    CHECK_CTX();
+    if (!has_dev(ctx)) return AVFS_OK;
+    CK(cudaStreamSynchronize(ctx->stream));
+    return AVFS_OK;
+}
+
+static avfs_status run_round(avfs_ctx* ctx, Round& R, int round_idx, const int32_t* d_sw_list, int32_t prev_W,
+                             int32_t prev_cstage, bool timed) {
+    const int32_t S = ctx->n_pi + ctx->n_gates;
+    (void)S;
+    int wpc = ctx->opt.warps_per_cta > 0 ? ctx->opt.warps_per_cta : 8;
+    int smem = sweep_smem_bytes(wpc, ctx->kmax, R.W, R.cstage);
+    while (wpc > 1 && smem > 227 * 1024) smem = sweep_smem_bytes(--wpc, ctx->kmax, R.W, R.cstage);
+    if (smem > 227 * 1024) return fail(ctx, AVFS_ERR_CAPACITY, "capacity %d needs %d B shared memory per warp", R.capacity, smem);
+    int bps = 0;
+    CK(sweep_occupancy(wpc, smem, &bps));
+    if (bps < 1) return fail(ctx, AVFS_ERR_CAPACITY, "sweep kernel does not fit on an SM (smem %d)", smem);
+    R.grid = (int32_t)std::min<int64_t>(R.n_sw, (int64_t)ctx->n_sm * bps);
+    if (R.grid < 1) R.grid = 1;
+    if ((int)ctx->scr.size() <= round_idx) ctx->scr.resize(round_idx + 1);
+    if ((int)ctx->pin.size() <= round_idx) ctx->pin.resize(round_idx + 1);
+    const size_t scr_bytes = (size_t)std::max(ctx->n_scratch, 1) * R.grid * R.region_bytes;
+    const size_t pin_bytes = (size_t)std::max(ctx->n_pinned, 1) * R.n_sw * R.region_bytes;
+    CK(ctx->scr[round_idx].ensure(scr_bytes));
+    CK(ctx->pin[round_idx].ensure(pin_bytes));
+    CK(ctx->d_ovf.ensure(std::max<int64_t>(R.n_sw, 1) * sizeof(int32_t)));
+    CK(cudaMemsetAsync(ctx->d_ovf.p, 0, R.n_sw * sizeof(int32_t), ctx->stream));
+    SweepParams p{};
+    p.gates = ctx->d_gates.as<GateDesc>();
+    p.level_ptr = ctx->d_level_ptr.as<int32_t>();
+    p.depth = ctx->depth;
+    p.coef = ctx->d_coef.as<double>();
+    p.deg_v = ctx->deg_v;
+    p.vdd = ctx->d_vdd.as<double>();
+    p.v_min = ctx->v_min;
+    p.v_max = ctx->v_max;
+    p.quantum = ctx->opt.quantum_ps;
+    p.p1t = ctx->d_p1t.as<uint32_t>();
+    p.p2t = ctx->d_p2t.as<uint32_t>();
+    p.n_pw = (int32_t)((ctx->n_pairs + 31) / 32);
+    p.n_pairs = ctx->n_pairs;
+    p.n_vdd = (int32_t)ctx->vdd.size();
+    p.slot_first = ctx->sim_first;
+    p.slot_end = ctx->sim_end;
+    p.sw_list = d_sw_list;
+    p.sw_first = R.sw_first;
+    p.n_sw = R.n_sw;
+    p.scratch = ctx->scr[round_idx].as<uint8_t>();
+    p.pinned = ctx->pin[round_idx].as<uint8_t>();
+    p.region_bytes = R.region_bytes;
+    p.W = R.W;
+    p.cstage = R.cstage;
+    p.prev_W = prev_W;
+    p.prev_cstage = prev_cstage;
+    p.kmax = ctx->kmax;
+    p.act = ctx->d_act.as<unsigned long long>();
+    p.latest = ctx->d_latest.as<unsigned int>();
+    p.ovf = ctx->d_ovf.as<int32_t>();
+    p.err = ctx->d_err.as<int32_t>();
+    if (timed) CK(cudaEventRecord(ctx->ev0, ctx->stream));
+    CK(launch_sweep(p, R.grid, wpc, ctx->stream));
+    if (timed) CK(cudaEventRecord(ctx->ev1, ctx->stream));
+    ctx->stats.launches++;
+    if (round_idx == 0) ctx->stats.warps_per_cta = wpc;
+    return AVFS_OK;
+}
+
+avfs_status avfs_simulate(avfs_ctx* ctx, void* cuda_stream) {
+    CHECK_CTX();
+    if (!has_dev(ctx)) return fail(ctx, AVFS_ERR_STATE, "host-only context");
+    if (!ctx->net_loaded || !ctx->stim_set || ctx->vdd.empty())
+        return fail(ctx, AVFS_ERR_STATE, "netlist, stimuli and operating points must be set");
+    const auto t0 = std::chrono::steady_clock::now();
+    CK(cudaSetDevice(ctx->dev));
+    ctx->stream = static_cast<cudaStream_t>(cuda_stream);
+    avfs_status st = build_plan(ctx);
+    if (st != AVFS_OK) return st;
+    st = upload_netlist(ctx);
+    if (st != AVFS_OK) return st;
+    invalidate_sim(ctx);
+    const int64_t P = ctx->n_pairs;
+    const int32_t V = (int32_t)ctx->vdd.size();
+    const int64_t total = P * V;
+    const int64_t first = ctx->slot_first;
+    const int64_t end = ctx->slot_count < 0 ? total : std::min(total, first + ctx->slot_count);
+    if (first >= end) return fail(ctx, AVFS_ERR_ARG, "empty slot range [%lld, %lld)", (long long)first, (long long)end);
+    ctx->sim_first = first;
+    ctx->sim_end = end;
+    const int32_t n_pw = (int32_t)((P + 31) / 32);
+    const int64_t sw_lo = (first / P) * n_pw + (first % P) / 32;
+    const int64_t sw_hi = ((end - 1) / P) * n_pw + ((end - 1) % P) / 32 + 1;
+    const int32_t S = ctx->n_pi + ctx->n_gates;
+    std::memset(&ctx->stats, 0, sizeof ctx->stats);
+
+    CK(ctx->d_p1t.ensure((size_t)std::max(ctx->n_pi, 1) * n_pw * 4));
+    CK(ctx->d_p2t.ensure((size_t)std::max(ctx->n_pi, 1) * n_pw * 4));
+    CK(ctx->d_act.ensure((size_t)S * V * sizeof(unsigned long long)));
+    CK(ctx->d_latest.ensure((size_t)V * 4));
+    CK(ctx->d_err.ensure(16));
+    CK(ctx->d_count.ensure(16));
+    CK(cudaMemsetAsync(ctx->d_act.p, 0, (size_t)S * V * sizeof(unsigned long long), ctx->stream));
+    CK(cudaMemsetAsync(ctx->d_latest.p, 0, (size_t)V * 4, ctx->stream));
+    CK(cudaMemsetAsync(ctx->d_err.p, 0, 16, ctx->stream));
+    // H4: stimulus expansion (transpose to PI-major 32-pair words)
+    CK(launch_expand(ctx->d_p1.as<uint32_t>(), ctx->d_p2.as<uint32_t>(), P, ctx->words, ctx->n_pi, n_pw,
+                     ctx->d_p1t.as<uint32_t>(), ctx->d_p2t.as<uint32_t>(), ctx->stream));
+    CK(launch_pi_activity(ctx->d_p1t.as<uint32_t>(), ctx->d_p2t.as<uint32_t>(), ctx->n_pi, n_pw, P, V, first, end,
+                          ctx->d_act.as<unsigned long long>(), ctx->stream));
+    ctx->stats.launches += 2;
+
+    ctx->rounds.clear();
+    Round R0;
+    R0.n_sw = sw_hi - sw_lo;
+    R0.sw_first = sw_lo;
+    R0.capacity = ctx->opt.capacity;
+    R0.W = 32 * R0.capacity;
+    R0.cstage = 2 * R0.capacity;
+    R0.region_bytes = 128 + 4 * (int64_t)R0.W;
+    st = run_round(ctx, R0, 0, nullptr, 0, 0, ctx->opt.profile != 0);
+    if (st != AVFS_OK) return st;
+    ctx->rounds.push_back(R0);
+    int cur = 0;
+    for (int r = 0;; ++r) {
+        const Round& prev = ctx->rounds.back();
+        CK(ctx->d_list[cur].ensure(std::max<int64_t>(prev.n_sw, 1) * sizeof(int32_t)));
+        CK(cudaMemsetAsync(ctx->d_count.p, 0, 16, ctx->stream));
+        CK(launch_compact_overflow(ctx->d_ovf.as<int32_t>(), prev.n_sw,
+                                   r == 0 ? nullptr : ctx->d_list[cur ^ 1].as<int32_t>(), prev.sw_first,
+                                   ctx->d_list[cur].as<int32_t>(), ctx->d_count.as<int32_t>(), ctx->stream));
+        ctx->stats.launches++;
+        CK(cudaMemcpyAsync(ctx->h_pinned, ctx->d_count.p, 4, cudaMemcpyDeviceToHost, ctx->stream));
+        CK(cudaMemcpyAsync(ctx->h_pinned + 1, ctx->d_err.p, 4, cudaMemcpyDeviceToHost, ctx->stream));
+        CK(cudaStreamSynchronize(ctx->stream));
+        if (ctx->h_pinned[1] & 1)
+            return fail(ctx, AVFS_ERR_DELAY_NONPOS, "a delay d' = d_nom (1 + f(P)) evaluated to <= 0");
+        const int32_t n_ovf = ctx->h_pinned[0];
+        if (n_ovf == 0) break;
+        if (r >= ctx->opt.max_rerun_rounds)
+            return fail(ctx, AVFS_ERR_CAPACITY, "%d slot groups still overflow at capacity %d after %d reruns",
+                        n_ovf, prev.capacity, r);
+        Round Rn;
+        Rn.n_sw = n_ovf;
+        Rn.sws.resize(n_ovf);
+        CK(cudaMemcpy(Rn.sws.data(), ctx->d_list[cur].p, n_ovf * sizeof(int32_t), cudaMemcpyDeviceToHost));
+        Rn.capacity = std::min(prev.capacity * 4, 1024);
+        Rn.W = 32 * Rn.capacity;
+        Rn.cstage = 2 * Rn.capacity;
+        Rn.region_bytes = 128 + 4 * (int64_t)Rn.W;
+        ctx->stats.overflow_slot_warps += n_ovf;
+        ctx->stats.rerun_rounds++;
+        st = run_round(ctx, Rn, r + 1, ctx->d_list[cur].as<int32_t>(), prev.W, prev.cstage, false);
+        if (st != AVFS_OK) return st;
+        ctx->rounds.push_back(std::move(Rn));
+        cur ^= 1;
+    }
+    if (ctx->opt.profile) {
+        float ms = 0;
+        CK(cudaEventElapsedTime(&ms, ctx->ev0, ctx->ev1));
+        ctx->stats.sweep_ms = ms;
+    }
+    ctx->sim_done = true;
+    ctx->stats.slots = end - first;
+    ctx->stats.evals = (int64_t)ctx->n_gates * (end - first);
+    ctx->stats.slot_warps = sw_hi - sw_lo;
+    ctx->stats.grid = ctx->rounds[0].grid;
+    ctx->stats.n_scratch_buffers = ctx->n_scratch;
+    ctx->stats.n_pinned = ctx->n_pinned;
+    int64_t ab = 0;
+    for (size_t r = 0; r < ctx->rounds.size(); ++r) ab += (int64_t)(ctx->scr[r].n + ctx->pin[r].n);
+    ctx->stats.arena_bytes = ab;
+    ctx->stats.sim_ms = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+    return AVFS_OK;
+}
+
+avfs_status avfs_get_activity(avfs_ctx* ctx, uint64_t* out, int32_t out_is_device) {
+    CHECK_CTX();
+    if (!out) return fail(ctx, AVFS_ERR_ARG, "null output");
+    if (!ctx->sim_done) return fail(ctx, AVFS_ERR_STATE, "simulate first");
+    const size_t n = (size_t)(ctx->n_pi + ctx->n_gates) * ctx->vdd.size() * sizeof(uint64_t);
+    CK(cudaMemcpyAsync(out, ctx->d_act.p, n, out_is_device ? cudaMemcpyDeviceToDevice : cudaMemcpyDeviceToHost,
+                       ctx->stream));
+    CK(cudaStreamSynchronize(ctx->stream));
+    return AVFS_OK;
+}
+
+avfs_status avfs_get_latest_arrival(avfs_ctx* ctx, float* out) {
+    CHECK_CTX();
+    if (!out) return fail(ctx, AVFS_ERR_ARG, "null output");
+    if (!ctx->sim_done) return fail(ctx, AVFS_ERR_STATE, "simulate first");
+    CK(cudaMemcpyAsync(out, ctx->d_latest.p, ctx->vdd.size() * 4, cudaMemcpyDeviceToHost, ctx->stream));
+    CK(cudaStreamSynchronize(ctx->stream));
+    return AVFS_OK;
+}
+
+static avfs_status gather(avfs_ctx* ctx, int32_t n_sig, const int32_t* sig, int64_t slot0, int64_t n_slots,
+                          int32_t cap, uint8_t* init, int32_t* count, float* times) {
+    if (!ctx->sim_done) return fail(ctx, AVFS_ERR_STATE, "simulate first");
+    if (n_sig < 0 || n_slots < 0 || cap < 0 || (n_sig > 0 && !sig)) return fail(ctx, AVFS_ERR_ARG, "bad readback arguments");
+    if (slot0 < ctx->sim_first || slot0 + n_slots > ctx->sim_end)
+        return fail(ctx, AVFS_ERR_ARG, "slots [%lld, %lld) outside the simulated range [%lld, %lld)",
+                    (long long)slot0, (long long)(slot0 + n_slots), (long long)ctx->sim_first, (long long)ctx->sim_end);
+    if (ctx->rounds.size() > 8) return fail(ctx, AVFS_ERR_STATE, "too many rounds");
+    std::vector<uint32_t> sl(n_sig);
+    for (int32_t i = 0; i < n_sig; ++i) {
+        if (sig[i] < 0 || sig[i] >= ctx->n_pi + ctx->n_gates) return fail(ctx, AVFS_ERR_ARG, "signal %d out of range", sig[i]);
+        sl[i] = ctx->loc[sig[i]];
+        if ((sl[i] & LOC_KIND) == LOC_SCRATCH)
+            return fail(ctx, AVFS_ERR_ARG, "signal %d is not kept (not a PO/probe; use keep_all)", sig[i]);
+    }
+    if (n_sig == 0 || n_slots == 0) return AVFS_OK;
+    const int32_t n_pw = (int32_t)((ctx->n_pairs + 31) / 32);
+    const int64_t n_sw_total = (int64_t)n_pw * ctx->vdd.size();
+    if (!ctx->map_valid) {
+        std::vector<int32_t> rnd(n_sw_total, -1), idx(n_sw_total, 0);
+        for (size_t r = 0; r < ctx->rounds.size(); ++r) {
+            const Round& R = ctx->rounds[r];
+            for (int64_t i = 0; i < R.n_sw; ++i) {
+                const int64_t sw = R.sws.empty() ? R.sw_first + i : R.sws[i];
+                rnd[sw] = (int32_t)r;
+                idx[sw] = (int32_t)i;
+            }
+        }
+        CK(ctx->d_swround.ensure(n_sw_total * 4));
+        CK(ctx->d_swindex.ensure(n_sw_total * 4));
+        CK(cudaMemcpy(ctx->d_swround.p, rnd.data(), n_sw_total * 4, cudaMemcpyHostToDevice));
+        CK(cudaMemcpy(ctx->d_swindex.p, idx.data(), n_sw_total * 4, cudaMemcpyHostToDevice));
+        ctx->map_valid = true;
+    }
+    const size_t n = (size_t)n_sig * n_slots;
+    CK(ctx->g_loc.ensure(n_sig * 4));
+    CK(ctx->g_init.ensure(n));
+    CK(ctx->g_count.ensure(n * 4));
+    if (times) CK(ctx->g_times.ensure(std::max<size_t>(n * cap * 4, 4)));
+    CK(ctx->g_bad.ensure(4));
+    CK(cudaMemcpy(ctx->g_loc.p, sl.data(), n_sig * 4, cudaMemcpyHostToDevice));
+    CK(cudaMemsetAsync(ctx->g_bad.p, 0, 4, ctx->stream));
+    GatherParams g{};
+    g.sig_loc = ctx->g_loc.as<uint32_t>();
+    g.n_sig = n_sig;
+    g.slot0 = slot0;
+    g.n_slots = n_slots;
+    g.n_pairs = ctx->n_pairs;
+    g.n_pw = n_pw;
+    g.p1t = ctx->d_p1t.as<uint32_t>();
+    g.p2t = ctx->d_p2t.as<uint32_t>();
+    g.sw_round = ctx->d_swround.as<int32_t>();
+    g.sw_index = ctx->d_swindex.as<int32_t>();
+    for (size_t r = 0; r < ctx->rounds.size(); ++r)
+        g.rounds[r] = GatherRound{ctx->pin[r].as<uint8_t>(), ctx->rounds[r].region_bytes, ctx->rounds[r].n_sw};
+    g.cap = times ? cap : 0;
+    g.init = ctx->g_init.as<uint8_t>();
+    g.count = ctx->g_count.as<int32_t>();
+    g.times = times ? ctx->g_times.as<float>() : nullptr;
+    g.bad = ctx->g_bad.as<int32_t>();
+    CK(launch_gather(g, ctx->stream));
+    int32_t bad = 0;
+    CK(cudaMemcpyAsync(&bad, ctx->g_bad.p, 4, cudaMemcpyDeviceToHost, ctx->stream));
+    if (init) CK(cudaMemcpyAsync(init, ctx->g_init.p, n, cudaMemcpyDeviceToHost, ctx->stream));
+    if (count) CK(cudaMemcpyAsync(count, ctx->g_count.p, n * 4, cudaMemcpyDeviceToHost, ctx->stream));
+    if (times && cap > 0) CK(cudaMemcpyAsync(times, ctx->g_times.p, n * cap * 4, cudaMemcpyDeviceToHost, ctx->stream));
+    CK(cudaStreamSynchronize(ctx->stream));
+    if (bad) return fail(ctx, AVFS_ERR_STATE, "readback hit slots without valid data (code %d)", bad);
+    return AVFS_OK;
+}
+
+avfs_status avfs_get_final_values(avfs_ctx* ctx, int32_t n_sig, const int32_t* sig, int64_t slot0,
+                                  int64_t n_slots, uint8_t* out) {
+    CHECK_CTX();
+    if (!out) return fail(ctx, AVFS_ERR_ARG, "null output");
+    const size_t n = (size_t)std::max(n_sig, 0) * std::max<int64_t>(n_slots, 0);
+    std::vector<uint8_t> init(n);
+    std::vector<int32_t> cnt(n);
+    avfs_status st = gather(ctx, n_sig, sig, slot0, n_slots, 0, init.data(), cnt.data(), nullptr);
+    if (st != AVFS_OK) return st;
+    for (size_t i = 0; i < n; ++i) out[i] = (uint8_t)(init[i] ^ (cnt[i] & 1));
+    return AVFS_OK;
+}
+
+avfs_status avfs_get_waveforms(avfs_ctx* ctx, int32_t n_sig, const int32_t* sig, int64_t slot0, int64_t n_slots,
+                               int32_t cap, uint8_t* init, int32_t* count, float* times) {
+    CHECK_CTX();
+    if (!init || !count || (cap > 0 && !times)) return fail(ctx, AVFS_ERR_ARG, "null output");
+    return gather(ctx, n_sig, sig, slot0, n_slots, cap, init, count, cap > 0 ? times : nullptr);
+}
+
+avfs_status avfs_get_stats(avfs_ctx* ctx, avfs_stats* st) {
+    CHECK_CTX();
+    if (!st) return fail(ctx, AVFS_ERR_ARG, "null output");
+    if (!ctx->sim_done) return fail(ctx, AVFS_ERR_STATE, "simulate first");
+    // algorithmic bytes of the sweep: every gate output
+    // is written once and read once per reading pin, 4 B header per slot plus
+    // 4 B per transition; PI words: 8 B per 32 slots per reading pin.
+    const int32_t V = (int32_t)ctx->vdd.size();
+    const int32_t S = ctx->n_pi + ctx->n_gates;
+    std::vector<uint64_t> act((size_t)S * V);
+    CK(cudaMemcpy(act.data(), ctx->d_act.p, act.size() * 8, cudaMemcpyDeviceToHost));
+    const double slots = (double)(ctx->sim_end - ctx->sim_first);
+    double b = 0;
+    for (int32_t s = ctx->n_pi; s < S; ++s) {
+        uint64_t a = 0;
+        for (int32_t k = 0; k < V; ++k) a += act[(size_t)s * V + k];
+        b += (1.0 + (double)ctx->fanout[s]) * (4.0 * slots + 4.0 * (double)a);
+    }
+    for (int32_t i = 0; i < ctx->n_pi; ++i) b += (double)ctx->fanout[i] * slots / 4.0;
+    ctx->stats.alg_bytes = (int64_t)b;
+    *st = ctx->stats;
+    return AVFS_OK;
+}
+
+}  // extern "C"

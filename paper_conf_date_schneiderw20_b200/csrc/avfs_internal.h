@@ -1,0 +1,111 @@
+// avfs_internal.h -- structures shared by the host runtime (avfs_host.cpp)
+// and the sm_100a kernels (avfs_kernels.cu).  Not part of the C-ABI.
+#pragma once
+#include <cstdint>
+#include <cuda_runtime.h>
+
+namespace avfs {
+
+constexpr int KMAX = 4;            // max cell inputs (truth table is 16 bits)
+constexpr int MAX_DEG = 7;         // max polynomial degree per variable
+
+// Location code of a waveform: kind in bits 30..31.
+constexpr uint32_t LOC_PI = 0u << 30;        // low bits: PI index (waveform derived from stimuli)
+constexpr uint32_t LOC_SCRATCH = 1u << 30;   // low bits: scratch buffer id (liveness-coloured)
+constexpr uint32_t LOC_PINNED = 2u << 30;    // low bits: pinned id (PO / probe / keep_all)
+constexpr uint32_t LOC_KIND = 3u << 30;
+constexpr uint32_t LOC_ID = ~LOC_KIND;
+
+// Header word of one (signal, slot) waveform (reading C1):
+constexpr uint32_t HDR_N = 0x000FFFFFu;      // transition count (exact, even on overflow)
+constexpr uint32_t HDR_INIT = 1u << 20;      // value before t = 0
+constexpr uint32_t HDR_POISON = 1u << 21;    // events not stored here or upstream
+constexpr uint32_t HDR_PREV = 1u << 22;      // would have been poisoned at the previous round's capacity
+
+// Gate descriptor, 96 B, read warp-uniformly (P:L154 step 1).
+struct alignas(16) GateDesc {
+    uint32_t in_loc[KMAX];
+    uint32_t out_loc;
+    uint32_t sig;        // output signal id (activity row)
+    uint16_t tt;         // truth table
+    uint8_t k;           // number of inputs
+    uint8_t flags;       // bit 0: drives a primary output (latest arrival)
+    uint32_t coef_off;   // offset (doubles) of [pin][pol][deg_v+1] coefficient block
+    double dnom[2 * KMAX];   // [pin][pol] nominal delay, ps
+};
+static_assert(sizeof(GateDesc) == 96, "GateDesc layout");
+
+// One slot-warp region: 32 header words followed by W = 32*C event times
+// (compact: lane l's events start at the exclusive prefix sum of the counts).
+struct SweepParams {
+    const GateDesc* __restrict__ gates;     // sorted by level
+    const int32_t* __restrict__ level_ptr;  // [depth+1] offsets into gates (level 1..depth)
+    int32_t depth;
+    const double* __restrict__ coef;        // coefficient blocks
+    int32_t deg_v;
+    const double* __restrict__ vdd;         // [n_vdd] volts
+    double v_min, v_max;
+    double quantum;                         // 0: F mode
+    const uint32_t* __restrict__ p1t;       // [n_pi][n_pw] bit-transposed stimuli
+    const uint32_t* __restrict__ p2t;
+    int32_t n_pw;                           // pair-warps (ceil(n_pairs/32))
+    int64_t n_pairs;
+    int32_t n_vdd;
+    int64_t slot_first, slot_end;           // public slot range simulated
+    // slot-warps of this run: sw = sw_list ? sw_list[i] : sw_first + i, i < n_sw
+    const int32_t* __restrict__ sw_list;
+    int64_t sw_first;
+    int64_t n_sw;
+    // arenas
+    uint8_t* scratch;                       // [n_scratch][gridDim.x][region]
+    uint8_t* pinned;                        // [n_pinned][n_sw][region]
+    int64_t region_bytes;
+    int32_t W;                              // event capacity per region (32*C)
+    int32_t cstage;                         // per-slot capacity (2*C)
+    int32_t prev_W, prev_cstage;            // previous round (0: first pass)
+    int32_t kmax;                           // max fan-in in the netlist (smem sizing)
+    // outputs
+    unsigned long long* act;                // [n_signals][n_vdd]
+    unsigned int* latest;                   // [n_vdd] float bits (non-negative)
+    int32_t* ovf;                           // [n_sw] overflow flag per slot-warp
+    int32_t* err;                           // bit 0: non-positive delay
+};
+
+// launch wrappers (avfs_kernels.cu)
+int sweep_smem_bytes(int warps_per_cta, int kmax, int W, int cstage);
+cudaError_t sweep_occupancy(int warps_per_cta, int smem, int* blocks_per_sm);
+cudaError_t launch_sweep(const SweepParams& p, int grid, int warps_per_cta, cudaStream_t st);
+cudaError_t launch_expand(const uint32_t* p1, const uint32_t* p2, int64_t n_pairs, int32_t words,
+                          int32_t n_pi, int32_t n_pw, uint32_t* p1t, uint32_t* p2t, cudaStream_t st);
+cudaError_t launch_pi_activity(const uint32_t* p1t, const uint32_t* p2t, int32_t n_pi, int32_t n_pw,
+                               int64_t n_pairs, int32_t n_vdd, int64_t slot_first, int64_t slot_end,
+                               unsigned long long* act, cudaStream_t st);
+cudaError_t launch_compact_overflow(const int32_t* ovf, int64_t n_sw, const int32_t* sw_list,
+                                    int64_t sw_first, int32_t* out_list, int32_t* out_count,
+                                    cudaStream_t st);
+
+struct GatherRound {       // one simulated round for readback
+    const uint8_t* pinned;
+    int64_t region_bytes;
+    int64_t n_sw;
+};
+struct GatherParams {
+    const uint32_t* sig_loc;    // [n_sig] location codes (PI or pinned)
+    int32_t n_sig;
+    int64_t slot0, n_slots;
+    int64_t n_pairs;
+    int32_t n_pw;
+    const uint32_t* p1t;
+    const uint32_t* p2t;
+    const int32_t* sw_round;    // [n_sw_total] round index holding the final data (-1: not simulated)
+    const int32_t* sw_index;    // [n_sw_total] index within that round
+    GatherRound rounds[8];
+    int32_t cap;
+    uint8_t* init;
+    int32_t* count;
+    float* times;
+    int32_t* bad;               // set when a requested slot was not simulated / still poisoned
+};
+cudaError_t launch_gather(const GatherParams& p, cudaStream_t st);
+
+}  // namespace avfs

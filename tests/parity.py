@@ -1,0 +1,65 @@
+"""Parity helpers: run the CUDA path through the C-ABI and the oracle on the
+same seeded inputs and compare element by element.
+
+Bar (north_star / DESIGN.md):
+  * transition counts, initial and final values: bit-exact
+    (F mode: on the (signal, slot) pairs the oracle does not taint -- reading C13)
+  * transition times: Q mode bit-exact; F mode |t_gpu - t_ref| <= 1e-5 |t_ref| + 1e-3 ps
+  * activity: exact per (signal, Vdd) wherever no contributing slot is tainted
+"""
+from __future__ import annotations
+
+import numpy as np
+
+Q = 2.0 ** -8
+REL, ABS = 1e-5, 1e-3
+
+
+def gpu_run(w_or_parts, quantum=0.0, capacity=None, keep_all=True, probes=None, slot_range=None,
+            stream=None, warps_per_cta=0, max_rerun_rounds=3, netlist=None):
+    from paper_conf_date_schneiderw20_b200 import Context, load_workload
+    nl = netlist if netlist is not None else w_or_parts.netlist
+    ctx = Context(0)
+    load_workload(ctx, nl, w_or_parts.library, w_or_parts.stimuli, w_or_parts.vdd)
+    ctx.set_options(capacity=capacity or w_or_parts.capacity, quantum_ps=quantum, keep_all=keep_all,
+                    probes=probes, warps_per_cta=warps_per_cta, max_rerun_rounds=max_rerun_rounds,
+                    profile=True)
+    if slot_range is not None:
+        ctx.set_slot_range(*slot_range)
+    ctx.simulate(stream)
+    return ctx
+
+
+def gpu_waveforms(ctx, sig, slots_first, n_slots, cap):
+    init, cnt, times = ctx.waveforms(np.asarray(sig, np.int32), slots_first, n_slots, cap=cap)
+    # -> [slot][sig] like the oracle
+    return init.T.copy(), cnt.T.copy(), times.transpose(1, 0, 2).copy()
+
+
+def compare(ref, init, cnt, times, quantum, label=""):
+    """ref: OracleResult with the same [slot][sig] layout.  Returns stats dict."""
+    ok = ref.taint == 0
+    assert np.array_equal(init, ref.init), f"{label}: init values differ"
+    bad = (cnt != ref.count) & ok
+    assert not bad.any(), f"{label}: {bad.sum()} untainted counts differ, first at {np.argwhere(bad)[:5]}"
+    cap = min(times.shape[2], ref.times.shape[2])
+    m = (np.arange(cap)[None, None, :] < np.minimum(cnt, ref.count)[:, :, None]) & ok[:, :, None]
+    gt = times[:, :, :cap][m].astype(np.float64)
+    rt = ref.times[:, :, :cap][m]
+    if quantum > 0:
+        assert np.array_equal(gt, rt), f"{label}: Q-mode times not bit-exact ({np.abs(gt - rt).max()})"
+        maxerr = 0.0
+    else:
+        err = np.abs(gt - rt)
+        tol = REL * np.abs(rt) + ABS
+        assert np.all(err <= tol), f"{label}: F-mode time error {err.max()} > tol"
+        maxerr = float(err.max()) if err.size else 0.0
+    return {"pairs": int(ok.size), "tainted": int((~ok).sum()), "events": int(m.sum()),
+            "max_time_err": maxerr, "flags": ref.flags}
+
+
+def activity_ref(ref, n_vdd, n_signals):
+    """[n_signals][n_vdd] sums of oracle counts over Vdd-major slots; mask of untainted rows."""
+    c = ref.count.reshape(n_vdd, -1, n_signals)
+    t = ref.taint.reshape(n_vdd, -1, n_signals)
+    return c.sum(1).T.astype(np.int64), (t.sum(1).T == 0)

@@ -1,0 +1,80 @@
+"""Parity at BASELINE.json's full sizes, in bench.py's launch configuration
+(F mode, default capacity, POs kept), on sampled slots the oracle computes
+one by one (-m gpu).
+
+For each config: (1) the full-size run's PO waveforms at sampled slots equal
+the oracle's (untainted pairs bit-exact counts, times within tolerance);
+(2) a run restricted to a 64-slot window (the multi-GPU shard mechanism)
+has activity equal to the oracle's per-signal sums over that window.
+"""
+import numpy as np
+import pytest
+
+import oracle
+from workloads import make_config
+from tests.parity import gpu_run, gpu_waveforms, compare, activity_ref
+
+pytestmark = pytest.mark.gpu
+
+SAMPLES = {2: 64, 3: 48, 4: 32, 5: 6}
+
+
+def sample_slots(w, n):
+    P, V = w.stimuli.n_pairs, len(w.vdd)
+    rng = np.random.default_rng(w.cfg)
+    s = np.sort(rng.choice(P * V, size=n, replace=False))
+    return s
+
+
+@pytest.mark.parametrize("cfg", [2, 3, 4, pytest.param(5, marks=pytest.mark.slow)])
+def test_fullsize_sampled_po_parity(cfg):
+    w = make_config(cfg)
+    nl = w.netlist
+    ctx = gpu_run(w, keep_all=False)
+    st = ctx.stats()
+    assert st["evals"] == w.evals
+    slots = sample_slots(w, SAMPLES[cfg])
+    P = w.stimuli.n_pairs
+    ref = oracle.simulate(nl, w.library, w.stimuli, w.vdd, slots % P, slots // P, quantum=0.0,
+                          cap=64, out_sig=nl.po_sig)
+    cap = max(1, min(64, int(ref.count.max())))
+    init = np.zeros((len(slots), len(nl.po_sig)), np.uint8)
+    cnt = np.zeros((len(slots), len(nl.po_sig)), np.int32)
+    times = np.zeros((len(slots), len(nl.po_sig), cap), np.float32)
+    for i, s in enumerate(slots):
+        a, b, c = gpu_waveforms(ctx, nl.po_sig, int(s), 1, cap)
+        init[i], cnt[i], times[i] = a[0], b[0], c[0]
+    ref.times = ref.times[:, :, :cap]
+    r = compare(ref, init, cnt, np.minimum(times, np.float32(3e38)), 0.0, f"cfg{cfg}")
+    assert r["events"] > 0
+    # latest arrival bounds the sampled PO transitions
+    lat = ctx.latest_arrival()
+    k = slots // P
+    last = np.where(cnt > 0, np.take_along_axis(times, np.clip(cnt - 1, 0, cap - 1)[:, :, None], 2)[:, :, 0], 0)
+    assert np.all(last.max(1) <= lat[k] + 1e-6)
+    ctx.close()
+
+
+@pytest.mark.parametrize("cfg", [2, 3, 4])
+def test_fullsize_window_activity(cfg):
+    w = make_config(cfg)
+    nl = w.netlist
+    P, V = w.stimuli.n_pairs, len(w.vdd)
+    first = (P * V) // 2 + 7
+    n = 64
+    ctx = gpu_run(w, keep_all=False, slot_range=(first, n))
+    act = ctx.activity().astype(np.int64)
+    slots = np.arange(first, first + n)
+    ref = oracle.simulate(nl, w.library, w.stimuli, w.vdd, slots % P, slots // P, quantum=0.0, cap=0)
+    cnt = ref.count.sum(0)
+    k = slots // P
+    for kv in np.unique(k):
+        sel = k == kv
+        ok = ref.taint[sel].sum(0) == 0
+        got = act[:, kv]
+        want = ref.count[sel].sum(0)
+        assert np.array_equal(got[ok], want[ok]), f"cfg{cfg} vdd{kv}"
+    others = np.setdiff1d(np.arange(V), np.unique(k))
+    assert np.all(act[:, others] == 0)
+    assert cnt.sum() > 0
+    ctx.close()

@@ -1,0 +1,243 @@
+"""GPU <-> oracle parity through the C-ABI (-m gpu).
+
+Small cases compare every (signal, slot); they span several 32-slot groups,
+ragged pair counts (not multiples of 32), 1..4-input cells, dangling gates,
+overflow reruns and slot-range shards.
+"""
+import numpy as np
+import pytest
+
+import oracle
+from workloads import make_config, make_library, make_stimuli, random_dag, exhaustive_pairs, c17
+from workloads.configs import Workload
+from workloads.netlists import _Builder
+from tests.parity import Q, gpu_run, gpu_waveforms, compare, activity_ref
+
+pytestmark = pytest.mark.gpu
+
+
+def full_compare(w, quantum, capacity=None, cap=None, label="", **kw):
+    nl = w.netlist
+    j, k = oracle.all_slots(w.stimuli.n_pairs, len(w.vdd))
+    ref = oracle.simulate(nl, w.library, w.stimuli, w.vdd, j, k, quantum=quantum, cap=cap or 64)
+    cap = cap or max(1, int(ref.count.max()))
+    ctx = gpu_run(w, quantum=quantum, capacity=capacity, **kw)
+    sig = np.arange(nl.n_signals, dtype=np.int32)
+    init, cnt, times = gpu_waveforms(ctx, sig, 0, len(j), cap)
+    st = compare(ref, init, cnt, times, quantum, label)
+    act = ctx.activity().astype(np.int64)
+    ra, ok = activity_ref(ref, len(w.vdd), nl.n_signals)
+    assert np.array_equal(act[ok], ra[ok]), f"{label}: activity differs"
+    lat = ctx.latest_arrival()
+    if quantum > 0:
+        po = nl.po_sig
+        n = ref.count[:, po]
+        last = np.take_along_axis(ref.times[:, po, :], np.maximum(n - 1, 0)[:, :, None], 2)[:, :, 0]
+        last = np.where(n > 0, last, 0.0).reshape(len(w.vdd), -1).max(1)
+        assert np.array_equal(lat.astype(np.float64), last), f"{label}: latest arrival differs"
+    st["stats"] = ctx.stats()
+    ctx.close()
+    return st
+
+
+@pytest.mark.parametrize("quantum", [Q, 0.0])
+def test_c17_config1(quantum):
+    st = full_compare(make_config(1), quantum, label="c17")
+    assert st["events"] > 0
+
+
+@pytest.mark.parametrize("quantum", [Q, 0.0])
+def test_c17_exhaustive_1024_pairs(quantum):
+    w = make_config(1)
+    w.stimuli = exhaustive_pairs(5)
+    full_compare(w, quantum, label="c17-exh")
+
+
+@pytest.mark.parametrize("quantum", [Q, 0.0])
+def test_multiplier_ragged(quantum):
+    w = make_config(2, n_pairs=100, n_vdd=3)
+    st = full_compare(w, quantum, capacity=32, label="mult")
+    assert st["events"] > 10000
+
+
+@pytest.mark.parametrize("quantum", [Q, 0.0])
+def test_random_dag_four_input_cells(quantum):
+    mix = {"NAND2": .2, "NOR2": .1, "XOR2": .1, "INV": .15, "BUF": .05, "AOI21": .1, "OAI21": .1,
+           "NAND4": .05, "NOR4": .05, "AOI22": .05, "OAI22": .05}
+    nl = random_dag(4242, 3000, 64, 25, mix=mix)
+    w = Workload(0, "rdag4", nl, make_library(77, deg_v=3), make_stimuli(78, nl.n_pi, 200),
+                 np.array([0.6, 0.75, 0.9, 1.1]), 8)
+    full_compare(w, quantum, label="rdag4")
+
+
+def test_deg_c_folded_polynomial_q_mode():
+    """Full 2-D (v, c) polynomial (Eq. 4) with load folding: bit-exact in Q mode."""
+    nl = random_dag(99, 1500, 40, 18)
+    w = Workload(0, "rdag-2d", nl, make_library(98, deg_v=3, deg_c=3), make_stimuli(97, nl.n_pi, 64),
+                 np.array([0.62, 0.8, 1.05]), 8)
+    full_compare(w, Q, label="2d")
+
+
+@pytest.mark.parametrize("quantum", [Q, 0.0])
+def test_overflow_reruns_equal_large_capacity(quantum):
+    """Capacity 1 forces reruns (1 -> 4 -> 16 -> 64); results equal capacity 64 and the oracle."""
+    w = make_config(2, n_pairs=64, n_vdd=2)
+    st = full_compare(w, quantum, capacity=1, label="cap1")
+    assert st["stats"]["rerun_rounds"] >= 2 and st["stats"]["overflow_slot_warps"] > 0
+    full_compare(w, quantum, capacity=64, label="cap64")
+
+
+def test_overflow_exact_across_runs():
+    w = make_config(2, n_pairs=96, n_vdd=2)
+    sig = np.arange(w.netlist.n_signals, dtype=np.int32)
+    out = []
+    for cap in (2, 64):
+        ctx = gpu_run(w, quantum=0.0, capacity=cap)
+        out.append((ctx.activity(), ctx.latest_arrival(), *ctx.waveforms(sig, 0, 192, cap=48)))
+        ctx.close()
+    for a, b in zip(out[0], out[1]):
+        assert np.array_equal(a, b)
+
+
+def test_capacity_exhausted_reports_error():
+    from paper_conf_date_schneiderw20_b200 import AvfsError
+    w = make_config(2, n_pairs=32, n_vdd=1)
+    with pytest.raises(AvfsError) as e:
+        gpu_run(w, capacity=1, max_rerun_rounds=0)
+    assert e.value.status == 7
+
+
+def test_determinism_bitwise():
+    w = make_config(3, n_pairs=64, n_vdd=2, scale=0.1)
+    runs = []
+    for _ in range(2):
+        ctx = gpu_run(w, keep_all=False)
+        runs.append((ctx.activity(), ctx.latest_arrival(),
+                     *ctx.waveforms(w.netlist.po_sig, 0, 128, cap=16)))
+        ctx.close()
+    for a, b in zip(*runs):
+        assert np.array_equal(a, b)
+
+
+def test_slot_range_shards_sum_to_full():
+    """Disjoint slot ranges (the multi-GPU shards) reproduce the full run exactly."""
+    from paper_conf_date_schneiderw20_b200 import shard_range
+    w = make_config(3, n_pairs=150, n_vdd=3, scale=0.05)
+    total = w.n_slots
+    full = gpu_run(w, keep_all=False)
+    act_full, lat_full = full.activity(), full.latest_arrival()
+    po = w.netlist.po_sig
+    wf_full = full.waveforms(po, 0, total, cap=16)
+    full.close()
+    acc = np.zeros_like(act_full)
+    lat = np.zeros_like(lat_full)
+    for r in range(3):
+        first, n = shard_range(total, r, 3)
+        ctx = gpu_run(w, keep_all=False, slot_range=(first, n))
+        acc += ctx.activity()
+        lat = np.maximum(lat, ctx.latest_arrival())
+        wf = ctx.waveforms(po, first, n, cap=16)
+        for a, b in zip(wf, wf_full):
+            assert np.array_equal(a, b[:, first:first + n])
+        ctx.close()
+    assert np.array_equal(acc, act_full)
+    assert np.array_equal(lat, lat_full)
+
+
+def test_permuted_gate_order_same_results():
+    w = make_config(3, n_pairs=64, n_vdd=2, scale=0.05)
+    perm = w.netlist.permuted(5)
+    a = gpu_run(w, keep_all=True)
+    b = gpu_run(w, keep_all=True, netlist=perm)
+    G = w.netlist.n_gates
+    n_pi = w.netlist.n_pi
+    new_of_old = np.empty(G, np.int64)
+    new_of_old[perm.meta["gate_perm"]] = np.arange(G)
+    sig_old = np.arange(n_pi + G)
+    sig_new = np.concatenate([np.arange(n_pi), n_pi + new_of_old])
+    wa = a.waveforms(sig_old, 0, 128, cap=16)
+    wb = b.waveforms(sig_new, 0, 128, cap=16)
+    for x, y in zip(wa, wb):
+        assert np.array_equal(x, y)
+    assert np.array_equal(a.activity(), b.activity()[sig_new])
+
+
+def test_bench_text_path_equals_array_path():
+    from paper_conf_date_schneiderw20_b200 import Context
+    from workloads import c17_bench_text
+    w = make_config(1)
+    a = gpu_run(w)
+    ctx = Context(0)
+    lib = w.library
+    ctx.load_library(lib.names, lib.n_inputs, lib.tt, lib.deg_v, lib.deg_c, lib.beta)
+    ctx.load_bench(c17_bench_text(), w.netlist.d_nom)
+    ctx.set_operating_points(w.vdd)
+    ctx.set_stimuli(w.stimuli.p1, w.stimuli.p2)
+    ctx.set_options(capacity=8, keep_all=True)
+    ctx.simulate()
+    sig = np.arange(11, dtype=np.int32)
+    for x, y in zip(a.waveforms(sig, 0, 96, cap=8), ctx.waveforms(sig, 0, 96, cap=8)):
+        assert np.array_equal(x, y)
+    assert ctx.find_signal("22") == 9
+
+
+def test_edge_cases_single_pair_dup_inputs_pi_po_dangling():
+    b = _Builder(3)
+    g0 = b.gate("NAND2", 0, 0)          # duplicate input signal
+    g1 = b.gate("XOR2", g0, 1)
+    g2 = b.gate("INV", g1)               # dangling (no reader, not PO)
+    g3 = b.gate("AOI21", g1, 2, 0)
+    nl = b.build("edge", [g3, 2])        # PI 2 is also a PO
+    nl.d_nom = np.random.default_rng(1).uniform(2, 8, size=(nl.n_edges, 2))
+    nl.c_load = np.ones(nl.n_gates)
+    for P in (1, 33):
+        w = Workload(0, "edge", nl, make_library(3, deg_v=2), make_stimuli(4, 3, P), np.array([0.7, 1.0]), 4)
+        full_compare(w, Q, label=f"edge{P}")
+        full_compare(w, 0.0, label=f"edge{P}")
+
+
+def test_nonpositive_delay_reported():
+    from paper_conf_date_schneiderw20_b200 import AvfsError
+    w = make_config(1)
+    w.library = make_library(0, deg_v=1, const=-2.0)     # d' = -d_nom
+    with pytest.raises(AvfsError) as e:
+        gpu_run(w)
+    assert e.value.status == 6
+
+
+def test_api_errors_and_state():
+    from paper_conf_date_schneiderw20_b200 import Context, AvfsError
+    ctx = Context(0)
+    with pytest.raises(AvfsError) as e:
+        ctx.simulate()
+    assert e.value.status == 3
+    w = make_config(1)
+    from paper_conf_date_schneiderw20_b200 import load_workload
+    load_workload(ctx, w.netlist, w.library, w.stimuli, w.vdd)
+    with pytest.raises(AvfsError):
+        ctx.activity()                     # before simulate
+    ctx.set_options(capacity=8)
+    ctx.simulate()
+    with pytest.raises(AvfsError):         # internal signal not kept
+        ctx.waveforms([6], 0, 4)
+    with pytest.raises(AvfsError):         # outside simulated range
+        ctx.waveforms([9], 90, 10)
+    ctx.close()
+
+
+def test_device_stimuli_and_torch_stream():
+    import torch
+    from paper_conf_date_schneiderw20_b200 import Context, load_workload
+    w = make_config(3, n_pairs=96, n_vdd=2, scale=0.05)
+    a = gpu_run(w, keep_all=False)
+    ctx = Context(0)
+    load_workload(ctx, w.netlist, w.library, None, w.vdd)
+    p1 = torch.from_numpy(w.stimuli.p1.view(np.int32)).cuda()
+    p2 = torch.from_numpy(w.stimuli.p2.view(np.int32)).cuda()
+    ctx.set_stimuli(p1, p2)
+    ctx.set_options(capacity=8)
+    s = torch.cuda.Stream()
+    ctx.simulate(s)
+    out = torch.zeros((w.netlist.n_signals, 2), dtype=torch.int64, device="cuda")
+    ctx.activity(out)
+    assert np.array_equal(out.cpu().numpy().astype(np.uint64), a.activity())
