@@ -118,7 +118,7 @@ struct avfs_ctx {
 
     // device state
     bool dev_net_valid = false, dev_vdd_valid = false;
-    DevBuf d_gates, d_coef, d_level_ptr, d_vdd, d_p1, d_p2, d_p1t, d_p2t, d_act, d_latest, d_ovf,
+    DevBuf d_gates, d_ddesc, d_dtab, d_coef, d_level_ptr, d_vdd, d_p1, d_p2, d_p1t, d_p2t, d_act, d_latest, d_ovf,
         d_err, d_list[2], d_count, d_swround, d_swindex, g_loc, g_init, g_count, g_times, g_bad;
     std::vector<DevBuf> scr, pin;     // per round
     int32_t* h_pinned = nullptr;      // small pinned host buffer (count, err)
@@ -312,24 +312,29 @@ avfs_status upload_netlist(avfs_ctx* ctx) {
     if (ctx->dev_net_valid) return AVFS_OK;
     const int32_t G = ctx->n_gates;
     std::vector<GateDesc> gd(std::max<int32_t>(G, 1));
+    std::vector<DelayDesc> dd(std::max<int32_t>(G, 1));
     for (int32_t i = 0; i < G; ++i) {
         const int32_t g = ctx->order[i];
         GateDesc& d = gd[i];
+        DelayDesc& e = dd[i];
         std::memset(&d, 0, sizeof d);
+        std::memset(&e, 0, sizeof e);
         const int k = (int)(ctx->fanin_ptr[g + 1] - ctx->fanin_ptr[g]);
         for (int p = 0; p < KMAX; ++p) d.in_loc[p] = p < k ? ctx->loc[ctx->fanin_sig[ctx->fanin_ptr[g] + p]] : 0u;
         d.out_loc = ctx->loc[ctx->n_pi + g];
         d.sig = (uint32_t)(ctx->n_pi + g);
-        d.tt = ctx->cell_tt[ctx->gate_cell[g]];
-        d.k = (uint8_t)k;
-        d.flags = ctx->is_po[ctx->n_pi + g] ? 1 : 0;
-        d.coef_off = ctx->coef_off[g];
+        d.ttk = (uint32_t)ctx->cell_tt[ctx->gate_cell[g]] | ((uint32_t)k << 16) |
+                ((ctx->is_po[ctx->n_pi + g] ? 1u : 0u) << 24);
+        e.coef_off = ctx->coef_off[g];
+        e.k = (uint32_t)k;
         for (int p = 0; p < k; ++p)
-            for (int pol = 0; pol < 2; ++pol) d.dnom[2 * p + pol] = ctx->d_nom[(ctx->fanin_ptr[g] + p) * 2 + pol];
-        for (int p = k; p < KMAX; ++p) d.dnom[2 * p] = d.dnom[2 * p + 1] = 1.0;
+            for (int pol = 0; pol < 2; ++pol) e.dnom[2 * p + pol] = ctx->d_nom[(ctx->fanin_ptr[g] + p) * 2 + pol];
+        for (int p = k; p < KMAX; ++p) e.dnom[2 * p] = e.dnom[2 * p + 1] = 1.0;
     }
     CK(ctx->d_gates.ensure(gd.size() * sizeof(GateDesc)));
     CK(cudaMemcpy(ctx->d_gates.p, gd.data(), gd.size() * sizeof(GateDesc), cudaMemcpyHostToDevice));
+    CK(ctx->d_ddesc.ensure(dd.size() * sizeof(DelayDesc)));
+    CK(cudaMemcpy(ctx->d_ddesc.p, dd.data(), dd.size() * sizeof(DelayDesc), cudaMemcpyHostToDevice));
     CK(ctx->d_coef.ensure(std::max<size_t>(ctx->coef.size(), 1) * sizeof(double)));
     if (!ctx->coef.empty())
         CK(cudaMemcpy(ctx->d_coef.p, ctx->coef.data(), ctx->coef.size() * sizeof(double), cudaMemcpyHostToDevice));
@@ -761,20 +766,25 @@ avfs_status avfs_sync(avfs_ctx* ctx) {
 
 static avfs_status run_round(avfs_ctx* ctx, Round& R, int round_idx, const int32_t* d_sw_list, int32_t prev_W,
                              int32_t prev_cstage, bool timed) {
-    const int32_t S = ctx->n_pi + ctx->n_gates;
-    (void)S;
-    int wpc = ctx->opt.warps_per_cta > 0 ? ctx->opt.warps_per_cta : 8;
-    int smem = sweep_smem_bytes(wpc, ctx->kmax, R.W, R.cstage);
-    while (wpc > 1 && smem > 227 * 1024) smem = sweep_smem_bytes(--wpc, ctx->kmax, R.W, R.cstage);
+    const bool persistent = (round_idx == 0);
+    // launch bounds: sweep_kernel 256 threads (4 CTAs/SM), level_kernel 512 threads
+    int wpc = ctx->opt.warps_per_cta > 0 ? ctx->opt.warps_per_cta : (persistent ? 8 : 16);
+    wpc = std::min(wpc, persistent ? 8 : 16);
+    const int stage_words = ctx->kmax * R.W;
+    int smem = sweep_smem_bytes(wpc, stage_words, R.cstage);
+    while (wpc > 1 && smem > 227 * 1024) smem = sweep_smem_bytes(--wpc, stage_words, R.cstage);
     if (smem > 227 * 1024) return fail(ctx, AVFS_ERR_CAPACITY, "capacity %d needs %d B shared memory per warp", R.capacity, smem);
     int bps = 0;
-    CK(sweep_occupancy(wpc, smem, &bps));
+    if (persistent) CK(sweep_occupancy(wpc, smem, &bps));
+    else CK(level_occupancy(wpc, smem, &bps));
     if (bps < 1) return fail(ctx, AVFS_ERR_CAPACITY, "sweep kernel does not fit on an SM (smem %d)", smem);
-    R.grid = (int32_t)std::min<int64_t>(R.n_sw, (int64_t)ctx->n_sm * bps);
+    const int64_t resident = (int64_t)ctx->n_sm * bps;
+    R.grid = (int32_t)(persistent ? std::min<int64_t>(R.n_sw, resident) : resident);
     if (R.grid < 1) R.grid = 1;
     if ((int)ctx->scr.size() <= round_idx) ctx->scr.resize(round_idx + 1);
     if ((int)ctx->pin.size() <= round_idx) ctx->pin.resize(round_idx + 1);
-    const size_t scr_bytes = (size_t)std::max(ctx->n_scratch, 1) * R.grid * R.region_bytes;
+    const int64_t scr_slots = persistent ? R.grid : R.n_sw;
+    const size_t scr_bytes = (size_t)std::max(ctx->n_scratch, 1) * scr_slots * R.region_bytes;
     const size_t pin_bytes = (size_t)std::max(ctx->n_pinned, 1) * R.n_sw * R.region_bytes;
     CK(ctx->scr[round_idx].ensure(scr_bytes));
     CK(ctx->pin[round_idx].ensure(pin_bytes));
@@ -784,12 +794,8 @@ static avfs_status run_round(avfs_ctx* ctx, Round& R, int round_idx, const int32
     p.gates = ctx->d_gates.as<GateDesc>();
     p.level_ptr = ctx->d_level_ptr.as<int32_t>();
     p.depth = ctx->depth;
-    p.coef = ctx->d_coef.as<double>();
-    p.deg_v = ctx->deg_v;
-    p.vdd = ctx->d_vdd.as<double>();
-    p.v_min = ctx->v_min;
-    p.v_max = ctx->v_max;
-    p.quantum = ctx->opt.quantum_ps;
+    p.n_gates = ctx->n_gates;
+    p.dtab = ctx->d_dtab.as<float4>();
     p.p1t = ctx->d_p1t.as<uint32_t>();
     p.p2t = ctx->d_p2t.as<uint32_t>();
     p.n_pw = (int32_t)((ctx->n_pairs + 31) / 32);
@@ -804,18 +810,22 @@ static avfs_status run_round(avfs_ctx* ctx, Round& R, int round_idx, const int32
     p.pinned = ctx->pin[round_idx].as<uint8_t>();
     p.region_bytes = R.region_bytes;
     p.W = R.W;
+    p.stage_words = stage_words;
     p.cstage = R.cstage;
     p.prev_W = prev_W;
     p.prev_cstage = prev_cstage;
-    p.kmax = ctx->kmax;
     p.act = ctx->d_act.as<unsigned long long>();
     p.latest = ctx->d_latest.as<unsigned int>();
     p.ovf = ctx->d_ovf.as<int32_t>();
-    p.err = ctx->d_err.as<int32_t>();
     if (timed) CK(cudaEventRecord(ctx->ev0, ctx->stream));
-    CK(launch_sweep(p, R.grid, wpc, ctx->stream));
+    if (persistent) {
+        CK(launch_sweep(p, R.grid, wpc, ctx->stream));
+        ctx->stats.launches++;
+    } else {
+        for (int L = 0; L < ctx->depth; ++L) CK(launch_level(p, L, R.grid, wpc, ctx->stream));
+        ctx->stats.launches += ctx->depth;
+    }
     if (timed) CK(cudaEventRecord(ctx->ev1, ctx->stream));
-    ctx->stats.launches++;
     if (round_idx == 0) ctx->stats.warps_per_cta = wpc;
     return AVFS_OK;
 }
@@ -856,6 +866,24 @@ avfs_status avfs_simulate(avfs_ctx* ctx, void* cuda_stream) {
     CK(cudaMemsetAsync(ctx->d_act.p, 0, (size_t)S * V * sizeof(unsigned long long), ctx->stream));
     CK(cudaMemsetAsync(ctx->d_latest.p, 0, (size_t)V * 4, ctx->stream));
     CK(cudaMemsetAsync(ctx->d_err.p, 0, 16, ctx->stream));
+    // delay computation kernel: d'(gate, pin, pol, Vdd) in FP64 -> binary32 table
+    CK(ctx->d_dtab.ensure((size_t)V * std::max(ctx->n_gates, 1) * 8 * sizeof(float)));
+    {
+        DelayParams dp{};
+        dp.dd = ctx->d_ddesc.as<DelayDesc>();
+        dp.n_gates = ctx->n_gates;
+        dp.coef = ctx->d_coef.as<double>();
+        dp.deg_v = ctx->deg_v;
+        dp.vdd = ctx->d_vdd.as<double>();
+        dp.n_vdd = V;
+        dp.v_min = ctx->v_min;
+        dp.v_max = ctx->v_max;
+        dp.quantum = ctx->opt.quantum_ps;
+        dp.dtab = ctx->d_dtab.as<float>();
+        dp.err = ctx->d_err.as<int32_t>();
+        CK(launch_delays(dp, ctx->stream));
+        ctx->stats.launches++;
+    }
     // H4: stimulus expansion (transpose to PI-major 32-pair words)
     CK(launch_expand(ctx->d_p1.as<uint32_t>(), ctx->d_p2.as<uint32_t>(), P, ctx->words, ctx->n_pi, n_pw,
                      ctx->d_p1t.as<uint32_t>(), ctx->d_p2t.as<uint32_t>(), ctx->stream));

@@ -22,18 +22,37 @@ constexpr uint32_t HDR_INIT = 1u << 20;      // value before t = 0
 constexpr uint32_t HDR_POISON = 1u << 21;    // events not stored here or upstream
 constexpr uint32_t HDR_PREV = 1u << 22;      // would have been poisoned at the previous round's capacity
 
-// Gate descriptor, 96 B, read warp-uniformly (P:L154 step 1).
+// Gate descriptor, 32 B, read warp-uniformly (P:L154 step 1).
 struct alignas(16) GateDesc {
     uint32_t in_loc[KMAX];
     uint32_t out_loc;
     uint32_t sig;        // output signal id (activity row)
-    uint16_t tt;         // truth table
-    uint8_t k;           // number of inputs
-    uint8_t flags;       // bit 0: drives a primary output (latest arrival)
-    uint32_t coef_off;   // offset (doubles) of [pin][pol][deg_v+1] coefficient block
-    double dnom[2 * KMAX];   // [pin][pol] nominal delay, ps
+    uint32_t ttk;        // bits 0..15 truth table, 16..23 #inputs, 24..31 flags (bit 24: PO)
+    uint32_t pad;
 };
-static_assert(sizeof(GateDesc) == 96, "GateDesc layout");
+static_assert(sizeof(GateDesc) == 32, "GateDesc layout");
+
+// Inputs of the delay computation kernel: per sorted gate.
+struct alignas(16) DelayDesc {
+    double dnom[2 * KMAX];   // [pin][pol] nominal delay, ps
+    uint32_t coef_off;       // offset (doubles) of the [pin][pol][deg_v+1] coefficient block
+    uint32_t k;
+    uint32_t pad[2];
+};
+static_assert(sizeof(DelayDesc) == 80, "DelayDesc layout");
+
+struct DelayParams {
+    const DelayDesc* __restrict__ dd;
+    int32_t n_gates;
+    const double* __restrict__ coef;
+    int32_t deg_v;
+    const double* __restrict__ vdd;          // [n_vdd] volts
+    int32_t n_vdd;
+    double v_min, v_max;
+    double quantum;                          // 0: F mode
+    float* dtab;                             // [n_vdd][n_gates][8] delays (binary32), ps
+    int32_t* err;                            // bit 0: non-positive delay
+};
 
 // One slot-warp region: 32 header words followed by W = 32*C event times
 // (compact: lane l's events start at the exclusive prefix sum of the counts).
@@ -41,11 +60,8 @@ struct SweepParams {
     const GateDesc* __restrict__ gates;     // sorted by level
     const int32_t* __restrict__ level_ptr;  // [depth+1] offsets into gates (level 1..depth)
     int32_t depth;
-    const double* __restrict__ coef;        // coefficient blocks
-    int32_t deg_v;
-    const double* __restrict__ vdd;         // [n_vdd] volts
-    double v_min, v_max;
-    double quantum;                         // 0: F mode
+    int32_t n_gates;
+    const float4* __restrict__ dtab;        // [n_vdd][n_gates][2] float4 delays
     const uint32_t* __restrict__ p1t;       // [n_pi][n_pw] bit-transposed stimuli
     const uint32_t* __restrict__ p2t;
     int32_t n_pw;                           // pair-warps (ceil(n_pairs/32))
@@ -57,24 +73,26 @@ struct SweepParams {
     int64_t sw_first;
     int64_t n_sw;
     // arenas
-    uint8_t* scratch;                       // [n_scratch][gridDim.x][region]
+    uint8_t* scratch;                       // persistent: [n_scratch][gridDim.x][region]; level: [n_scratch][n_sw][region]
     uint8_t* pinned;                        // [n_pinned][n_sw][region]
     int64_t region_bytes;
     int32_t W;                              // event capacity per region (32*C)
+    int32_t stage_words;                    // per-warp input staging: max fan-in x W
     int32_t cstage;                         // per-slot capacity (2*C)
     int32_t prev_W, prev_cstage;            // previous round (0: first pass)
-    int32_t kmax;                           // max fan-in in the netlist (smem sizing)
     // outputs
     unsigned long long* act;                // [n_signals][n_vdd]
     unsigned int* latest;                   // [n_vdd] float bits (non-negative)
     int32_t* ovf;                           // [n_sw] overflow flag per slot-warp
-    int32_t* err;                           // bit 0: non-positive delay
 };
 
 // launch wrappers (avfs_kernels.cu)
-int sweep_smem_bytes(int warps_per_cta, int kmax, int W, int cstage);
+int sweep_smem_bytes(int warps_per_cta, int stage_words, int cstage);
 cudaError_t sweep_occupancy(int warps_per_cta, int smem, int* blocks_per_sm);
+cudaError_t launch_delays(const DelayParams& p, cudaStream_t st);
 cudaError_t launch_sweep(const SweepParams& p, int grid, int warps_per_cta, cudaStream_t st);
+cudaError_t level_occupancy(int warps_per_cta, int smem, int* blocks_per_sm);
+cudaError_t launch_level(const SweepParams& p, int level, int grid, int warps_per_cta, cudaStream_t st);
 cudaError_t launch_expand(const uint32_t* p1, const uint32_t* p2, int64_t n_pairs, int32_t words,
                           int32_t n_pi, int32_t n_pw, uint32_t* p1t, uint32_t* p2t, cudaStream_t st);
 cudaError_t launch_pi_activity(const uint32_t* p1t, const uint32_t* p2t, int32_t n_pi, int32_t n_pw,

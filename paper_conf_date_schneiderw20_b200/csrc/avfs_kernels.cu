@@ -62,26 +62,77 @@ __device__ __forceinline__ uint32_t warp_incl_scan(uint32_t v, int lane) {
 }
 
 // ---------------------------------------------------------------------------
-// Per-slot merge of up to K sorted input event lists with the inertial filter
-// (reading C3: cancel the pending last output event iff it lies strictly after
-// the input event; C4: no reschedule on confirming events; C5: ties in time
-// are taken in ascending pin order).  Returns the exact output count; the
-// first `cstage` surviving events are left in s_out[i*32 + lane].
+// Delay computation kernel (P:L139, P:L152-L160 steps 3-5): one thread per
+// (operating point, gate, pin, polarity).  f(P) of Eq. (4) by Horner with FMA
+// in FP64, d' = d_nom (1 + f) (Eq. 9), optional Q-mode rounding
+// (reading C12), rounded once to binary32 (reading C11).  The sweep reads the
+// 8 delays of a gate as two uniform float4 loads per 32 slots.
 // ---------------------------------------------------------------------------
+__global__ void delay_kernel(const DelayParams p) {
+    const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    const int64_t total = (int64_t)p.n_vdd * p.n_gates * 8;
+    if (t >= total) return;
+    const int e = (int)(t & 7);
+    const int64_t vg = t >> 3;
+    const int g = (int)(vg % p.n_gates);
+    const int kv = (int)(vg / p.n_gates);
+    const DelayDesc& D = p.dd[g];
+    float out = 1.0f;
+    if (e < 2 * (int)D.k) {
+        const double x = (p.vdd[kv] - p.v_min) / (p.v_max - p.v_min);      // phi_V
+        const double* cf = p.coef + D.coef_off + e * (p.deg_v + 1);
+        double f = cf[p.deg_v];
+        for (int i = p.deg_v - 1; i >= 0; --i) f = fma(f, x, cf[i]);
+        double d = D.dnom[e] * (1.0 + f);
+        if (p.quantum > 0.0) d = p.quantum * rint(d / p.quantum);
+        if (!(d > 0.0)) atomicOr(p.err, 1);
+        out = __double2float_rn(d);
+    }
+    p.dtab[t] = out;
+}
+
+cudaError_t launch_delays(const DelayParams& p, cudaStream_t st) {
+    const int64_t n = (int64_t)p.n_vdd * p.n_gates * 8;
+    if (n == 0) return cudaSuccess;
+    delay_kernel<<<(unsigned)((n + 255) / 256), 256, 0, st>>>(p);
+    return cudaGetLastError();
+}
+
+// ---------------------------------------------------------------------------
+// Per-slot merge of K sorted input event lists with the inertial filter
+// (reading C3: cancel the pending last output event iff it lies
+// strictly after the input event; C4: no reschedule on confirming events;
+// C5: ties in time are taken in ascending pin order).  Branch-free body; the
+// element after each head is prefetched from shared memory one step ahead.
+// Returns the exact output count; the first `cstage` surviving events are in
+// s_out[i*32 + lane].
+// ---------------------------------------------------------------------------
+__device__ __forceinline__ float lds_f32(uint32_t addr) {
+    float v;
+    asm volatile("ld.shared.f32 %0, [%1];\n" : "=f"(v) : "r"(addr));
+    return v;
+}
+__device__ __forceinline__ void sts_f32(uint32_t addr, float v) {
+    asm volatile("st.shared.f32 [%0], %1;\n" ::"r"(addr), "f"(v) : "memory");
+}
+
 template <int K>
-__device__ __forceinline__ int merge_slot(const float* __restrict__ s_in, const int (&c0)[KMAX],
-                                          const int (&n)[KMAX], const bool (&pi)[KMAX],
-                                          const float (&df)[KMAX], const float (&dr)[KMAX],
-                                          uint32_t tt, uint32_t bits, uint32_t proj,
-                                          float* __restrict__ s_out, int cstage, int lane) {
+__device__ __forceinline__ int merge_slot(uint32_t s_in, const int (&cb)[KMAX], const int (&n)[KMAX],
+                                          const bool (&pi)[KMAX], const float (&dl)[8], uint32_t tt,
+                                          uint32_t bits, uint32_t proj, uint32_t s_out_lane, int cstage) {
     const float INF = __int_as_float(0x7f800000);
-    float h[K];
+    float h[K], nh[K];
     int c[K], e[K];
 #pragma unroll
     for (int q = 0; q < K; ++q) {
-        c[q] = pi[q] ? 0 : c0[q];
-        e[q] = c[q] + n[q];
-        h[q] = (n[q] > 0) ? (pi[q] ? 0.0f : s_in[c[q]]) : INF;
+        c[q] = cb[q];
+        e[q] = cb[q] + n[q];
+        // every address below stays inside the per-warp staging area (budget + 16 words):
+        // loads beyond a list return garbage that is replaced by INF.
+        const float a0 = lds_f32(s_in + 4u * (uint32_t)c[q]);
+        const float a1 = lds_f32(s_in + 4u * (uint32_t)(c[q] + 1));
+        h[q] = n[q] > 0 ? (pi[q] ? 0.0f : a0) : INF;
+        nh[q] = (n[q] > 1 && !pi[q]) ? a1 : INF;
     }
     int n_out = 0;
     float tl = -INF;
@@ -89,32 +140,35 @@ __device__ __forceinline__ int merge_slot(const float* __restrict__ s_in, const 
         float t = h[0];
         int pm = 0;
 #pragma unroll
-        for (int q = 1; q < K; ++q)
-            if (h[q] < t) { t = h[q]; pm = q; }
+        for (int q = 1; q < K; ++q) {
+            const bool lt = h[q] < t;
+            t = lt ? h[q] : t;
+            pm = lt ? q : pm;
+        }
         if (!(t < INF)) break;
+        // consume the head of pin pm; prefetch the element after its new head
         int cn = c[0], en = e[0];
-        float d_r = dr[0], d_f = df[0];
+        float hn = nh[0], dfp = dl[0], drp = dl[1];
 #pragma unroll
         for (int q = 1; q < K; ++q)
-            if (q == pm) { cn = c[q]; en = e[q]; d_r = dr[q]; d_f = df[q]; }
+            if (pm == q) { cn = c[q]; en = e[q]; hn = nh[q]; dfp = dl[2 * q]; drp = dl[2 * q + 1]; }
         ++cn;
-        const float hn = (cn < en) ? s_in[cn] : INF;
+        const float raw = lds_f32(s_in + 4u * (uint32_t)(cn + 1));
+        const float nn = (cn + 1 < en) ? raw : INF;
 #pragma unroll
         for (int q = 0; q < K; ++q)
-            if (q == pm) { c[q] = cn; h[q] = hn; }
+            if (pm == q) { c[q] = cn; h[q] = hn; nh[q] = nn; }
         bits ^= 1u << pm;
         const uint32_t y = (tt >> bits) & 1u;
-        if (y != proj) {
-            proj = y;
-            if (tl > t) {            // pending output lies after t: pulse filtered
-                --n_out;
-                tl = -INF;           // the event before it is <= t (never cancelled twice)
-            } else {
-                tl = t + (y ? d_r : d_f);
-                if (n_out < cstage) s_out[n_out * 32 + lane] = tl;
-                ++n_out;
-            }
-        }
+        const bool change = y != proj;
+        const bool cancel = change && (tl > t);     // pending output lies after t: pulse filtered
+        const bool push = change && !cancel;
+        const float tn = t + (y ? drp : dfp);
+        // unconditional store to the next free row (clamped): harmless unless pushed
+        sts_f32(s_out_lane + 128u * (uint32_t)min(n_out, cstage), tn);
+        n_out += push ? 1 : (cancel ? -1 : 0);
+        tl = push ? tn : (cancel ? -INF : tl);      // after a cancel the last event is <= t
+        proj = y;
     }
     return n_out;
 }
@@ -125,179 +179,236 @@ __device__ __forceinline__ uint8_t* region_of(uint32_t loc, uint8_t* scr, int64_
     return ((loc & LOC_KIND) == LOC_SCRATCH) ? scr + id * scr_stride : pin + id * pin_stride;
 }
 
-__global__ void __launch_bounds__(512) sweep_kernel(const SweepParams p) {
+// Where one warp's 32 slots live for the gate being evaluated.
+struct Env {
+    uint8_t* scr;
+    int64_t scr_stride;
+    uint8_t* pin;
+    int64_t pin_stride;
+    int64_t i;           // index of the slot group in this run (overflow flag)
+    uint32_t mask;       // lanes holding a simulated slot
+    int pw, kv, lane;
+    float* s_in;         // per-warp input staging (budget + 16 words)
+    float* s_out;        // per-warp output staging (32 * (cstage + 1) words)
+    uint32_t s_in_a;     // the same, as shared-window addresses
+    uint32_t s_out_a;    // s_out + 4 * lane
+};
+
+// One gate for one 32-slot group: input headers,
+// compact staging, merge/filter, output compaction, reductions.
+template <int K>
+__device__ __forceinline__ void eval_gate(const SweepParams& p, const Env& E, const uint4 ins, const uint4 hd,
+                                          const float (&dl)[8]) {
+    const int lane = E.lane;
+    const uint32_t out_loc = hd.x, sig = hd.y;
+    const uint32_t tt = hd.z & 0xffffu;
+    const uint32_t gflags = hd.z >> 24;
+    const uint32_t in_loc[KMAX] = {ins.x, ins.y, ins.z, ins.w};
+    int n[KMAX], cb[KMAX];
+    bool isp[KMAX];
+    const float* ev[KMAX];
+    uint32_t bits = 0, pois = 0, prevp = 0;
+    int sum = 0;
+#pragma unroll
+    for (int q = 0; q < KMAX; ++q) {
+        n[q] = 0;
+        cb[q] = 0;
+        isp[q] = true;
+        ev[q] = nullptr;
+        if (q < K) {
+            const uint32_t loc = in_loc[q];
+            if ((loc & LOC_KIND) == LOC_PI) {
+                const int64_t o = (int64_t)(loc & LOC_ID) * p.n_pw + E.pw;
+                const uint32_t w1 = __ldg(p.p1t + o) & E.mask;
+                const uint32_t w2 = __ldg(p.p2t + o) & E.mask;
+                bits |= ((w1 >> lane) & 1u) << q;
+                n[q] = (int)(((w1 ^ w2) >> lane) & 1u);
+            } else {
+                const uint8_t* r = region_of(loc, E.scr, E.scr_stride, E.pin, E.pin_stride);
+                const uint32_t h = ld_u32(r + 4 * lane);
+                n[q] = (int)(h & HDR_N);
+                bits |= ((h >> 20) & 1u) << q;
+                pois |= h & HDR_POISON;
+                prevp |= h & HDR_PREV;
+                isp[q] = false;
+                ev[q] = reinterpret_cast<const float*>(r + 128);
+            }
+            sum += n[q];
+        }
+    }
+    const uint32_t y0 = (tt >> bits) & 1u;
+    uint8_t* ro = region_of(out_loc, E.scr, E.scr_stride, E.pin, E.pin_stride);
+    uint32_t* ro_hdr = reinterpret_cast<uint32_t*>(ro);
+    const bool first_pass = (p.prev_W == 0);
+    const bool any_prev = first_pass || __any_sync(0xffffffffu, prevp != 0);
+    if (__any_sync(0xffffffffu, pois != 0)) {          // upstream overflow: nothing valid here
+        __stcg(ro_hdr + lane, HDR_POISON | HDR_PREV | (y0 << 20));
+        return;
+    }
+    if (!__any_sync(0xffffffffu, sum != 0)) {          // no input event in any slot: constant output
+        __stcg(ro_hdr + lane, (y0 << 20) | (any_prev ? HDR_PREV : 0u));
+        return;
+    }
+    // compact per-pin offsets: exclusive warp scans of the stored counts (2 pins per scan)
+    int tot[KMAX] = {0, 0, 0, 0};
+    {
+        const uint32_t a = (uint32_t)(isp[0] ? 0 : n[0]) | ((uint32_t)(K > 1 && !isp[1] ? n[1] : 0) << 16);
+        const uint32_t ia = warp_incl_scan(a, lane);
+        const uint32_t ta = __shfl_sync(0xffffffffu, ia, 31);
+        const uint32_t ea = ia - a;
+        cb[0] = (int)(ea & 0xffffu);  tot[0] = (int)(ta & 0xffffu);
+        cb[1] = (int)(ea >> 16);      tot[1] = (int)(ta >> 16);
+        if (K > 2) {
+            const uint32_t b = (uint32_t)(isp[2] ? 0 : n[2]) | ((uint32_t)(K > 3 && !isp[3] ? n[3] : 0) << 16);
+            const uint32_t ib = warp_incl_scan(b, lane);
+            const uint32_t tb = __shfl_sync(0xffffffffu, ib, 31);
+            const uint32_t eb = ib - b;
+            cb[2] = (int)(eb & 0xffffu);  tot[2] = (int)(tb & 0xffffu);
+            cb[3] = (int)(eb >> 16);      tot[3] = (int)(tb >> 16);
+        }
+    }
+    // stage the compact input lists (16-B cp.async)
+    int base = 0;
+#pragma unroll
+    for (int q = 0; q < K; ++q) {
+        if (!isp[q]) {
+            cb[q] += base;
+            base += (tot[q] + 3) & ~3;
+        }
+    }
+    if (base > p.stage_words) {                        // cannot happen: each input total <= W
+        __stcg(ro_hdr + lane, HDR_POISON | HDR_PREV | (y0 << 20));
+        if (lane == 0) p.ovf[E.i] = 1;
+        return;
+    }
+    {
+        int off = 0;
+#pragma unroll
+        for (int q = 0; q < K; ++q) {
+            if (!isp[q]) {
+                const int nv = (tot[q] + 3) >> 2;
+                for (int v = lane; v < nv; v += 32) cp_async16(E.s_in + off + 4 * v, ev[q] + 4 * v);
+                off += nv * 4;
+            }
+        }
+    }
+    cp_async_wait_all();
+    __syncwarp();
+    const int n_out = merge_slot<K>(E.s_in_a, cb, n, isp, dl, tt, bits, y0, E.s_out_a, p.cstage);
+    // output: scan, overflow ballot, direct compact stores
+    const uint32_t incl = warp_incl_scan((uint32_t)n_out, lane);
+    const uint32_t total = __shfl_sync(0xffffffffu, incl, 31);
+    const uint32_t excl = incl - (uint32_t)n_out;
+    const bool ovf = __any_sync(0xffffffffu, n_out > p.cstage) || total > (uint32_t)p.W;
+    bool prev = true;
+    if (!first_pass)
+        prev = any_prev || __any_sync(0xffffffffu, n_out > p.prev_cstage) || total > (uint32_t)p.prev_W;
+    if (!ovf) {
+        float* dst = reinterpret_cast<float*>(ro + 128) + excl;
+        for (int t = 0; t < n_out; ++t) __stcg(dst + t, E.s_out[t * 32 + lane]);
+    } else if (lane == 0) {
+        p.ovf[E.i] = 1;
+    }
+    __stcg(ro_hdr + lane, (uint32_t)min(n_out, (int)HDR_N) | (y0 << 20) | (ovf ? HDR_POISON : 0u) |
+                              (prev ? HDR_PREV : 0u));
+    // activity (reading C15) and latest PO arrival: counted once per
+    // slot across overflow rounds (where prev && !ovf)
+    if (!ovf && prev) {
+        if (lane == 0 && total) atomicAdd(p.act + (int64_t)sig * p.n_vdd + E.kv, (unsigned long long)total);
+        if (gflags & 1u) {
+            const float last = n_out ? E.s_out[(n_out - 1) * 32 + lane] : 0.0f;
+            const uint32_t m = __reduce_max_sync(0xffffffffu, __float_as_uint(last));
+            if (lane == 0 && m) atomicMax(p.latest + E.kv, m);
+        }
+    }
+    __syncwarp();
+}
+
+__device__ __forceinline__ void eval_dispatch(const SweepParams& p, const Env& E, const uint4 ins, const uint4 hd,
+                                              const float4 d0, const float4 d1) {
+    const float dl[8] = {d0.x, d0.y, d0.z, d0.w, d1.x, d1.y, d1.z, d1.w};
+    switch ((hd.z >> 16) & 0xffu) {
+        case 1: eval_gate<1>(p, E, ins, hd, dl); break;
+        case 2: eval_gate<2>(p, E, ins, hd, dl); break;
+        case 3: eval_gate<3>(p, E, ins, hd, dl); break;
+        default: eval_gate<4>(p, E, ins, hd, dl); break;
+    }
+}
+
+__device__ __forceinline__ void slot_group(const SweepParams& p, int64_t i, int lane, Env& E) {
+    const int64_t sw = p.sw_list ? (int64_t)p.sw_list[i] : p.sw_first + i;
+    E.kv = (int)(sw / p.n_pw);
+    E.pw = (int)(sw % p.n_pw);
+    const int64_t j = (int64_t)E.pw * 32 + lane;
+    const int64_t pub = (int64_t)E.kv * p.n_pairs + j;
+    const bool valid = j < p.n_pairs && pub >= p.slot_first && pub < p.slot_end;
+    E.mask = __ballot_sync(0xffffffffu, valid);
+    E.i = i;
+    E.lane = lane;
+}
+
+// Persistent level sweep (pass 0): one CTA owns one 32-slot group at a time
+// and walks all levels with a CTA barrier between levels.  Gate
+// descriptors and delays are prefetched one gate ahead.
+__global__ void __launch_bounds__(256, 4) sweep_kernel(const SweepParams p) {
     extern __shared__ __align__(16) float smem[];
     const int lane = threadIdx.x & 31;
     const int warp = threadIdx.x >> 5;
     const int nw = blockDim.x >> 5;
-    const int in_words = p.kmax * p.W + 16;
-    float* s_in = smem + (size_t)warp * (size_t)(in_words + 32 * p.cstage);
-    float* s_out = s_in + in_words;
-    const bool first_pass = (p.prev_W == 0);
-    const int64_t scr_stride = (int64_t)gridDim.x * p.region_bytes;
-    const int64_t pin_stride = p.n_sw * p.region_bytes;
-
+    Env E;
+    E.s_in = smem + (size_t)warp * (size_t)(p.stage_words + 16 + 32 * (p.cstage + 1));
+    E.s_out = E.s_in + p.stage_words + 16;
+    E.s_in_a = static_cast<uint32_t>(__cvta_generic_to_shared(E.s_in));
+    E.s_out_a = static_cast<uint32_t>(__cvta_generic_to_shared(E.s_out)) + 4u * (uint32_t)lane;
+    E.scr_stride = (int64_t)gridDim.x * p.region_bytes;
+    E.pin_stride = p.n_sw * p.region_bytes;
+    const uint4* gd = reinterpret_cast<const uint4*>(p.gates);
     for (int64_t i = blockIdx.x; i < p.n_sw; i += gridDim.x) {
-        const int64_t sw = p.sw_list ? (int64_t)p.sw_list[i] : p.sw_first + i;
-        const int kv = (int)(sw / p.n_pw);
-        const int pw = (int)(sw % p.n_pw);
-        const int64_t j = (int64_t)pw * 32 + lane;
-        const int64_t pub = (int64_t)kv * p.n_pairs + j;
-        const bool valid = j < p.n_pairs && pub >= p.slot_first && pub < p.slot_end;
-        const uint32_t mask = __ballot_sync(0xffffffffu, valid);
-        // Step 2: the operating point of this slot group, normalised
-        const double x = (p.vdd[kv] - p.v_min) / (p.v_max - p.v_min);
-        uint8_t* scr = p.scratch + (int64_t)blockIdx.x * p.region_bytes;
-        uint8_t* pin = p.pinned + i * p.region_bytes;
-
+        slot_group(p, i, lane, E);
+        E.scr = p.scratch + (int64_t)blockIdx.x * p.region_bytes;
+        E.pin = p.pinned + i * p.region_bytes;
+        const float4* dt = p.dtab + (int64_t)E.kv * p.n_gates * 2;
         for (int L = 0; L < p.depth; ++L) {
-            const int g_end = p.level_ptr[L + 1];
-            for (int gi = p.level_ptr[L] + warp; gi < g_end; gi += nw) {
-                const GateDesc* G = p.gates + gi;
-                // Step 1: gate description, warp-uniform
-                const uint4 ins = __ldg(reinterpret_cast<const uint4*>(G));
-                const uint4 hd = __ldg(reinterpret_cast<const uint4*>(G) + 1);
-                const uint32_t out_loc = hd.x, sig = hd.y;
-                const uint32_t tt = hd.z & 0xffffu;
-                const int K = (int)((hd.z >> 16) & 0xffu);
-                const uint32_t gflags = hd.z >> 24;
-                // Steps 3-5, repeated per pin-to-pin delay: lane
-                // 2*pin+pol evaluates Eq. (4) by Horner/FMA in FP64 and Eq. (9)
-                float dl = 1.0f;
-                if (lane < 2 * K) {
-                    const double* cf = p.coef + hd.w + lane * (p.deg_v + 1);
-                    double f = __ldg(cf + p.deg_v);
-                    for (int t = p.deg_v - 1; t >= 0; --t) f = fma(f, x, __ldg(cf + t));
-                    double d = __ldg(&G->dnom[lane]) * (1.0 + f);
-                    if (p.quantum > 0.0) d = p.quantum * rint(d / p.quantum);
-                    if (!(d > 0.0)) atomicOr(p.err, 1);
-                    dl = __double2float_rn(d);
-                }
-                float df[KMAX], dr[KMAX];
-#pragma unroll
-                for (int q = 0; q < KMAX; ++q) {
-                    df[q] = __shfl_sync(0xffffffffu, dl, 2 * q);
-                    dr[q] = __shfl_sync(0xffffffffu, dl, 2 * q + 1);
-                }
-                // input waveforms: headers (coalesced) or PI bits (broadcast)
-                const uint32_t in_loc[KMAX] = {ins.x, ins.y, ins.z, ins.w};
-                int n[KMAX];
-                bool isp[KMAX];
-                const float* ev[KMAX];
-                uint32_t bits = 0, pois = 0, prevp = 0;
-#pragma unroll
-                for (int q = 0; q < KMAX; ++q) {
-                    n[q] = 0;
-                    isp[q] = true;
-                    ev[q] = nullptr;
-                    if (q < K) {
-                        const uint32_t loc = in_loc[q];
-                        if ((loc & LOC_KIND) == LOC_PI) {
-                            const int64_t o = (int64_t)(loc & LOC_ID) * p.n_pw + pw;
-                            const uint32_t w1 = __ldg(p.p1t + o) & mask;
-                            const uint32_t w2 = __ldg(p.p2t + o) & mask;
-                            bits |= ((w1 >> lane) & 1u) << q;
-                            n[q] = (int)(((w1 ^ w2) >> lane) & 1u);
-                        } else {
-                            const uint8_t* r = region_of(loc, scr, scr_stride, pin, pin_stride);
-                            const uint32_t h = ld_u32(r + 4 * lane);
-                            n[q] = (int)(h & HDR_N);
-                            bits |= ((h >> 20) & 1u) << q;
-                            pois |= h & HDR_POISON;
-                            prevp |= h & HDR_PREV;
-                            isp[q] = false;
-                            ev[q] = reinterpret_cast<const float*>(r + 128);
-                        }
-                    }
-                }
-                const uint32_t y0 = (tt >> bits) & 1u;
-                uint8_t* ro = region_of(out_loc, scr, scr_stride, pin, pin_stride);
-                uint32_t* ro_hdr = reinterpret_cast<uint32_t*>(ro);
-                const bool any_prev = __any_sync(0xffffffffu, prevp != 0);
-                if (__any_sync(0xffffffffu, pois != 0)) {
-                    ro_hdr[lane] = HDR_POISON | HDR_PREV | (y0 << 20);
-                    continue;
-                }
-                // compact per-pin offsets: exclusive warp scans of the counts
-                int c0[KMAX], tot[KMAX];
-                {
-                    const uint32_t a = (uint32_t)(isp[0] ? 0 : n[0]) | ((uint32_t)(isp[1] ? 0 : n[1]) << 16);
-                    const uint32_t ia = warp_incl_scan(a, lane);
-                    const uint32_t ta = __shfl_sync(0xffffffffu, ia, 31);
-                    const uint32_t ea = ia - a;
-                    c0[0] = (int)(ea & 0xffffu);  tot[0] = (int)(ta & 0xffffu);
-                    c0[1] = (int)(ea >> 16);      tot[1] = (int)(ta >> 16);
-                    if (K > 2) {
-                        const uint32_t b = (uint32_t)(isp[2] ? 0 : n[2]) | ((uint32_t)(isp[3] ? 0 : n[3]) << 16);
-                        const uint32_t ib = warp_incl_scan(b, lane);
-                        const uint32_t tb = __shfl_sync(0xffffffffu, ib, 31);
-                        const uint32_t eb = ib - b;
-                        c0[2] = (int)(eb & 0xffffu);  tot[2] = (int)(tb & 0xffffu);
-                        c0[3] = (int)(eb >> 16);      tot[3] = (int)(tb >> 16);
-                    } else {
-                        c0[2] = c0[3] = tot[2] = tot[3] = 0;
-                    }
-                }
-                // stage the compact input lists into shared memory (16-B cp.async)
-                int base = 0;
-#pragma unroll
-                for (int q = 0; q < KMAX; ++q) {
-                    if (q < K && !isp[q]) {
-                        const int nv = (tot[q] + 3) >> 2;
-                        for (int v = lane; v < nv; v += 32) cp_async16(s_in + base + 4 * v, ev[q] + 4 * v);
-                        c0[q] += base;
-                        base += nv * 4;
-                    }
-                }
-                cp_async_wait_all();
-                __syncwarp();
-                int n_out;
-                switch (K) {
-                    case 1: n_out = merge_slot<1>(s_in, c0, n, isp, df, dr, tt, bits, y0, s_out, p.cstage, lane); break;
-                    case 2: n_out = merge_slot<2>(s_in, c0, n, isp, df, dr, tt, bits, y0, s_out, p.cstage, lane); break;
-                    case 3: n_out = merge_slot<3>(s_in, c0, n, isp, df, dr, tt, bits, y0, s_out, p.cstage, lane); break;
-                    default: n_out = merge_slot<4>(s_in, c0, n, isp, df, dr, tt, bits, y0, s_out, p.cstage, lane); break;
-                }
-                // output: scan, overflow ballot, compaction, 128-bit stores
-                const uint32_t incl = warp_incl_scan((uint32_t)n_out, lane);
-                const uint32_t total = __shfl_sync(0xffffffffu, incl, 31);
-                const uint32_t excl = incl - (uint32_t)n_out;
-                const bool ovf = __any_sync(0xffffffffu, n_out > p.cstage) || total > (uint32_t)p.W;
-                bool prev = true;
-                if (!first_pass)
-                    prev = any_prev || __any_sync(0xffffffffu, n_out > p.prev_cstage) || total > (uint32_t)p.prev_W;
-                __syncwarp();
-                if (!ovf) {
-                    for (int t = 0; t < n_out; ++t) s_in[excl + t] = s_out[t * 32 + lane];
-                    __syncwarp();
-                    float* dst = reinterpret_cast<float*>(ro + 128);
-                    const int nv = (int)((total + 3) >> 2);
-                    for (int v = lane; v < nv; v += 32)
-                        st_global_v4(dst + 4 * v, reinterpret_cast<const float4*>(s_in)[v]);
-                } else if (lane == 0) {
-                    p.ovf[i] = 1;
-                }
-                ro_hdr[lane] = (uint32_t)min(n_out, (int)HDR_N) | (y0 << 20) | (ovf ? HDR_POISON : 0u) |
-                               (prev ? HDR_PREV : 0u);
-                // activity (reading C15) and latest PO arrival: counted
-                // once per slot across overflow rounds (only where prev && !ovf)
-                if (!ovf && prev) {
-                    if (lane == 0 && total) atomicAdd(p.act + (int64_t)sig * p.n_vdd + kv, (unsigned long long)total);
-                    if (gflags & 1u) {
-                        const float last = n_out ? s_out[(n_out - 1) * 32 + lane] : 0.0f;
-                        const uint32_t m = __reduce_max_sync(0xffffffffu, __float_as_uint(last));
-                        if (lane == 0 && m) atomicMax(p.latest + kv, m);
-                    }
-                }
-                __syncwarp();
-            }
+            const int g_end = __ldg(p.level_ptr + L + 1);
+            for (int gi = __ldg(p.level_ptr + L) + warp; gi < g_end; gi += nw)
+                eval_dispatch(p, E, __ldg(gd + 2 * gi), __ldg(gd + 2 * gi + 1), __ldg(dt + 2 * gi),
+                              __ldg(dt + 2 * gi + 1));
             __syncthreads();
         }
     }
 }
 
-int sweep_smem_bytes(int warps_per_cta, int kmax, int W, int cstage) {
-    return warps_per_cta * (kmax * W + 16 + 32 * cstage) * 4;
+// Level-parallel variant for overflow reruns (few slot groups): one launch per
+// level, warps take (gate, slot group) items of the level grid-wide.
+__global__ void __launch_bounds__(512, 2) level_kernel(const SweepParams p, int L) {
+    extern __shared__ __align__(16) float smem[];
+    const int lane = threadIdx.x & 31;
+    const int warp = threadIdx.x >> 5;
+    Env E;
+    E.s_in = smem + (size_t)warp * (size_t)(p.stage_words + 16 + 32 * (p.cstage + 1));
+    E.s_out = E.s_in + p.stage_words + 16;
+    E.s_in_a = static_cast<uint32_t>(__cvta_generic_to_shared(E.s_in));
+    E.s_out_a = static_cast<uint32_t>(__cvta_generic_to_shared(E.s_out)) + 4u * (uint32_t)lane;
+    E.scr_stride = p.n_sw * p.region_bytes;
+    E.pin_stride = p.n_sw * p.region_bytes;
+    const uint4* gd = reinterpret_cast<const uint4*>(p.gates);
+    const int g0 = __ldg(p.level_ptr + L);
+    const int64_t items = (int64_t)(__ldg(p.level_ptr + L + 1) - g0) * p.n_sw;
+    const int64_t gw = (int64_t)blockIdx.x * (blockDim.x >> 5) + warp;
+    const int64_t nwarps = (int64_t)gridDim.x * (blockDim.x >> 5);
+    for (int64_t it = gw; it < items; it += nwarps) {
+        const int gi = g0 + (int)(it / p.n_sw);
+        const int64_t i = it % p.n_sw;
+        slot_group(p, i, lane, E);
+        E.scr = p.scratch + i * p.region_bytes;
+        E.pin = p.pinned + i * p.region_bytes;
+        const float4* dt = p.dtab + (int64_t)E.kv * p.n_gates * 2;
+        eval_dispatch(p, E, __ldg(gd + 2 * gi), __ldg(gd + 2 * gi + 1), __ldg(dt + 2 * gi), __ldg(dt + 2 * gi + 1));
+    }
+}
+
+int sweep_smem_bytes(int warps_per_cta, int stage_words, int cstage) {
+    return warps_per_cta * (stage_words + 16 + 32 * (cstage + 1)) * 4;
 }
 
 cudaError_t sweep_occupancy(int warps_per_cta, int smem, int* blocks_per_sm) {
@@ -307,10 +418,24 @@ cudaError_t sweep_occupancy(int warps_per_cta, int smem, int* blocks_per_sm) {
 }
 
 cudaError_t launch_sweep(const SweepParams& p, int grid, int warps_per_cta, cudaStream_t st) {
-    const int smem = sweep_smem_bytes(warps_per_cta, p.kmax, p.W, p.cstage);
+    const int smem = sweep_smem_bytes(warps_per_cta, p.stage_words, p.cstage);
     cudaError_t e = cudaFuncSetAttribute(sweep_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
     if (e != cudaSuccess) return e;
     sweep_kernel<<<grid, warps_per_cta * 32, smem, st>>>(p);
+    return cudaGetLastError();
+}
+
+cudaError_t level_occupancy(int warps_per_cta, int smem, int* blocks_per_sm) {
+    cudaError_t e = cudaFuncSetAttribute(level_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+    if (e != cudaSuccess) return e;
+    return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, level_kernel, warps_per_cta * 32, smem);
+}
+
+cudaError_t launch_level(const SweepParams& p, int level, int grid, int warps_per_cta, cudaStream_t st) {
+    const int smem = sweep_smem_bytes(warps_per_cta, p.stage_words, p.cstage);
+    cudaError_t e = cudaFuncSetAttribute(level_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+    if (e != cudaSuccess) return e;
+    level_kernel<<<grid, warps_per_cta * 32, smem, st>>>(p, level);
     return cudaGetLastError();
 }
 
