@@ -783,11 +783,20 @@ static avfs_status run_round(avfs_ctx* ctx, Round& R, int round_idx, const int32
     if (R.grid < 1) R.grid = 1;
     if ((int)ctx->scr.size() <= round_idx) ctx->scr.resize(round_idx + 1);
     if ((int)ctx->pin.size() <= round_idx) ctx->pin.resize(round_idx + 1);
-    const int64_t scr_slots = persistent ? R.grid : R.n_sw;
-    const size_t scr_bytes = (size_t)std::max(ctx->n_scratch, 1) * scr_slots * R.region_bytes;
     const size_t pin_bytes = (size_t)std::max(ctx->n_pinned, 1) * R.n_sw * R.region_bytes;
-    CK(ctx->scr[round_idx].ensure(scr_bytes));
     CK(ctx->pin[round_idx].ensure(pin_bytes));
+    // scratch: per resident CTA (persistent sweep) or per slot group of a rerun
+    // chunk (level-parallel), chunks sized to a quarter of the free memory
+    int64_t chunk = R.n_sw;
+    const size_t per_group = (size_t)std::max(ctx->n_scratch, 1) * R.region_bytes;
+    if (!persistent) {
+        size_t free_b = 0, total_b = 0;
+        CK(cudaMemGetInfo(&free_b, &total_b));
+        const size_t budget = std::max<size_t>(free_b / 4 + ctx->scr[round_idx].n, per_group);
+        chunk = std::max<int64_t>(1, std::min<int64_t>(R.n_sw, (int64_t)(budget / per_group)));
+    }
+    const int64_t scr_slots = persistent ? R.grid : chunk;
+    CK(ctx->scr[round_idx].ensure(per_group * scr_slots));
     CK(ctx->d_ovf.ensure(std::max<int64_t>(R.n_sw, 1) * sizeof(int32_t)));
     CK(cudaMemsetAsync(ctx->d_ovf.p, 0, R.n_sw * sizeof(int32_t), ctx->stream));
     SweepParams p{};
@@ -806,6 +815,8 @@ static avfs_status run_round(avfs_ctx* ctx, Round& R, int round_idx, const int32
     p.sw_list = d_sw_list;
     p.sw_first = R.sw_first;
     p.n_sw = R.n_sw;
+    p.i_base = 0;
+    p.pin_n_sw = R.n_sw;
     p.scratch = ctx->scr[round_idx].as<uint8_t>();
     p.pinned = ctx->pin[round_idx].as<uint8_t>();
     p.region_bytes = R.region_bytes;
@@ -822,8 +833,13 @@ static avfs_status run_round(avfs_ctx* ctx, Round& R, int round_idx, const int32
         CK(launch_sweep(p, R.grid, wpc, ctx->stream));
         ctx->stats.launches++;
     } else {
-        for (int L = 0; L < ctx->depth; ++L) CK(launch_level(p, L, R.grid, wpc, ctx->stream));
-        ctx->stats.launches += ctx->depth;
+        for (int64_t c0 = 0; c0 < R.n_sw; c0 += chunk) {
+            p.i_base = c0;
+            p.n_sw = std::min<int64_t>(chunk, R.n_sw - c0);
+            p.sw_list = d_sw_list + c0;
+            for (int L = 0; L < ctx->depth; ++L) CK(launch_level(p, L, R.grid, wpc, ctx->stream));
+            ctx->stats.launches += ctx->depth;
+        }
     }
     if (timed) CK(cudaEventRecord(ctx->ev1, ctx->stream));
     if (round_idx == 0) ctx->stats.warps_per_cta = wpc;

@@ -71,7 +71,9 @@ struct SweepParams {
     // slot-warps of this run: sw = sw_list ? sw_list[i] : sw_first + i, i < n_sw
     const int32_t* __restrict__ sw_list;
     int64_t sw_first;
-    int64_t n_sw;
+    int64_t n_sw;                           // slot groups in this launch
+    int64_t i_base;                         // index of this launch's first group within the round
+    int64_t pin_n_sw;                       // slot groups in the round (pinned arena / ovf flags)
     // arenas
     uint8_t* scratch;                       // persistent: [n_scratch][gridDim.x][region]; level: [n_scratch][n_sw][region]
     uint8_t* pinned;                        // [n_pinned][n_sw][region]

@@ -278,7 +278,7 @@ __device__ __forceinline__ void eval_gate(const SweepParams& p, const Env& E, co
     }
     if (base > p.stage_words) {                        // cannot happen: each input total <= W
         __stcg(ro_hdr + lane, HDR_POISON | HDR_PREV | (y0 << 20));
-        if (lane == 0) p.ovf[E.i] = 1;
+        if (lane == 0) p.ovf[p.i_base + E.i] = 1;
         return;
     }
     {
@@ -307,7 +307,7 @@ __device__ __forceinline__ void eval_gate(const SweepParams& p, const Env& E, co
         float* dst = reinterpret_cast<float*>(ro + 128) + excl;
         for (int t = 0; t < n_out; ++t) __stcg(dst + t, E.s_out[t * 32 + lane]);
     } else if (lane == 0) {
-        p.ovf[E.i] = 1;
+        p.ovf[p.i_base + E.i] = 1;
     }
     __stcg(ro_hdr + lane, (uint32_t)min(n_out, (int)HDR_N) | (y0 << 20) | (ovf ? HDR_POISON : 0u) |
                               (prev ? HDR_PREV : 0u));
@@ -361,7 +361,7 @@ __global__ void __launch_bounds__(256, 4) sweep_kernel(const SweepParams p) {
     E.s_in_a = static_cast<uint32_t>(__cvta_generic_to_shared(E.s_in));
     E.s_out_a = static_cast<uint32_t>(__cvta_generic_to_shared(E.s_out)) + 4u * (uint32_t)lane;
     E.scr_stride = (int64_t)gridDim.x * p.region_bytes;
-    E.pin_stride = p.n_sw * p.region_bytes;
+    E.pin_stride = p.pin_n_sw * p.region_bytes;
     const uint4* gd = reinterpret_cast<const uint4*>(p.gates);
     for (int64_t i = blockIdx.x; i < p.n_sw; i += gridDim.x) {
         slot_group(p, i, lane, E);
@@ -390,7 +390,7 @@ __global__ void __launch_bounds__(512, 2) level_kernel(const SweepParams p, int 
     E.s_in_a = static_cast<uint32_t>(__cvta_generic_to_shared(E.s_in));
     E.s_out_a = static_cast<uint32_t>(__cvta_generic_to_shared(E.s_out)) + 4u * (uint32_t)lane;
     E.scr_stride = p.n_sw * p.region_bytes;
-    E.pin_stride = p.n_sw * p.region_bytes;
+    E.pin_stride = p.pin_n_sw * p.region_bytes;
     const uint4* gd = reinterpret_cast<const uint4*>(p.gates);
     const int g0 = __ldg(p.level_ptr + L);
     const int64_t items = (int64_t)(__ldg(p.level_ptr + L + 1) - g0) * p.n_sw;
@@ -401,7 +401,7 @@ __global__ void __launch_bounds__(512, 2) level_kernel(const SweepParams p, int 
         const int64_t i = it % p.n_sw;
         slot_group(p, i, lane, E);
         E.scr = p.scratch + i * p.region_bytes;
-        E.pin = p.pinned + i * p.region_bytes;
+        E.pin = p.pinned + (p.i_base + i) * p.region_bytes;
         const float4* dt = p.dtab + (int64_t)E.kv * p.n_gates * 2;
         eval_dispatch(p, E, __ldg(gd + 2 * gi), __ldg(gd + 2 * gi + 1), __ldg(dt + 2 * gi), __ldg(dt + 2 * gi + 1));
     }
