@@ -796,6 +796,8 @@ static avfs_status run_round(avfs_ctx* ctx, Round& R, int round_idx, const int32
         chunk = std::max<int64_t>(1, std::min<int64_t>(R.n_sw, (int64_t)(budget / per_group)));
     }
     const int64_t scr_slots = persistent ? R.grid : chunk;
+    if ((uint64_t)scr_slots * R.region_bytes >= (1ull << 32) || (uint64_t)R.n_sw * R.region_bytes >= (1ull << 32))
+        return fail(ctx, AVFS_ERR_NOMEM, "slot-group stride exceeds 4 GiB; restrict the slot range");
     CK(ctx->scr[round_idx].ensure(per_group * scr_slots));
     CK(ctx->d_ovf.ensure(std::max<int64_t>(R.n_sw, 1) * sizeof(int32_t)));
     CK(cudaMemsetAsync(ctx->d_ovf.p, 0, R.n_sw * sizeof(int32_t), ctx->stream));

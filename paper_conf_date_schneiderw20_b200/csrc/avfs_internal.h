@@ -17,10 +17,13 @@ constexpr uint32_t LOC_KIND = 3u << 30;
 constexpr uint32_t LOC_ID = ~LOC_KIND;
 
 // Header word of one (signal, slot) waveform (reading C1):
-constexpr uint32_t HDR_N = 0x000FFFFFu;      // transition count (exact, even on overflow)
-constexpr uint32_t HDR_INIT = 1u << 20;      // value before t = 0
-constexpr uint32_t HDR_POISON = 1u << 21;    // events not stored here or upstream
-constexpr uint32_t HDR_PREV = 1u << 22;      // would have been poisoned at the previous round's capacity
+constexpr uint32_t HDR_N = 0x00000FFFu;      // transition count (< 4096; larger counts overflow)
+constexpr int HDR_OFF_SHIFT = 12;            // bits 12..27: offset of the slot's first event in the
+constexpr uint32_t HDR_OFF = 0xFFFFu;        //   region (exclusive prefix of the counts of lanes < l)
+constexpr int HDR_INIT_SHIFT = 28;
+constexpr uint32_t HDR_INIT = 1u << 28;      // value before t = 0
+constexpr uint32_t HDR_POISON = 1u << 29;    // events not stored here or upstream
+constexpr uint32_t HDR_PREV = 1u << 30;      // would have been poisoned at the previous round's capacity
 
 // Gate descriptor, 32 B, read warp-uniformly (P:L154 step 1).
 struct alignas(16) GateDesc {

@@ -43,6 +43,33 @@ __device__ __forceinline__ void cp_async16(void* smem, const void* gmem) {
     uint32_t s = static_cast<uint32_t>(__cvta_generic_to_shared(smem));
     asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"(s), "l"(gmem) : "memory");
 }
+__device__ __forceinline__ void cp_async16_a(uint32_t s, const void* gmem) {
+    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"(s), "l"(gmem) : "memory");
+}
+// TMA bulk copy global -> shared, completion signalled on an mbarrier (tx bytes)
+__device__ __forceinline__ void tma_bulk_g2s(uint32_t dst, const void* src, uint32_t bytes, uint32_t bar) {
+    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];\n"
+                 ::"r"(dst), "l"(src), "r"(bytes), "r"(bar) : "memory");
+}
+__device__ __forceinline__ void mbar_init(uint32_t bar) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;\n" ::"r"(bar) : "memory");
+    asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
+}
+__device__ __forceinline__ void mbar_expect_tx(uint32_t bar, uint32_t bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;\n" ::"r"(bar), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint32_t bar, uint32_t phase) {
+    asm volatile(
+        "{\n .reg .pred P;\n WAIT_%=:\n"
+        " mbarrier.try_wait.parity.shared::cta.b64 P, [%0], %1;\n"
+        " @!P bra WAIT_%=;\n}\n" ::"r"(bar), "r"(phase) : "memory");
+}
+__device__ __forceinline__ void fence_proxy_async_smem() {
+    asm volatile("fence.proxy.async.shared::cta;\n" ::: "memory");
+}
+__device__ __forceinline__ void fence_proxy_async_global() {
+    asm volatile("fence.proxy.async.global;\n" ::: "memory");
+}
 __device__ __forceinline__ void cp_async_wait_all() {
     asm volatile("cp.async.wait_all;\n" ::: "memory");
 }
@@ -99,13 +126,13 @@ cudaError_t launch_delays(const DelayParams& p, cudaStream_t st) {
 }
 
 // ---------------------------------------------------------------------------
-// Per-slot merge of K sorted input event lists with the inertial filter
-// (reading C3: cancel the pending last output event iff it lies
-// strictly after the input event; C4: no reschedule on confirming events;
-// C5: ties in time are taken in ascending pin order).  Branch-free body; the
-// element after each head is prefetched from shared memory one step ahead.
-// Returns the exact output count; the first `cstage` surviving events are in
-// s_out[i*32 + lane].
+// Per-slot merge of the K sorted input event lists of a gate with the inertial
+// filter (reading C3: the pending last output event is cancelled iff
+// it lies strictly after the input event; C4: no reschedule on confirming
+// events; C5: ties in time are taken in ascending pin order).  Branch-free
+// bodies; the element after each head is prefetched from shared memory one
+// step ahead.  Returns the exact output count; the first `cstage` surviving
+// events are left in shared memory rows s_out[i][lane].
 // ---------------------------------------------------------------------------
 __device__ __forceinline__ float lds_f32(uint32_t addr) {
     float v;
@@ -116,26 +143,98 @@ __device__ __forceinline__ void sts_f32(uint32_t addr, float v) {
     asm volatile("st.shared.f32 [%0], %1;\n" ::"r"(addr), "f"(v) : "memory");
 }
 
+#define AVFS_INF __int_as_float(0x7f800000)
+
+// filter step shared by all merges: one input event at time t whose pin flip
+// gives evaluated output y; d_r / d_f = the pin's rise / fall delays.
+struct OutState {
+    int n;          // surviving output events
+    float tl;       // time of the last surviving event (-inf if it is <= every later input)
+    uint32_t proj;  // projected output value
+};
+
+__device__ __forceinline__ void filter_step(OutState& o, float t, uint32_t y, float d_r, float d_f,
+                                            uint32_t s_out_lane, int cstage) {
+    const bool change = y != o.proj;
+    const bool cancel = change && (o.tl > t);   // pending output lies after t: pulse filtered
+    const bool push = change && !cancel;
+    const float tn = t + (y ? d_r : d_f);
+    // unconditional store to the next free row (clamped): harmless unless pushed
+    sts_f32(s_out_lane + 128u * (uint32_t)min(o.n, cstage), tn);
+    o.n += push ? 1 : (cancel ? -1 : 0);
+    o.tl = push ? tn : (cancel ? -AVFS_INF : o.tl);   // after a cancel the last event is <= t
+    o.proj = y;
+}
+
+// one input (BUF / INV / any 1-input cell)
+__device__ __forceinline__ int merge1(uint32_t s_in, int c, int n, bool pi, float d_f, float d_r, uint32_t tt,
+                                     uint32_t bits, uint32_t proj, uint32_t s_out_lane, int cstage) {
+    const int e = c + n;
+    const float a0 = lds_f32(s_in + 4u * (uint32_t)c);
+    const float a1 = lds_f32(s_in + 4u * (uint32_t)(c + 1));
+    float h = n > 0 ? (pi ? 0.0f : a0) : AVFS_INF;
+    float nh = (n > 1 && !pi) ? a1 : AVFS_INF;
+    OutState o{0, -AVFS_INF, proj};
+    while (h < AVFS_INF) {
+        const float t = h;
+        ++c;
+        const float raw = lds_f32(s_in + 4u * (uint32_t)(c + 1));
+        h = nh;
+        nh = (c + 1 < e) ? raw : AVFS_INF;
+        bits ^= 1u;
+        filter_step(o, t, (tt >> bits) & 1u, d_r, d_f, s_out_lane, cstage);
+    }
+    return o.n;
+}
+
+// two inputs, hand-specialised (62 % of gates on the random DAGs)
+__device__ __forceinline__ int merge2(uint32_t s_in, int c0, int n0, bool pi0, int c1, int n1, bool pi1,
+                                     const float (&dl)[8], uint32_t tt, uint32_t bits, uint32_t proj,
+                                     uint32_t s_out_lane, int cstage) {
+    const int e0 = c0 + n0, e1 = c1 + n1;
+    float h0, h1, nh0, nh1;
+    {
+        const float a = lds_f32(s_in + 4u * (uint32_t)c0), b = lds_f32(s_in + 4u * (uint32_t)(c0 + 1));
+        const float x = lds_f32(s_in + 4u * (uint32_t)c1), z = lds_f32(s_in + 4u * (uint32_t)(c1 + 1));
+        h0 = n0 > 0 ? (pi0 ? 0.0f : a) : AVFS_INF;
+        nh0 = (n0 > 1 && !pi0) ? b : AVFS_INF;
+        h1 = n1 > 0 ? (pi1 ? 0.0f : x) : AVFS_INF;
+        nh1 = (n1 > 1 && !pi1) ? z : AVFS_INF;
+    }
+    OutState o{0, -AVFS_INF, proj};
+    for (;;) {
+        const bool p1 = h1 < h0;                 // ties: pin 0 first
+        const float t = p1 ? h1 : h0;
+        if (!(t < AVFS_INF)) break;
+        const int cn = (p1 ? c1 : c0) + 1;
+        const int en = p1 ? e1 : e0;
+        const float raw = lds_f32(s_in + 4u * (uint32_t)(cn + 1));
+        const float hn = p1 ? nh1 : nh0;
+        const float nn = (cn + 1 < en) ? raw : AVFS_INF;
+        if (p1) { h1 = hn; nh1 = nn; c1 = cn; } else { h0 = hn; nh0 = nn; c0 = cn; }
+        bits ^= p1 ? 2u : 1u;
+        filter_step(o, t, (tt >> bits) & 1u, p1 ? dl[3] : dl[1], p1 ? dl[2] : dl[0], s_out_lane, cstage);
+    }
+    return o.n;
+}
+
+// generic K (3 and 4 inputs)
 template <int K>
-__device__ __forceinline__ int merge_slot(uint32_t s_in, const int (&cb)[KMAX], const int (&n)[KMAX],
-                                          const bool (&pi)[KMAX], const float (&dl)[8], uint32_t tt,
-                                          uint32_t bits, uint32_t proj, uint32_t s_out_lane, int cstage) {
-    const float INF = __int_as_float(0x7f800000);
+__device__ __forceinline__ int merge_k(uint32_t s_in, const int (&cb)[KMAX], const int (&n)[KMAX],
+                                       const bool (&pi)[KMAX], const float (&dl)[8], uint32_t tt, uint32_t bits,
+                                       uint32_t proj, uint32_t s_out_lane, int cstage) {
     float h[K], nh[K];
     int c[K], e[K];
 #pragma unroll
     for (int q = 0; q < K; ++q) {
         c[q] = cb[q];
         e[q] = cb[q] + n[q];
-        // every address below stays inside the per-warp staging area (budget + 16 words):
-        // loads beyond a list return garbage that is replaced by INF.
         const float a0 = lds_f32(s_in + 4u * (uint32_t)c[q]);
         const float a1 = lds_f32(s_in + 4u * (uint32_t)(c[q] + 1));
-        h[q] = n[q] > 0 ? (pi[q] ? 0.0f : a0) : INF;
-        nh[q] = (n[q] > 1 && !pi[q]) ? a1 : INF;
+        h[q] = n[q] > 0 ? (pi[q] ? 0.0f : a0) : AVFS_INF;
+        nh[q] = (n[q] > 1 && !pi[q]) ? a1 : AVFS_INF;
     }
-    int n_out = 0;
-    float tl = -INF;
+    OutState o{0, -AVFS_INF, proj};
     for (;;) {
         float t = h[0];
         int pm = 0;
@@ -145,8 +244,7 @@ __device__ __forceinline__ int merge_slot(uint32_t s_in, const int (&cb)[KMAX], 
             t = lt ? h[q] : t;
             pm = lt ? q : pm;
         }
-        if (!(t < INF)) break;
-        // consume the head of pin pm; prefetch the element after its new head
+        if (!(t < AVFS_INF)) break;
         int cn = c[0], en = e[0];
         float hn = nh[0], dfp = dl[0], drp = dl[1];
 #pragma unroll
@@ -154,148 +252,132 @@ __device__ __forceinline__ int merge_slot(uint32_t s_in, const int (&cb)[KMAX], 
             if (pm == q) { cn = c[q]; en = e[q]; hn = nh[q]; dfp = dl[2 * q]; drp = dl[2 * q + 1]; }
         ++cn;
         const float raw = lds_f32(s_in + 4u * (uint32_t)(cn + 1));
-        const float nn = (cn + 1 < en) ? raw : INF;
+        const float nn = (cn + 1 < en) ? raw : AVFS_INF;
 #pragma unroll
         for (int q = 0; q < K; ++q)
             if (pm == q) { c[q] = cn; h[q] = hn; nh[q] = nn; }
         bits ^= 1u << pm;
-        const uint32_t y = (tt >> bits) & 1u;
-        const bool change = y != proj;
-        const bool cancel = change && (tl > t);     // pending output lies after t: pulse filtered
-        const bool push = change && !cancel;
-        const float tn = t + (y ? drp : dfp);
-        // unconditional store to the next free row (clamped): harmless unless pushed
-        sts_f32(s_out_lane + 128u * (uint32_t)min(n_out, cstage), tn);
-        n_out += push ? 1 : (cancel ? -1 : 0);
-        tl = push ? tn : (cancel ? -INF : tl);      // after a cancel the last event is <= t
-        proj = y;
+        filter_step(o, t, (tt >> bits) & 1u, drp, dfp, s_out_lane, cstage);
     }
-    return n_out;
-}
-
-__device__ __forceinline__ uint8_t* region_of(uint32_t loc, uint8_t* scr, int64_t scr_stride,
-                                              uint8_t* pin, int64_t pin_stride) {
-    const int64_t id = loc & LOC_ID;
-    return ((loc & LOC_KIND) == LOC_SCRATCH) ? scr + id * scr_stride : pin + id * pin_stride;
+    return o.n;
 }
 
 // Where one warp's 32 slots live for the gate being evaluated.
 struct Env {
-    uint8_t* scr;
-    int64_t scr_stride;
-    uint8_t* pin;
-    int64_t pin_stride;
-    int64_t i;           // index of the slot group in this run (overflow flag)
-    uint32_t mask;       // lanes holding a simulated slot
+    uint8_t* scr;                  // scratch row of this CTA (persistent) / slot group (level)
+    uint8_t* pin;                  // pinned row of this slot group
+    uint32_t scr_stride, pin_stride;   // bytes between buffers (< 4 GiB, checked on the host)
+    int64_t i;                     // index of the slot group in the round (overflow flag)
+    uint32_t mask;                 // lanes holding a simulated slot
     int pw, kv, lane;
-    float* s_in;         // per-warp input staging (budget + 16 words)
-    float* s_out;        // per-warp output staging (32 * (cstage + 1) words)
-    uint32_t s_in_a;     // the same, as shared-window addresses
-    uint32_t s_out_a;    // s_out + 4 * lane
+    uint32_t s_in_a;               // per-warp input staging (shared window address)
+    uint32_t s_out_a;              // per-warp output rows + 4*lane
+    uint32_t bar;                  // per-warp mbarrier for the TMA staging
+    uint32_t phase;                // its current parity
+    unsigned long long* act_kv;    // &act[0][kv]
 };
+
+__device__ __forceinline__ uint8_t* region(uint32_t loc, const Env& E) {
+    const bool scr = (loc & LOC_SCRATCH) != 0;
+    uint8_t* b = scr ? E.scr : E.pin;
+    return b + (uint64_t)(loc & LOC_ID) * (uint64_t)(scr ? E.scr_stride : E.pin_stride);
+}
 
 // One gate for one 32-slot group: input headers,
 // compact staging, merge/filter, output compaction, reductions.
 template <int K>
-__device__ __forceinline__ void eval_gate(const SweepParams& p, const Env& E, const uint4 ins, const uint4 hd,
+__device__ __forceinline__ void eval_gate(const SweepParams& p, Env& E, const uint4 ins, const uint4 hd,
                                           const float (&dl)[8]) {
     const int lane = E.lane;
     const uint32_t out_loc = hd.x, sig = hd.y;
     const uint32_t tt = hd.z & 0xffffu;
-    const uint32_t gflags = hd.z >> 24;
     const uint32_t in_loc[KMAX] = {ins.x, ins.y, ins.z, ins.w};
-    int n[KMAX], cb[KMAX];
+    // all input loads first (headers of kept/scratch waveforms, stimulus words of PIs)
+    const uint8_t* rg[KMAX];
+    uint32_t w1[KMAX], w2[KMAX];
     bool isp[KMAX];
-    const float* ev[KMAX];
+#pragma unroll
+    for (int q = 0; q < K; ++q) {
+        const uint32_t loc = in_loc[q];
+        isp[q] = (loc & LOC_KIND) == LOC_PI;
+        const uint32_t* pa = p.p1t + (size_t)(loc & LOC_ID) * (uint32_t)p.n_pw + E.pw;
+        rg[q] = region(loc, E);
+        w1[q] = __ldcg(isp[q] ? pa : reinterpret_cast<const uint32_t*>(rg[q]) + lane);
+        w2[q] = isp[q] ? __ldcg(pa + (p.p2t - p.p1t)) : 0u;
+    }
+    int n[KMAX], cb[KMAX];
     uint32_t bits = 0, pois = 0, prevp = 0;
     int sum = 0;
 #pragma unroll
     for (int q = 0; q < KMAX; ++q) {
         n[q] = 0;
         cb[q] = 0;
-        isp[q] = true;
-        ev[q] = nullptr;
         if (q < K) {
-            const uint32_t loc = in_loc[q];
-            if ((loc & LOC_KIND) == LOC_PI) {
-                const int64_t o = (int64_t)(loc & LOC_ID) * p.n_pw + E.pw;
-                const uint32_t w1 = __ldg(p.p1t + o) & E.mask;
-                const uint32_t w2 = __ldg(p.p2t + o) & E.mask;
-                bits |= ((w1 >> lane) & 1u) << q;
-                n[q] = (int)(((w1 ^ w2) >> lane) & 1u);
-            } else {
-                const uint8_t* r = region_of(loc, E.scr, E.scr_stride, E.pin, E.pin_stride);
-                const uint32_t h = ld_u32(r + 4 * lane);
-                n[q] = (int)(h & HDR_N);
-                bits |= ((h >> 20) & 1u) << q;
-                pois |= h & HDR_POISON;
-                prevp |= h & HDR_PREV;
-                isp[q] = false;
-                ev[q] = reinterpret_cast<const float*>(r + 128);
-            }
+            const uint32_t a = w1[q] & E.mask, b = w2[q] & E.mask;
+            const uint32_t h = w1[q];
+            n[q] = isp[q] ? (int)(((a ^ b) >> lane) & 1u) : (int)(h & HDR_N);
+            cb[q] = isp[q] ? 0 : (int)((h >> HDR_OFF_SHIFT) & HDR_OFF);
+            bits |= (isp[q] ? ((a >> lane) & 1u) : ((h >> HDR_INIT_SHIFT) & 1u)) << q;
+            pois |= isp[q] ? 0u : h;
+            prevp |= isp[q] ? 0u : h;
             sum += n[q];
         }
     }
     const uint32_t y0 = (tt >> bits) & 1u;
-    uint8_t* ro = region_of(out_loc, E.scr, E.scr_stride, E.pin, E.pin_stride);
+    uint8_t* ro = region(out_loc, E);
     uint32_t* ro_hdr = reinterpret_cast<uint32_t*>(ro);
     const bool first_pass = (p.prev_W == 0);
-    const bool any_prev = first_pass || __any_sync(0xffffffffu, prevp != 0);
-    if (__any_sync(0xffffffffu, pois != 0)) {          // upstream overflow: nothing valid here
-        __stcg(ro_hdr + lane, HDR_POISON | HDR_PREV | (y0 << 20));
+    const bool any_prev = first_pass || __any_sync(0xffffffffu, (prevp & HDR_PREV) != 0);
+    if (__any_sync(0xffffffffu, (pois & HDR_POISON) != 0)) {   // upstream overflow: nothing valid here
+        __stcg(ro_hdr + lane, HDR_POISON | HDR_PREV | (y0 << HDR_INIT_SHIFT));
         return;
     }
-    if (!__any_sync(0xffffffffu, sum != 0)) {          // no input event in any slot: constant output
-        __stcg(ro_hdr + lane, (y0 << 20) | (any_prev ? HDR_PREV : 0u));
+    if (!__any_sync(0xffffffffu, sum != 0)) {                   // no input event in any slot: constant output
+        __stcg(ro_hdr + lane, (y0 << HDR_INIT_SHIFT) | (any_prev ? HDR_PREV : 0u));
         return;
     }
-    // compact per-pin offsets: exclusive warp scans of the stored counts (2 pins per scan)
-    int tot[KMAX] = {0, 0, 0, 0};
+    // stage each input's compact event list into shared memory with one TMA
+    // bulk copy per input (extent = lane 31's offset + count), one mbarrier
     {
-        const uint32_t a = (uint32_t)(isp[0] ? 0 : n[0]) | ((uint32_t)(K > 1 && !isp[1] ? n[1] : 0) << 16);
-        const uint32_t ia = warp_incl_scan(a, lane);
-        const uint32_t ta = __shfl_sync(0xffffffffu, ia, 31);
-        const uint32_t ea = ia - a;
-        cb[0] = (int)(ea & 0xffffu);  tot[0] = (int)(ta & 0xffffu);
-        cb[1] = (int)(ea >> 16);      tot[1] = (int)(ta >> 16);
-        if (K > 2) {
-            const uint32_t b = (uint32_t)(isp[2] ? 0 : n[2]) | ((uint32_t)(K > 3 && !isp[3] ? n[3] : 0) << 16);
-            const uint32_t ib = warp_incl_scan(b, lane);
-            const uint32_t tb = __shfl_sync(0xffffffffu, ib, 31);
-            const uint32_t eb = ib - b;
-            cb[2] = (int)(eb & 0xffffu);  tot[2] = (int)(tb & 0xffffu);
-            cb[3] = (int)(eb >> 16);      tot[3] = (int)(tb >> 16);
-        }
-    }
-    // stage the compact input lists (16-B cp.async)
-    int base = 0;
-#pragma unroll
-    for (int q = 0; q < K; ++q) {
-        if (!isp[q]) {
-            cb[q] += base;
-            base += (tot[q] + 3) & ~3;
-        }
-    }
-    if (base > p.stage_words) {                        // cannot happen: each input total <= W
-        __stcg(ro_hdr + lane, HDR_POISON | HDR_PREV | (y0 << 20));
-        if (lane == 0) p.ovf[p.i_base + E.i] = 1;
-        return;
-    }
-    {
-        int off = 0;
+        int base = 0;
+        int ext[KMAX];
 #pragma unroll
         for (int q = 0; q < K; ++q) {
-            if (!isp[q]) {
-                const int nv = (tot[q] + 3) >> 2;
-                for (int v = lane; v < nv; v += 32) cp_async16(E.s_in + off + 4 * v, ev[q] + 4 * v);
-                off += nv * 4;
+            ext[q] = __shfl_sync(0xffffffffu, cb[q] + n[q], 31);
+            ext[q] = isp[q] ? 0 : (ext[q] + 3) & ~3;
+            cb[q] += base;
+            base += ext[q];
+        }
+        if (base > p.stage_words) {                    // cannot happen: each input extent <= W
+            __stcg(ro_hdr + lane, HDR_POISON | HDR_PREV | (y0 << HDR_INIT_SHIFT));
+            if (lane == 0) p.ovf[p.i_base + E.i] = 1;
+            return;
+        }
+        if (base > 0) {
+            if (lane == 0) {
+                fence_proxy_async_smem();              // earlier generic reads of the staging area
+                mbar_expect_tx(E.bar, 4u * (uint32_t)base);
+                uint32_t dst = E.s_in_a;
+#pragma unroll
+                for (int q = 0; q < K; ++q) {
+                    if (ext[q] > 0) tma_bulk_g2s(dst, rg[q] + 128, 4u * (uint32_t)ext[q], E.bar);
+                    dst += 4u * (uint32_t)ext[q];
+                }
             }
+            mbar_wait(E.bar, E.phase);
+            E.phase ^= 1u;
         }
     }
-    cp_async_wait_all();
-    __syncwarp();
-    const int n_out = merge_slot<K>(E.s_in_a, cb, n, isp, dl, tt, bits, y0, E.s_out_a, p.cstage);
-    // output: scan, overflow ballot, direct compact stores
+    int n_out;
+    if (K == 1) {
+        n_out = merge1(E.s_in_a, cb[0], n[0], isp[0], dl[0], dl[1], tt, bits, y0, E.s_out_a, p.cstage);
+    } else if (K == 2) {
+        n_out = merge2(E.s_in_a, cb[0], n[0], isp[0], cb[1], n[1], isp[K > 1 ? 1 : 0], dl, tt, bits, y0,
+                       E.s_out_a, p.cstage);
+    } else {
+        n_out = merge_k<K>(E.s_in_a, cb, n, isp, dl, tt, bits, y0, E.s_out_a, p.cstage);
+    }
+    // output: scan, overflow ballot, compact stores row by row (warp-uniform loop)
     const uint32_t incl = warp_incl_scan((uint32_t)n_out, lane);
     const uint32_t total = __shfl_sync(0xffffffffu, incl, 31);
     const uint32_t excl = incl - (uint32_t)n_out;
@@ -304,19 +386,23 @@ __device__ __forceinline__ void eval_gate(const SweepParams& p, const Env& E, co
     if (!first_pass)
         prev = any_prev || __any_sync(0xffffffffu, n_out > p.prev_cstage) || total > (uint32_t)p.prev_W;
     if (!ovf) {
+        const int rows = (int)__reduce_max_sync(0xffffffffu, (uint32_t)n_out);
         float* dst = reinterpret_cast<float*>(ro + 128) + excl;
-        for (int t = 0; t < n_out; ++t) __stcg(dst + t, E.s_out[t * 32 + lane]);
+        for (int r = 0; r < rows; ++r) {
+            const float v = lds_f32(E.s_out_a + 128u * (uint32_t)r);
+            if (r < n_out) __stcg(dst + r, v);
+        }
     } else if (lane == 0) {
         p.ovf[p.i_base + E.i] = 1;
     }
-    __stcg(ro_hdr + lane, (uint32_t)min(n_out, (int)HDR_N) | (y0 << 20) | (ovf ? HDR_POISON : 0u) |
-                              (prev ? HDR_PREV : 0u));
+    __stcg(ro_hdr + lane, (uint32_t)min(n_out, (int)HDR_N) | ((excl & HDR_OFF) << HDR_OFF_SHIFT) |
+                              (y0 << HDR_INIT_SHIFT) | (ovf ? HDR_POISON : 0u) | (prev ? HDR_PREV : 0u));
     // activity (reading C15) and latest PO arrival: counted once per
     // slot across overflow rounds (where prev && !ovf)
     if (!ovf && prev) {
-        if (lane == 0 && total) atomicAdd(p.act + (int64_t)sig * p.n_vdd + E.kv, (unsigned long long)total);
-        if (gflags & 1u) {
-            const float last = n_out ? E.s_out[(n_out - 1) * 32 + lane] : 0.0f;
+        if (lane == 0 && total) atomicAdd(E.act_kv + (size_t)sig * (uint32_t)p.n_vdd, (unsigned long long)total);
+        if (hd.z & (1u << 24)) {
+            const float last = n_out ? lds_f32(E.s_out_a + 128u * (uint32_t)(n_out - 1)) : 0.0f;
             const uint32_t m = __reduce_max_sync(0xffffffffu, __float_as_uint(last));
             if (lane == 0 && m) atomicMax(p.latest + E.kv, m);
         }
@@ -324,7 +410,7 @@ __device__ __forceinline__ void eval_gate(const SweepParams& p, const Env& E, co
     __syncwarp();
 }
 
-__device__ __forceinline__ void eval_dispatch(const SweepParams& p, const Env& E, const uint4 ins, const uint4 hd,
+__device__ __forceinline__ void eval_dispatch(const SweepParams& p, Env& E, const uint4 ins, const uint4 hd,
                                               const float4 d0, const float4 d1) {
     const float dl[8] = {d0.x, d0.y, d0.z, d0.w, d1.x, d1.y, d1.z, d1.w};
     switch ((hd.z >> 16) & 0xffu) {
@@ -345,34 +431,42 @@ __device__ __forceinline__ void slot_group(const SweepParams& p, int64_t i, int 
     E.mask = __ballot_sync(0xffffffffu, valid);
     E.i = i;
     E.lane = lane;
+    E.act_kv = p.act + E.kv;
+    E.pin = p.pinned + (p.i_base + i) * p.region_bytes;
+}
+
+__device__ __forceinline__ void warp_smem(const SweepParams& p, int warp, int lane, Env& E) {
+    extern __shared__ __align__(16) float smem[];
+    float* s_in = smem + (size_t)warp * (size_t)(p.stage_words + 16 + 32 * (p.cstage + 1));
+    E.s_in_a = static_cast<uint32_t>(__cvta_generic_to_shared(s_in));
+    E.s_out_a = E.s_in_a + 4u * (uint32_t)(p.stage_words + 16) + 4u * (uint32_t)lane;
+    E.bar = E.s_in_a + 4u * (uint32_t)(p.stage_words + 14);   // 8-B aligned, past any over-read
+    E.phase = 0;
+    if (lane == 0) mbar_init(E.bar);
+    __syncwarp();
 }
 
 // Persistent level sweep (pass 0): one CTA owns one 32-slot group at a time
-// and walks all levels with a CTA barrier between levels.  Gate
-// descriptors and delays are prefetched one gate ahead.
+// and walks all levels with a CTA barrier between levels.
 __global__ void __launch_bounds__(256, 4) sweep_kernel(const SweepParams p) {
-    extern __shared__ __align__(16) float smem[];
     const int lane = threadIdx.x & 31;
     const int warp = threadIdx.x >> 5;
     const int nw = blockDim.x >> 5;
     Env E;
-    E.s_in = smem + (size_t)warp * (size_t)(p.stage_words + 16 + 32 * (p.cstage + 1));
-    E.s_out = E.s_in + p.stage_words + 16;
-    E.s_in_a = static_cast<uint32_t>(__cvta_generic_to_shared(E.s_in));
-    E.s_out_a = static_cast<uint32_t>(__cvta_generic_to_shared(E.s_out)) + 4u * (uint32_t)lane;
-    E.scr_stride = (int64_t)gridDim.x * p.region_bytes;
-    E.pin_stride = p.pin_n_sw * p.region_bytes;
+    warp_smem(p, warp, lane, E);
+    E.scr_stride = (uint32_t)(gridDim.x * p.region_bytes);
+    E.pin_stride = (uint32_t)(p.pin_n_sw * p.region_bytes);
     const uint4* gd = reinterpret_cast<const uint4*>(p.gates);
     for (int64_t i = blockIdx.x; i < p.n_sw; i += gridDim.x) {
         slot_group(p, i, lane, E);
         E.scr = p.scratch + (int64_t)blockIdx.x * p.region_bytes;
-        E.pin = p.pinned + i * p.region_bytes;
         const float4* dt = p.dtab + (int64_t)E.kv * p.n_gates * 2;
         for (int L = 0; L < p.depth; ++L) {
             const int g_end = __ldg(p.level_ptr + L + 1);
             for (int gi = __ldg(p.level_ptr + L) + warp; gi < g_end; gi += nw)
                 eval_dispatch(p, E, __ldg(gd + 2 * gi), __ldg(gd + 2 * gi + 1), __ldg(dt + 2 * gi),
                               __ldg(dt + 2 * gi + 1));
+            fence_proxy_async_global();   // this level's stores -> next levels' TMA reads
             __syncthreads();
         }
     }
@@ -381,16 +475,12 @@ __global__ void __launch_bounds__(256, 4) sweep_kernel(const SweepParams p) {
 // Level-parallel variant for overflow reruns (few slot groups): one launch per
 // level, warps take (gate, slot group) items of the level grid-wide.
 __global__ void __launch_bounds__(512, 2) level_kernel(const SweepParams p, int L) {
-    extern __shared__ __align__(16) float smem[];
     const int lane = threadIdx.x & 31;
     const int warp = threadIdx.x >> 5;
     Env E;
-    E.s_in = smem + (size_t)warp * (size_t)(p.stage_words + 16 + 32 * (p.cstage + 1));
-    E.s_out = E.s_in + p.stage_words + 16;
-    E.s_in_a = static_cast<uint32_t>(__cvta_generic_to_shared(E.s_in));
-    E.s_out_a = static_cast<uint32_t>(__cvta_generic_to_shared(E.s_out)) + 4u * (uint32_t)lane;
-    E.scr_stride = p.n_sw * p.region_bytes;
-    E.pin_stride = p.pin_n_sw * p.region_bytes;
+    warp_smem(p, warp, lane, E);
+    E.scr_stride = (uint32_t)(p.n_sw * p.region_bytes);
+    E.pin_stride = (uint32_t)(p.pin_n_sw * p.region_bytes);
     const uint4* gd = reinterpret_cast<const uint4*>(p.gates);
     const int g0 = __ldg(p.level_ptr + L);
     const int64_t items = (int64_t)(__ldg(p.level_ptr + L + 1) - g0) * p.n_sw;
@@ -401,10 +491,10 @@ __global__ void __launch_bounds__(512, 2) level_kernel(const SweepParams p, int 
         const int64_t i = it % p.n_sw;
         slot_group(p, i, lane, E);
         E.scr = p.scratch + i * p.region_bytes;
-        E.pin = p.pinned + (p.i_base + i) * p.region_bytes;
         const float4* dt = p.dtab + (int64_t)E.kv * p.n_gates * 2;
         eval_dispatch(p, E, __ldg(gd + 2 * gi), __ldg(gd + 2 * gi + 1), __ldg(dt + 2 * gi), __ldg(dt + 2 * gi + 1));
     }
+    fence_proxy_async_global();   // stores -> next launch's TMA reads
 }
 
 int sweep_smem_bytes(int warps_per_cta, int stage_words, int cstage) {
@@ -570,10 +660,9 @@ __global__ void gather_kernel(const GatherParams p) {
         const uint32_t* hdr = reinterpret_cast<const uint32_t*>(base);
         const uint32_t h = hdr[lane];
         if (h & HDR_POISON) { atomicOr(p.bad, 2); return; }
-        init = (h >> 20) & 1u;
+        init = (h >> HDR_INIT_SHIFT) & 1u;
         n = (int)(h & HDR_N);
-        int off = 0;
-        for (int l = 0; l < lane; ++l) off += (int)(hdr[l] & HDR_N);
+        const int off = (int)((h >> HDR_OFF_SHIFT) & HDR_OFF);
         const float* ev = reinterpret_cast<const float*>(base + 128) + off;
         if (tout) for (int i = 0; i < p.cap; ++i) tout[i] = i < n ? ev[i] : 0.0f;
     }
