@@ -18,6 +18,7 @@
 #include <cmath>
 #include <cstdarg>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <string>
 #include <unordered_map>
@@ -742,7 +743,7 @@ avfs_status avfs_set_options(avfs_ctx* ctx, const avfs_options* o) {
     if (o->capacity < 1 || o->capacity > 1024) return fail(ctx, AVFS_ERR_ARG, "capacity must be in [1, 1024]");
     if (o->quantum_ps < 0 || !std::isfinite(o->quantum_ps)) return fail(ctx, AVFS_ERR_ARG, "bad quantum");
     if (o->n_probe < 0 || (o->n_probe > 0 && !o->probe_sig)) return fail(ctx, AVFS_ERR_ARG, "bad probes");
-    if (o->warps_per_cta < 0 || o->warps_per_cta > 16) return fail(ctx, AVFS_ERR_ARG, "warps_per_cta in [0,16]");
+    if (o->warps_per_cta < 0 || o->warps_per_cta > 32) return fail(ctx, AVFS_ERR_ARG, "warps_per_cta in [0,32]");
     if (o->max_rerun_rounds < 0 || o->max_rerun_rounds > 6) return fail(ctx, AVFS_ERR_ARG, "max_rerun_rounds in [0,6]");
     std::vector<int32_t> pr(o->probe_sig, o->probe_sig + o->n_probe);
     if (ctx->net_loaded)
@@ -767,9 +768,9 @@ avfs_status avfs_sync(avfs_ctx* ctx) {
 static avfs_status run_round(avfs_ctx* ctx, Round& R, int round_idx, const int32_t* d_sw_list, int32_t prev_W,
                              int32_t prev_cstage, bool timed) {
     const bool persistent = (round_idx == 0);
-    // launch bounds: sweep_kernel 256 threads (4 CTAs/SM), level_kernel 512 threads
-    int wpc = ctx->opt.warps_per_cta > 0 ? ctx->opt.warps_per_cta : (persistent ? 8 : 16);
-    wpc = std::min(wpc, persistent ? 8 : 16);
+    // launch bounds: sweep_kernel up to 1024 threads, level_kernel 512 threads
+    int wpc = ctx->opt.warps_per_cta > 0 ? ctx->opt.warps_per_cta : (persistent ? 32 : 16);
+    wpc = std::min(wpc, persistent ? 32 : 16);
     const int stage_words = ctx->kmax * R.W;
     int smem = sweep_smem_bytes(wpc, stage_words, R.cstage);
     while (wpc > 1 && smem > 227 * 1024) smem = sweep_smem_bytes(--wpc, stage_words, R.cstage);
@@ -830,6 +831,10 @@ static avfs_status run_round(avfs_ctx* ctx, Round& R, int round_idx, const int32
     p.act = ctx->d_act.as<unsigned long long>();
     p.latest = ctx->d_latest.as<unsigned int>();
     p.ovf = ctx->d_ovf.as<int32_t>();
+    {
+        const char* dg = getenv("AVFS_DYN_GRAB");
+        p.dyn_grab = dg ? atoi(dg) : 0;   // measured: static striding is as fast at 32 warps/CTA
+    }
     if (timed) CK(cudaEventRecord(ctx->ev0, ctx->stream));
     if (persistent) {
         CK(launch_sweep(p, R.grid, wpc, ctx->stream));

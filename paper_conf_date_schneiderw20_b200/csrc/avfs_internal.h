@@ -85,6 +85,7 @@ struct SweepParams {
     int32_t stage_words;                    // per-warp input staging: max fan-in x W
     int32_t cstage;                         // per-slot capacity (2*C)
     int32_t prev_W, prev_cstage;            // previous round (0: first pass)
+    int32_t dyn_grab;                       // 1: warps take gates of a level from a shared counter
     // outputs
     unsigned long long* act;                // [n_signals][n_vdd]
     unsigned int* latest;                   // [n_vdd] float bits (non-negative)

@@ -437,7 +437,7 @@ __device__ __forceinline__ void slot_group(const SweepParams& p, int64_t i, int 
 
 __device__ __forceinline__ void warp_smem(const SweepParams& p, int warp, int lane, Env& E) {
     extern __shared__ __align__(16) float smem[];
-    float* s_in = smem + (size_t)warp * (size_t)(p.stage_words + 16 + 32 * (p.cstage + 1));
+    float* s_in = smem + 4 + (size_t)warp * (size_t)(p.stage_words + 16 + 32 * (p.cstage + 1));
     E.s_in_a = static_cast<uint32_t>(__cvta_generic_to_shared(s_in));
     E.s_out_a = E.s_in_a + 4u * (uint32_t)(p.stage_words + 16) + 4u * (uint32_t)lane;
     E.bar = E.s_in_a + 4u * (uint32_t)(p.stage_words + 14);   // 8-B aligned, past any over-read
@@ -448,7 +448,9 @@ __device__ __forceinline__ void warp_smem(const SweepParams& p, int warp, int la
 
 // Persistent level sweep (pass 0): one CTA owns one 32-slot group at a time
 // and walks all levels with a CTA barrier between levels.
-__global__ void __launch_bounds__(256, 4) sweep_kernel(const SweepParams p) {
+__global__ void __launch_bounds__(1024, 1) sweep_kernel(const SweepParams p) {
+    extern __shared__ __align__(16) float smem[];
+    int* ctr = reinterpret_cast<int*>(smem);             // two level counters (16-B header)
     const int lane = threadIdx.x & 31;
     const int warp = threadIdx.x >> 5;
     const int nw = blockDim.x >> 5;
@@ -461,11 +463,27 @@ __global__ void __launch_bounds__(256, 4) sweep_kernel(const SweepParams p) {
         slot_group(p, i, lane, E);
         E.scr = p.scratch + (int64_t)blockIdx.x * p.region_bytes;
         const float4* dt = p.dtab + (int64_t)E.kv * p.n_gates * 2;
+        if (threadIdx.x == 0) ctr[0] = __ldg(p.level_ptr);
+        __syncthreads();
         for (int L = 0; L < p.depth; ++L) {
             const int g_end = __ldg(p.level_ptr + L + 1);
-            for (int gi = __ldg(p.level_ptr + L) + warp; gi < g_end; gi += nw)
-                eval_dispatch(p, E, __ldg(gd + 2 * gi), __ldg(gd + 2 * gi + 1), __ldg(dt + 2 * gi),
-                              __ldg(dt + 2 * gi + 1));
+            if (p.dyn_grab) {
+                // warps take gates of the level from a shared counter (load balance)
+                int* c = ctr + (L & 1);
+                for (;;) {
+                    int gi = 0;
+                    if (lane == 0) gi = atomicAdd(c, 1);
+                    gi = __shfl_sync(0xffffffffu, gi, 0);
+                    if (gi >= g_end) break;
+                    eval_dispatch(p, E, __ldg(gd + 2 * gi), __ldg(gd + 2 * gi + 1), __ldg(dt + 2 * gi),
+                                  __ldg(dt + 2 * gi + 1));
+                }
+                if (threadIdx.x == 0 && L + 1 < p.depth) ctr[(L + 1) & 1] = g_end;
+            } else {
+                for (int gi = __ldg(p.level_ptr + L) + warp; gi < g_end; gi += nw)
+                    eval_dispatch(p, E, __ldg(gd + 2 * gi), __ldg(gd + 2 * gi + 1), __ldg(dt + 2 * gi),
+                                  __ldg(dt + 2 * gi + 1));
+            }
             fence_proxy_async_global();   // this level's stores -> next levels' TMA reads
             __syncthreads();
         }
@@ -498,7 +516,7 @@ __global__ void __launch_bounds__(512, 2) level_kernel(const SweepParams p, int 
 }
 
 int sweep_smem_bytes(int warps_per_cta, int stage_words, int cstage) {
-    return warps_per_cta * (stage_words + 16 + 32 * (cstage + 1)) * 4;
+    return 16 + warps_per_cta * (stage_words + 16 + 32 * (cstage + 1)) * 4;
 }
 
 cudaError_t sweep_occupancy(int warps_per_cta, int smem, int* blocks_per_sm) {
