@@ -59,7 +59,7 @@ struct Round {
     int64_t n_sw = 0;
     int64_t sw_first = 0;            // pass 0: contiguous range
     std::vector<int32_t> sws;        // reruns: explicit list
-    int32_t capacity = 0, W = 0, cstage = 0;
+    int32_t capacity = 0, W = 0, cstage = 0, stage_words = 0;
     int64_t region_bytes = 0;
     int32_t grid = 0;
 };
@@ -771,7 +771,9 @@ static avfs_status run_round(avfs_ctx* ctx, Round& R, int round_idx, const int32
     // launch bounds: sweep_kernel up to 1024 threads, level_kernel 512 threads
     int wpc = ctx->opt.warps_per_cta > 0 ? ctx->opt.warps_per_cta : (persistent ? 32 : 16);
     wpc = std::min(wpc, persistent ? 32 : 16);
-    const int stage_words = ctx->kmax * R.W;
+    // input staging budget per warp: min(max fan-in, 2) x W words (more -> overflow, rerun)
+    const int stage_words = std::min(ctx->kmax, 2) * R.W;
+    R.stage_words = stage_words;
     int smem = sweep_smem_bytes(wpc, stage_words, R.cstage);
     while (wpc > 1 && smem > 227 * 1024) smem = sweep_smem_bytes(--wpc, stage_words, R.cstage);
     if (smem > 227 * 1024) return fail(ctx, AVFS_ERR_CAPACITY, "capacity %d needs %d B shared memory per warp", R.capacity, smem);
@@ -828,6 +830,7 @@ static avfs_status run_round(avfs_ctx* ctx, Round& R, int round_idx, const int32
     p.cstage = R.cstage;
     p.prev_W = prev_W;
     p.prev_cstage = prev_cstage;
+    p.prev_stage_words = prev_W ? std::min(ctx->kmax, 2) * prev_W : 0;
     p.act = ctx->d_act.as<unsigned long long>();
     p.latest = ctx->d_latest.as<unsigned int>();
     p.ovf = ctx->d_ovf.as<int32_t>();

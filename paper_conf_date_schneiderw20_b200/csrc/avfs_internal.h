@@ -82,9 +82,10 @@ struct SweepParams {
     uint8_t* pinned;                        // [n_pinned][n_sw][region]
     int64_t region_bytes;
     int32_t W;                              // event capacity per region (32*C)
-    int32_t stage_words;                    // per-warp input staging: max fan-in x W
+    int32_t stage_words;                    // per-warp input staging: min(max fan-in, 2) x W
     int32_t cstage;                         // per-slot capacity (2*C)
     int32_t prev_W, prev_cstage;            // previous round (0: first pass)
+    int32_t prev_stage_words;               // previous round's staging budget (0: first pass)
     int32_t dyn_grab;                       // 1: warps take gates of a level from a shared counter
     // outputs
     unsigned long long* act;                // [n_signals][n_vdd]

@@ -338,6 +338,7 @@ __device__ __forceinline__ void eval_gate(const SweepParams& p, Env& E, const ui
     }
     // stage each input's compact event list into shared memory with one TMA
     // bulk copy per input (extent = lane 31's offset + count), one mbarrier
+    int stage_base = 0;
     {
         int base = 0;
         int ext[KMAX];
@@ -348,11 +349,12 @@ __device__ __forceinline__ void eval_gate(const SweepParams& p, Env& E, const ui
             cb[q] += base;
             base += ext[q];
         }
-        if (base > p.stage_words) {                    // cannot happen: each input extent <= W
+        if (base > p.stage_words) {                    // inputs exceed this capacity's staging: rerun
             __stcg(ro_hdr + lane, HDR_POISON | HDR_PREV | (y0 << HDR_INIT_SHIFT));
             if (lane == 0) p.ovf[p.i_base + E.i] = 1;
             return;
         }
+        stage_base = base;
         if (base > 0) {
             if (lane == 0) {
                 fence_proxy_async_smem();              // earlier generic reads of the staging area
@@ -384,7 +386,8 @@ __device__ __forceinline__ void eval_gate(const SweepParams& p, Env& E, const ui
     const bool ovf = __any_sync(0xffffffffu, n_out > p.cstage) || total > (uint32_t)p.W;
     bool prev = true;
     if (!first_pass)
-        prev = any_prev || __any_sync(0xffffffffu, n_out > p.prev_cstage) || total > (uint32_t)p.prev_W;
+        prev = any_prev || stage_base > p.prev_stage_words || __any_sync(0xffffffffu, n_out > p.prev_cstage) ||
+               total > (uint32_t)p.prev_W;
     if (!ovf) {
         const int rows = (int)__reduce_max_sync(0xffffffffu, (uint32_t)n_out);
         float* dst = reinterpret_cast<float*>(ro + 128) + excl;
