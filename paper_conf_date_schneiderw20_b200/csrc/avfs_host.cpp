@@ -121,7 +121,7 @@ struct avfs_ctx {
     bool dev_net_valid = false, dev_vdd_valid = false;
     DevBuf d_gates, d_ddesc, d_dtab, d_coef, d_level_ptr, d_vdd, d_p1, d_p2, d_p1t, d_p2t, d_act, d_latest, d_ovf,
         d_err, d_list[2], d_count, d_swround, d_swindex, g_loc, g_init, g_count, g_times, g_bad;
-    std::vector<DevBuf> scr, pin;     // per round
+    std::vector<DevBuf> arena;        // per round: [buffer][slot group][region]
     int32_t* h_pinned = nullptr;      // small pinned host buffer (count, err)
     cudaEvent_t ev0 = nullptr, ev1 = nullptr;
 
@@ -309,6 +309,14 @@ avfs_status build_plan(avfs_ctx* ctx) {
     return AVFS_OK;
 }
 
+// arena buffer of a location: PIs 0..n_pi-1, kept signals next, scratch last
+uint32_t buffer_id(const avfs_ctx* ctx, uint32_t loc) {
+    const uint32_t kind = loc & LOC_KIND, id = loc & LOC_ID;
+    if (kind == LOC_PI) return id;
+    if (kind == LOC_PINNED) return (uint32_t)ctx->n_pi + id;
+    return (uint32_t)(ctx->n_pi + ctx->n_pinned) + id;
+}
+
 avfs_status upload_netlist(avfs_ctx* ctx) {
     if (ctx->dev_net_valid) return AVFS_OK;
     const int32_t G = ctx->n_gates;
@@ -321,8 +329,8 @@ avfs_status upload_netlist(avfs_ctx* ctx) {
         std::memset(&d, 0, sizeof d);
         std::memset(&e, 0, sizeof e);
         const int k = (int)(ctx->fanin_ptr[g + 1] - ctx->fanin_ptr[g]);
-        for (int p = 0; p < KMAX; ++p) d.in_loc[p] = p < k ? ctx->loc[ctx->fanin_sig[ctx->fanin_ptr[g] + p]] : 0u;
-        d.out_loc = ctx->loc[ctx->n_pi + g];
+        for (int p = 0; p < KMAX; ++p) d.in_loc[p] = p < k ? buffer_id(ctx, ctx->loc[ctx->fanin_sig[ctx->fanin_ptr[g] + p]]) : 0u;
+        d.out_loc = buffer_id(ctx, ctx->loc[ctx->n_pi + g]);
         d.sig = (uint32_t)(ctx->n_pi + g);
         d.ttk = (uint32_t)ctx->cell_tt[ctx->gate_cell[g]] | ((uint32_t)k << 16) |
                 ((ctx->is_po[ctx->n_pi + g] ? 1u : 0u) << 24);
@@ -784,24 +792,11 @@ static avfs_status run_round(avfs_ctx* ctx, Round& R, int round_idx, const int32
     const int64_t resident = (int64_t)ctx->n_sm * bps;
     R.grid = (int32_t)(persistent ? std::min<int64_t>(R.n_sw, resident) : resident);
     if (R.grid < 1) R.grid = 1;
-    if ((int)ctx->scr.size() <= round_idx) ctx->scr.resize(round_idx + 1);
-    if ((int)ctx->pin.size() <= round_idx) ctx->pin.resize(round_idx + 1);
-    const size_t pin_bytes = (size_t)std::max(ctx->n_pinned, 1) * R.n_sw * R.region_bytes;
-    CK(ctx->pin[round_idx].ensure(pin_bytes));
-    // scratch: per resident CTA (persistent sweep) or per slot group of a rerun
-    // chunk (level-parallel), chunks sized to a quarter of the free memory
-    int64_t chunk = R.n_sw;
-    const size_t per_group = (size_t)std::max(ctx->n_scratch, 1) * R.region_bytes;
-    if (!persistent) {
-        size_t free_b = 0, total_b = 0;
-        CK(cudaMemGetInfo(&free_b, &total_b));
-        const size_t budget = std::max<size_t>(free_b / 4 + ctx->scr[round_idx].n, per_group);
-        chunk = std::max<int64_t>(1, std::min<int64_t>(R.n_sw, (int64_t)(budget / per_group)));
-    }
-    const int64_t scr_slots = persistent ? R.grid : chunk;
-    if ((uint64_t)scr_slots * R.region_bytes >= (1ull << 32) || (uint64_t)R.n_sw * R.region_bytes >= (1ull << 32))
+    if ((int)ctx->arena.size() <= round_idx) ctx->arena.resize(round_idx + 1);
+    const int64_t n_buf = (int64_t)ctx->n_pi + ctx->n_pinned + ctx->n_scratch;
+    if ((uint64_t)R.n_sw * R.region_bytes >= (1ull << 32))
         return fail(ctx, AVFS_ERR_NOMEM, "slot-group stride exceeds 4 GiB; restrict the slot range");
-    CK(ctx->scr[round_idx].ensure(per_group * scr_slots));
+    CK(ctx->arena[round_idx].ensure((size_t)std::max<int64_t>(n_buf, 1) * R.n_sw * R.region_bytes));
     CK(ctx->d_ovf.ensure(std::max<int64_t>(R.n_sw, 1) * sizeof(int32_t)));
     CK(cudaMemsetAsync(ctx->d_ovf.p, 0, R.n_sw * sizeof(int32_t), ctx->stream));
     SweepParams p{};
@@ -822,8 +817,7 @@ static avfs_status run_round(avfs_ctx* ctx, Round& R, int round_idx, const int32
     p.n_sw = R.n_sw;
     p.i_base = 0;
     p.pin_n_sw = R.n_sw;
-    p.scratch = ctx->scr[round_idx].as<uint8_t>();
-    p.pinned = ctx->pin[round_idx].as<uint8_t>();
+    p.arena = ctx->arena[round_idx].as<uint8_t>();
     p.region_bytes = R.region_bytes;
     p.W = R.W;
     p.stage_words = stage_words;
@@ -838,18 +832,15 @@ static avfs_status run_round(avfs_ctx* ctx, Round& R, int round_idx, const int32
         const char* dg = getenv("AVFS_DYN_GRAB");
         p.dyn_grab = dg ? atoi(dg) : 0;   // measured: static striding is as fast at 32 warps/CTA
     }
+    CK(launch_pi_regions(p, ctx->n_pi, ctx->stream));   // materialise the PI waveforms of this round
+    ctx->stats.launches++;
     if (timed) CK(cudaEventRecord(ctx->ev0, ctx->stream));
     if (persistent) {
         CK(launch_sweep(p, R.grid, wpc, ctx->stream));
         ctx->stats.launches++;
     } else {
-        for (int64_t c0 = 0; c0 < R.n_sw; c0 += chunk) {
-            p.i_base = c0;
-            p.n_sw = std::min<int64_t>(chunk, R.n_sw - c0);
-            p.sw_list = d_sw_list + c0;
-            for (int L = 0; L < ctx->depth; ++L) CK(launch_level(p, L, R.grid, wpc, ctx->stream));
-            ctx->stats.launches += ctx->depth;
-        }
+        for (int L = 0; L < ctx->depth; ++L) CK(launch_level(p, L, R.grid, wpc, ctx->stream));
+        ctx->stats.launches += ctx->depth;
     }
     if (timed) CK(cudaEventRecord(ctx->ev1, ctx->stream));
     if (round_idx == 0) ctx->stats.warps_per_cta = wpc;
@@ -975,7 +966,7 @@ avfs_status avfs_simulate(avfs_ctx* ctx, void* cuda_stream) {
     ctx->stats.n_scratch_buffers = ctx->n_scratch;
     ctx->stats.n_pinned = ctx->n_pinned;
     int64_t ab = 0;
-    for (size_t r = 0; r < ctx->rounds.size(); ++r) ab += (int64_t)(ctx->scr[r].n + ctx->pin[r].n);
+    for (size_t r = 0; r < ctx->rounds.size(); ++r) ab += (int64_t)ctx->arena[r].n;
     ctx->stats.arena_bytes = ab;
     ctx->stats.sim_ms = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
     return AVFS_OK;
@@ -1015,6 +1006,7 @@ static avfs_status gather(avfs_ctx* ctx, int32_t n_sig, const int32_t* sig, int6
         sl[i] = ctx->loc[sig[i]];
         if ((sl[i] & LOC_KIND) == LOC_SCRATCH)
             return fail(ctx, AVFS_ERR_ARG, "signal %d is not kept (not a PO/probe; use keep_all)", sig[i]);
+        if ((sl[i] & LOC_KIND) == LOC_PINNED) sl[i] = LOC_PINNED | buffer_id(ctx, sl[i]);
     }
     if (n_sig == 0 || n_slots == 0) return AVFS_OK;
     const int32_t n_pw = (int32_t)((ctx->n_pairs + 31) / 32);
@@ -1055,7 +1047,7 @@ static avfs_status gather(avfs_ctx* ctx, int32_t n_sig, const int32_t* sig, int6
     g.sw_round = ctx->d_swround.as<int32_t>();
     g.sw_index = ctx->d_swindex.as<int32_t>();
     for (size_t r = 0; r < ctx->rounds.size(); ++r)
-        g.rounds[r] = GatherRound{ctx->pin[r].as<uint8_t>(), ctx->rounds[r].region_bytes, ctx->rounds[r].n_sw};
+        g.rounds[r] = GatherRound{ctx->arena[r].as<uint8_t>(), ctx->rounds[r].region_bytes, ctx->rounds[r].n_sw};
     g.cap = times ? cap : 0;
     g.init = ctx->g_init.as<uint8_t>();
     g.count = ctx->g_count.as<int32_t>();
@@ -1096,21 +1088,20 @@ avfs_status avfs_get_stats(avfs_ctx* ctx, avfs_stats* st) {
     CHECK_CTX();
     if (!st) return fail(ctx, AVFS_ERR_ARG, "null output");
     if (!ctx->sim_done) return fail(ctx, AVFS_ERR_STATE, "simulate first");
-    // algorithmic bytes of the sweep: every gate output
-    // is written once and read once per reading pin, 4 B header per slot plus
-    // 4 B per transition; PI words: 8 B per 32 slots per reading pin.
+    // algorithmic bytes of the sweep: every signal's
+    // waveform (PIs included) is written once and read once per reading pin,
+    // 4 B header per slot plus 4 B per transition.
     const int32_t V = (int32_t)ctx->vdd.size();
     const int32_t S = ctx->n_pi + ctx->n_gates;
     std::vector<uint64_t> act((size_t)S * V);
     CK(cudaMemcpy(act.data(), ctx->d_act.p, act.size() * 8, cudaMemcpyDeviceToHost));
     const double slots = (double)(ctx->sim_end - ctx->sim_first);
     double b = 0;
-    for (int32_t s = ctx->n_pi; s < S; ++s) {
+    for (int32_t s = 0; s < S; ++s) {
         uint64_t a = 0;
         for (int32_t k = 0; k < V; ++k) a += act[(size_t)s * V + k];
         b += (1.0 + (double)ctx->fanout[s]) * (4.0 * slots + 4.0 * (double)a);
     }
-    for (int32_t i = 0; i < ctx->n_pi; ++i) b += (double)ctx->fanout[i] * slots / 4.0;
     ctx->stats.alg_bytes = (int64_t)b;
     *st = ctx->stats;
     return AVFS_OK;

@@ -77,9 +77,8 @@ struct SweepParams {
     int64_t n_sw;                           // slot groups in this launch
     int64_t i_base;                         // index of this launch's first group within the round
     int64_t pin_n_sw;                       // slot groups in the round (pinned arena / ovf flags)
-    // arenas
-    uint8_t* scratch;                       // persistent: [n_scratch][gridDim.x][region]; level: [n_scratch][n_sw][region]
-    uint8_t* pinned;                        // [n_pinned][n_sw][region]
+    // arena of the round: [buffer][pin_n_sw][region]; buffers = PIs, kept signals, scratch
+    uint8_t* arena;
     int64_t region_bytes;
     int32_t W;                              // event capacity per region (32*C)
     int32_t stage_words;                    // per-warp input staging: min(max fan-in, 2) x W
@@ -100,6 +99,7 @@ cudaError_t launch_delays(const DelayParams& p, cudaStream_t st);
 cudaError_t launch_sweep(const SweepParams& p, int grid, int warps_per_cta, cudaStream_t st);
 cudaError_t level_occupancy(int warps_per_cta, int smem, int* blocks_per_sm);
 cudaError_t launch_level(const SweepParams& p, int level, int grid, int warps_per_cta, cudaStream_t st);
+cudaError_t launch_pi_regions(const SweepParams& p, int32_t n_pi, cudaStream_t st);
 cudaError_t launch_expand(const uint32_t* p1, const uint32_t* p2, int64_t n_pairs, int32_t words,
                           int32_t n_pi, int32_t n_pw, uint32_t* p1t, uint32_t* p2t, cudaStream_t st);
 cudaError_t launch_pi_activity(const uint32_t* p1t, const uint32_t* p2t, int32_t n_pi, int32_t n_pw,

@@ -167,13 +167,13 @@ __device__ __forceinline__ void filter_step(OutState& o, float t, uint32_t y, fl
 }
 
 // one input (BUF / INV / any 1-input cell)
-__device__ __forceinline__ int merge1(uint32_t s_in, int c, int n, bool pi, float d_f, float d_r, uint32_t tt,
+__device__ __forceinline__ int merge1(uint32_t s_in, int c, int n, float d_f, float d_r, uint32_t tt,
                                      uint32_t bits, uint32_t proj, uint32_t s_out_lane, int cstage) {
     const int e = c + n;
     const float a0 = lds_f32(s_in + 4u * (uint32_t)c);
     const float a1 = lds_f32(s_in + 4u * (uint32_t)(c + 1));
-    float h = n > 0 ? (pi ? 0.0f : a0) : AVFS_INF;
-    float nh = (n > 1 && !pi) ? a1 : AVFS_INF;
+    float h = n > 0 ? a0 : AVFS_INF;
+    float nh = n > 1 ? a1 : AVFS_INF;
     OutState o{0, -AVFS_INF, proj};
     while (h < AVFS_INF) {
         const float t = h;
@@ -188,7 +188,7 @@ __device__ __forceinline__ int merge1(uint32_t s_in, int c, int n, bool pi, floa
 }
 
 // two inputs, hand-specialised (62 % of gates on the random DAGs)
-__device__ __forceinline__ int merge2(uint32_t s_in, int c0, int n0, bool pi0, int c1, int n1, bool pi1,
+__device__ __forceinline__ int merge2(uint32_t s_in, int c0, int n0, int c1, int n1,
                                      const float (&dl)[8], uint32_t tt, uint32_t bits, uint32_t proj,
                                      uint32_t s_out_lane, int cstage) {
     const int e0 = c0 + n0, e1 = c1 + n1;
@@ -196,10 +196,10 @@ __device__ __forceinline__ int merge2(uint32_t s_in, int c0, int n0, bool pi0, i
     {
         const float a = lds_f32(s_in + 4u * (uint32_t)c0), b = lds_f32(s_in + 4u * (uint32_t)(c0 + 1));
         const float x = lds_f32(s_in + 4u * (uint32_t)c1), z = lds_f32(s_in + 4u * (uint32_t)(c1 + 1));
-        h0 = n0 > 0 ? (pi0 ? 0.0f : a) : AVFS_INF;
-        nh0 = (n0 > 1 && !pi0) ? b : AVFS_INF;
-        h1 = n1 > 0 ? (pi1 ? 0.0f : x) : AVFS_INF;
-        nh1 = (n1 > 1 && !pi1) ? z : AVFS_INF;
+        h0 = n0 > 0 ? a : AVFS_INF;
+        nh0 = n0 > 1 ? b : AVFS_INF;
+        h1 = n1 > 0 ? x : AVFS_INF;
+        nh1 = n1 > 1 ? z : AVFS_INF;
     }
     OutState o{0, -AVFS_INF, proj};
     for (;;) {
@@ -221,7 +221,7 @@ __device__ __forceinline__ int merge2(uint32_t s_in, int c0, int n0, bool pi0, i
 // generic K (3 and 4 inputs)
 template <int K>
 __device__ __forceinline__ int merge_k(uint32_t s_in, const int (&cb)[KMAX], const int (&n)[KMAX],
-                                       const bool (&pi)[KMAX], const float (&dl)[8], uint32_t tt, uint32_t bits,
+                                       const float (&dl)[8], uint32_t tt, uint32_t bits,
                                        uint32_t proj, uint32_t s_out_lane, int cstage) {
     float h[K], nh[K];
     int c[K], e[K];
@@ -231,8 +231,8 @@ __device__ __forceinline__ int merge_k(uint32_t s_in, const int (&cb)[KMAX], con
         e[q] = cb[q] + n[q];
         const float a0 = lds_f32(s_in + 4u * (uint32_t)c[q]);
         const float a1 = lds_f32(s_in + 4u * (uint32_t)(c[q] + 1));
-        h[q] = n[q] > 0 ? (pi[q] ? 0.0f : a0) : AVFS_INF;
-        nh[q] = (n[q] > 1 && !pi[q]) ? a1 : AVFS_INF;
+        h[q] = n[q] > 0 ? a0 : AVFS_INF;
+        nh[q] = n[q] > 1 ? a1 : AVFS_INF;
     }
     OutState o{0, -AVFS_INF, proj};
     for (;;) {
@@ -262,14 +262,14 @@ __device__ __forceinline__ int merge_k(uint32_t s_in, const int (&cb)[KMAX], con
     return o.n;
 }
 
-// Where one warp's 32 slots live for the gate being evaluated.
+// Where one warp's 32 slots live for the gate being evaluated.  All regions
+// of a round live in one arena [buffer][slot group][region] (buffers: PIs,
+// kept signals, scratch), so a region address is one multiply-add.
 struct Env {
-    uint8_t* scr;                  // scratch row of this CTA (persistent) / slot group (level)
-    uint8_t* pin;                  // pinned row of this slot group
-    uint32_t scr_stride, pin_stride;   // bytes between buffers (< 4 GiB, checked on the host)
+    uint8_t* row;                  // arena + i * region_bytes
+    uint32_t stride;               // bytes between buffers = n_sw * region_bytes (< 4 GiB, checked on host)
     int64_t i;                     // index of the slot group in the round (overflow flag)
-    uint32_t mask;                 // lanes holding a simulated slot
-    int pw, kv, lane;
+    int kv, lane;
     uint32_t s_in_a;               // per-warp input staging (shared window address)
     uint32_t s_out_a;              // per-warp output rows + 4*lane
     uint32_t bar;                  // per-warp mbarrier for the TMA staging
@@ -277,10 +277,8 @@ struct Env {
     unsigned long long* act_kv;    // &act[0][kv]
 };
 
-__device__ __forceinline__ uint8_t* region(uint32_t loc, const Env& E) {
-    const bool scr = (loc & LOC_SCRATCH) != 0;
-    uint8_t* b = scr ? E.scr : E.pin;
-    return b + (uint64_t)(loc & LOC_ID) * (uint64_t)(scr ? E.scr_stride : E.pin_stride);
+__device__ __forceinline__ uint8_t* region(uint32_t buf, const Env& E) {
+    return E.row + (uint64_t)buf * (uint64_t)E.stride;
 }
 
 // One gate for one 32-slot group: input headers,
@@ -292,18 +290,13 @@ __device__ __forceinline__ void eval_gate(const SweepParams& p, Env& E, const ui
     const uint32_t out_loc = hd.x, sig = hd.y;
     const uint32_t tt = hd.z & 0xffffu;
     const uint32_t in_loc[KMAX] = {ins.x, ins.y, ins.z, ins.w};
-    // all input loads first (headers of kept/scratch waveforms, stimulus words of PIs)
+    // all input header loads first (one coalesced 128-B row per input)
     const uint8_t* rg[KMAX];
-    uint32_t w1[KMAX], w2[KMAX];
-    bool isp[KMAX];
+    uint32_t hw[KMAX];
 #pragma unroll
     for (int q = 0; q < K; ++q) {
-        const uint32_t loc = in_loc[q];
-        isp[q] = (loc & LOC_KIND) == LOC_PI;
-        const uint32_t* pa = p.p1t + (size_t)(loc & LOC_ID) * (uint32_t)p.n_pw + E.pw;
-        rg[q] = region(loc, E);
-        w1[q] = __ldcg(isp[q] ? pa : reinterpret_cast<const uint32_t*>(rg[q]) + lane);
-        w2[q] = isp[q] ? __ldcg(pa + (p.p2t - p.p1t)) : 0u;
+        rg[q] = region(in_loc[q], E);
+        hw[q] = __ldcg(reinterpret_cast<const uint32_t*>(rg[q]) + lane);
     }
     int n[KMAX], cb[KMAX];
     uint32_t bits = 0, pois = 0, prevp = 0;
@@ -313,13 +306,12 @@ __device__ __forceinline__ void eval_gate(const SweepParams& p, Env& E, const ui
         n[q] = 0;
         cb[q] = 0;
         if (q < K) {
-            const uint32_t a = w1[q] & E.mask, b = w2[q] & E.mask;
-            const uint32_t h = w1[q];
-            n[q] = isp[q] ? (int)(((a ^ b) >> lane) & 1u) : (int)(h & HDR_N);
-            cb[q] = isp[q] ? 0 : (int)((h >> HDR_OFF_SHIFT) & HDR_OFF);
-            bits |= (isp[q] ? ((a >> lane) & 1u) : ((h >> HDR_INIT_SHIFT) & 1u)) << q;
-            pois |= isp[q] ? 0u : h;
-            prevp |= isp[q] ? 0u : h;
+            const uint32_t h = hw[q];
+            n[q] = (int)(h & HDR_N);
+            cb[q] = (int)((h >> HDR_OFF_SHIFT) & HDR_OFF);
+            bits |= ((h >> HDR_INIT_SHIFT) & 1u) << q;
+            pois |= h;
+            prevp |= h;
             sum += n[q];
         }
     }
@@ -345,7 +337,7 @@ __device__ __forceinline__ void eval_gate(const SweepParams& p, Env& E, const ui
 #pragma unroll
         for (int q = 0; q < K; ++q) {
             ext[q] = __shfl_sync(0xffffffffu, cb[q] + n[q], 31);
-            ext[q] = isp[q] ? 0 : (ext[q] + 3) & ~3;
+            ext[q] = (ext[q] + 3) & ~3;
             cb[q] += base;
             base += ext[q];
         }
@@ -372,12 +364,11 @@ __device__ __forceinline__ void eval_gate(const SweepParams& p, Env& E, const ui
     }
     int n_out;
     if (K == 1) {
-        n_out = merge1(E.s_in_a, cb[0], n[0], isp[0], dl[0], dl[1], tt, bits, y0, E.s_out_a, p.cstage);
+        n_out = merge1(E.s_in_a, cb[0], n[0], dl[0], dl[1], tt, bits, y0, E.s_out_a, p.cstage);
     } else if (K == 2) {
-        n_out = merge2(E.s_in_a, cb[0], n[0], isp[0], cb[1], n[1], isp[K > 1 ? 1 : 0], dl, tt, bits, y0,
-                       E.s_out_a, p.cstage);
+        n_out = merge2(E.s_in_a, cb[0], n[0], cb[1], n[1], dl, tt, bits, y0, E.s_out_a, p.cstage);
     } else {
-        n_out = merge_k<K>(E.s_in_a, cb, n, isp, dl, tt, bits, y0, E.s_out_a, p.cstage);
+        n_out = merge_k<K>(E.s_in_a, cb, n, dl, tt, bits, y0, E.s_out_a, p.cstage);
     }
     // output: scan, overflow ballot, compact stores row by row (warp-uniform loop)
     const uint32_t incl = warp_incl_scan((uint32_t)n_out, lane);
@@ -427,15 +418,10 @@ __device__ __forceinline__ void eval_dispatch(const SweepParams& p, Env& E, cons
 __device__ __forceinline__ void slot_group(const SweepParams& p, int64_t i, int lane, Env& E) {
     const int64_t sw = p.sw_list ? (int64_t)p.sw_list[i] : p.sw_first + i;
     E.kv = (int)(sw / p.n_pw);
-    E.pw = (int)(sw % p.n_pw);
-    const int64_t j = (int64_t)E.pw * 32 + lane;
-    const int64_t pub = (int64_t)E.kv * p.n_pairs + j;
-    const bool valid = j < p.n_pairs && pub >= p.slot_first && pub < p.slot_end;
-    E.mask = __ballot_sync(0xffffffffu, valid);
     E.i = i;
     E.lane = lane;
     E.act_kv = p.act + E.kv;
-    E.pin = p.pinned + (p.i_base + i) * p.region_bytes;
+    E.row = p.arena + (p.i_base + i) * p.region_bytes;
 }
 
 __device__ __forceinline__ void warp_smem(const SweepParams& p, int warp, int lane, Env& E) {
@@ -459,12 +445,10 @@ __global__ void __launch_bounds__(1024, 1) sweep_kernel(const SweepParams p) {
     const int nw = blockDim.x >> 5;
     Env E;
     warp_smem(p, warp, lane, E);
-    E.scr_stride = (uint32_t)(gridDim.x * p.region_bytes);
-    E.pin_stride = (uint32_t)(p.pin_n_sw * p.region_bytes);
+    E.stride = (uint32_t)(p.pin_n_sw * p.region_bytes);
     const uint4* gd = reinterpret_cast<const uint4*>(p.gates);
     for (int64_t i = blockIdx.x; i < p.n_sw; i += gridDim.x) {
         slot_group(p, i, lane, E);
-        E.scr = p.scratch + (int64_t)blockIdx.x * p.region_bytes;
         const float4* dt = p.dtab + (int64_t)E.kv * p.n_gates * 2;
         if (threadIdx.x == 0) ctr[0] = __ldg(p.level_ptr);
         __syncthreads();
@@ -500,8 +484,7 @@ __global__ void __launch_bounds__(512, 2) level_kernel(const SweepParams p, int 
     const int warp = threadIdx.x >> 5;
     Env E;
     warp_smem(p, warp, lane, E);
-    E.scr_stride = (uint32_t)(p.n_sw * p.region_bytes);
-    E.pin_stride = (uint32_t)(p.pin_n_sw * p.region_bytes);
+    E.stride = (uint32_t)(p.pin_n_sw * p.region_bytes);
     const uint4* gd = reinterpret_cast<const uint4*>(p.gates);
     const int g0 = __ldg(p.level_ptr + L);
     const int64_t items = (int64_t)(__ldg(p.level_ptr + L + 1) - g0) * p.n_sw;
@@ -511,11 +494,41 @@ __global__ void __launch_bounds__(512, 2) level_kernel(const SweepParams p, int 
         const int gi = g0 + (int)(it / p.n_sw);
         const int64_t i = it % p.n_sw;
         slot_group(p, i, lane, E);
-        E.scr = p.scratch + i * p.region_bytes;
         const float4* dt = p.dtab + (int64_t)E.kv * p.n_gates * 2;
         eval_dispatch(p, E, __ldg(gd + 2 * gi), __ldg(gd + 2 * gi + 1), __ldg(dt + 2 * gi), __ldg(dt + 2 * gi + 1));
     }
     fence_proxy_async_global();   // stores -> next launch's TMA reads
+}
+
+// Materialise PI waveforms of a round's slot groups (reading C2: one event at
+// t = 0 iff p1 != p2) as regions of buffers 0..n_pi-1: one warp per (PI, group).
+__global__ void pi_regions_kernel(const SweepParams p, int32_t n_pi) {
+    const int lane = threadIdx.x & 31;
+    const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    if (gw >= (int64_t)n_pi * p.pin_n_sw) return;
+    const int pi = (int)(gw / p.pin_n_sw);
+    const int64_t i = gw % p.pin_n_sw;
+    const int64_t sw = p.sw_list ? (int64_t)p.sw_list[i] : p.sw_first + i;
+    const int kv = (int)(sw / p.n_pw), pw = (int)(sw % p.n_pw);
+    const int64_t j = (int64_t)pw * 32 + lane;
+    const int64_t pub = (int64_t)kv * p.n_pairs + j;
+    const bool valid = j < p.n_pairs && pub >= p.slot_first && pub < p.slot_end;
+    const uint32_t mask = __ballot_sync(0xffffffffu, valid);
+    const uint32_t w1 = p.p1t[(int64_t)pi * p.n_pw + pw] & mask;
+    const uint32_t w2 = p.p2t[(int64_t)pi * p.n_pw + pw] & mask;
+    const uint32_t tog = w1 ^ w2;
+    const uint32_t n = (tog >> lane) & 1u;
+    const uint32_t off = __popc(tog & ((1u << lane) - 1u));
+    uint8_t* r = p.arena + ((int64_t)pi * p.pin_n_sw + i) * p.region_bytes;
+    reinterpret_cast<uint32_t*>(r)[lane] = n | (off << HDR_OFF_SHIFT) | (((w1 >> lane) & 1u) << HDR_INIT_SHIFT);
+    reinterpret_cast<float*>(r + 128)[lane] = 0.0f;
+}
+
+cudaError_t launch_pi_regions(const SweepParams& p, int32_t n_pi, cudaStream_t st) {
+    const int64_t threads = (int64_t)n_pi * p.pin_n_sw * 32;
+    if (threads == 0) return cudaSuccess;
+    pi_regions_kernel<<<(unsigned)((threads + 255) / 256), 256, 0, st>>>(p, n_pi);
+    return cudaGetLastError();
 }
 
 int sweep_smem_bytes(int warps_per_cta, int stage_words, int cstage) {

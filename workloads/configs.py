@@ -68,7 +68,7 @@ def make_config(i: int, n_pairs: int | None = None, n_vdd: int | None = None,
     elif i in (3, 4, 5):
         G, PI, PO, L, P0, V0, cap = {
             3: (30_000, 1452, 1512, 60, 4096, 16, 8),
-            4: (200_000, 6663, 6672, 80, 2048, 32, 8),
+            4: (200_000, 6663, 6672, 80, 2048, 32, 12),   # pilot: C = 8 overflows 42/2048 groups
             5: (2_000_000, 50_000, 50_000, 120, 1024, 51, 4),
         }[i]
         G = max(64, int(G * scale))
