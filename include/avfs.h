@@ -191,6 +191,31 @@ avfs_status avfs_get_waveforms(avfs_ctx *ctx, int32_t n_sig, const int32_t *sig,
                                int64_t slot0, int64_t n_slots, int32_t cap,
                                uint8_t *init, int32_t *count, float *times);
 
+/* NEXT-1 -- capture / test-response analysis (P:L141 step 4 "test
+ * responses"; the frequency half of AVFS).  Every primary output
+ * of every simulated pair j is sampled at the capture time t_clk[k] of its
+ * operating point k: value(t) = init xor (#{t_i <= t} mod 2) (reading C1).
+ * Pair j fails at k if some PO's captured value differs from its settled
+ * (final) value.  Its slack is t_clk[k] - (last PO transition time), or
+ * t_clk[k] if no PO switches.
+ *   t_clk[n_vdd]               capture time per operating point, ps
+ *   fail_pairs[n_vdd]          failing simulated pairs per point
+ *   fail_po[n_po][n_vdd]       failing pairs per PO (PO order of the netlist); may be NULL
+ *   slack_hist[n_vdd][n_bins]  slack histogram, bin b = [lo + b w, lo + (b+1) w),
+ *                              values outside clamp to the first / last bin; may be NULL
+ *   fail_bits[n_slots_sim]     1 byte per simulated public slot (in slot order of the
+ *                              simulated range), 1 = fails; may be NULL
+ * Runs on the device over the kept PO waveforms of the last simulate.       */
+avfs_status avfs_capture(avfs_ctx *ctx, const float *t_clk, int32_t n_bins, float lo_ps,
+                         float width_ps, uint32_t *fail_pairs, uint32_t *fail_po,
+                         uint32_t *slack_hist, uint8_t *fail_bits);
+
+/* NEXT-4 -- switching energy per operating point (P:L37 power estimation):
+ * out[k] = 1/2 sum_g act[g][k] * c_load(g) * v_k^2, in fJ (c_load in fF from
+ * the netlist, v in V), summed over the simulated pairs.  Gate outputs only
+ * (primary inputs are driven externally).  Computed on the device.        */
+avfs_status avfs_get_switching_energy(avfs_ctx *ctx, double *out_fJ);
+
 typedef struct {
     int64_t evals;               /* gates x simulated slots                  */
     int64_t slots, slot_warps;   /* simulated slots / 32-slot groups         */

@@ -24,7 +24,7 @@ EXPORTS = [
     "avfs_set_operating_points", "avfs_set_stimuli", "avfs_set_slot_range",
     "avfs_set_options", "avfs_default_options", "avfs_simulate", "avfs_sync",
     "avfs_get_activity", "avfs_get_latest_arrival", "avfs_get_final_values",
-    "avfs_get_waveforms", "avfs_get_stats",
+    "avfs_get_waveforms", "avfs_get_stats", "avfs_capture", "avfs_get_switching_energy",
 ]
 
 
@@ -97,6 +97,8 @@ def load_library(path: str = LIB_PATH):
             "avfs_get_final_values": ([P, I32, P, I64, I64, P], C.c_int),
             "avfs_get_waveforms": ([P, I32, P, I64, I64, I32, P, P, P], C.c_int),
             "avfs_get_stats": ([P, P], C.c_int),
+            "avfs_capture": ([P, P, I32, C.c_float, C.c_float, P, P, P, P], C.c_int),
+            "avfs_get_switching_energy": ([P, P], C.c_int),
         }
         for name, (args, res) in sig.items():
             f = getattr(lib, name)
@@ -279,6 +281,27 @@ class Context:
                                              _p(init), _p(count), _p(times)))
         return init, count, times[:, :, :cap]
 
+    def capture(self, t_clk, n_bins=64, lo_ps=-500.0, width_ps=25.0):
+        """NEXT-1: sample every PO at t_clk[k]; returns dict with fail_pairs [n_vdd],
+        fail_po [n_po][n_vdd], slack_hist [n_vdd][n_bins], fail_bits [n_sim_slots]."""
+        t = _c(t_clk, np.float32)
+        V = self.n_vdd
+        n_po = int(self.netlist_info()["n_po"])
+        st = self.stats()
+        fp = np.zeros(V, np.uint32)
+        fpo = np.zeros((max(n_po, 1), V), np.uint32)
+        hist = np.zeros((V, n_bins), np.uint32)
+        bits = np.zeros(max(int(st["slots"]), 1), np.uint8)
+        self._ck(self.lib.avfs_capture(self.h, _p(t), int(n_bins), float(lo_ps), float(width_ps), _p(fp), _p(fpo),
+                                       _p(hist), _p(bits)))
+        return {"fail_pairs": fp, "fail_po": fpo[:n_po], "slack_hist": hist, "fail_bits": bits[:int(st["slots"])]}
+
+    def switching_energy(self) -> np.ndarray:
+        """NEXT-4: 1/2 sum act * c_load * v^2 per operating point, fJ."""
+        out = np.zeros(self.n_vdd, np.float64)
+        self._ck(self.lib.avfs_get_switching_energy(self.h, _p(out)))
+        return out
+
     def stats(self) -> dict:
         st = avfs_stats()
         self._ck(self.lib.avfs_get_stats(self.h, C.byref(st)))
@@ -290,7 +313,7 @@ def load_workload(ctx: Context, netlist, library, stimuli, vdd):
     ctx.load_library(library.names, library.n_inputs, library.tt, library.deg_v, library.deg_c,
                      library.beta, library.v_min, library.v_max, library.c_min, library.c_max)
     ctx.load_netlist(netlist.n_pi, netlist.gate_cell, netlist.fanin_ptr, netlist.fanin_sig,
-                     netlist.d_nom, netlist.c_load if library.deg_c > 0 else None, netlist.po_sig)
+                     netlist.d_nom, netlist.c_load, netlist.po_sig)
     ctx.set_operating_points(vdd)
     if stimuli is not None:
         ctx.set_stimuli(stimuli.p1, stimuli.p2)

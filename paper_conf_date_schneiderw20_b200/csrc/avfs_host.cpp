@@ -119,7 +119,7 @@ struct avfs_ctx {
 
     // device state
     bool dev_net_valid = false, dev_vdd_valid = false;
-    DevBuf d_gates, d_ddesc, d_dtab, d_coef, d_level_ptr, d_vdd, d_p1, d_p2, d_p1t, d_p2t, d_act, d_latest, d_ovf,
+    DevBuf d_gates, d_ddesc, d_dtab, d_coef, d_cload, d_energy, c_loc, c_tclk, c_slot, c_out, d_level_ptr, d_vdd, d_p1, d_p2, d_p1t, d_p2t, d_act, d_latest, d_ovf,
         d_err, d_list[2], d_count, d_swround, d_swindex, g_loc, g_init, g_count, g_times, g_bad;
     std::vector<DevBuf> arena;        // per round: [buffer][slot group][region]
     int32_t* h_pinned = nullptr;      // small pinned host buffer (count, err)
@@ -347,6 +347,8 @@ avfs_status upload_netlist(avfs_ctx* ctx) {
     CK(ctx->d_coef.ensure(std::max<size_t>(ctx->coef.size(), 1) * sizeof(double)));
     if (!ctx->coef.empty())
         CK(cudaMemcpy(ctx->d_coef.p, ctx->coef.data(), ctx->coef.size() * sizeof(double), cudaMemcpyHostToDevice));
+    CK(ctx->d_cload.ensure((size_t)std::max<int32_t>(G, 1) * sizeof(double)));
+    CK(cudaMemcpy(ctx->d_cload.p, ctx->c_load.data(), (size_t)G * sizeof(double), cudaMemcpyHostToDevice));
     CK(ctx->d_level_ptr.ensure(ctx->level_ptr.size() * sizeof(int32_t)));
     CK(cudaMemcpy(ctx->d_level_ptr.p, ctx->level_ptr.data(), ctx->level_ptr.size() * sizeof(int32_t),
                   cudaMemcpyHostToDevice));
@@ -992,6 +994,29 @@ avfs_status avfs_get_latest_arrival(avfs_ctx* ctx, float* out) {
     return AVFS_OK;
 }
 
+// device map slot group -> (round holding its final data, index in that round)
+static avfs_status ensure_round_map(avfs_ctx* ctx) {
+    const int32_t n_pw = (int32_t)((ctx->n_pairs + 31) / 32);
+    const int64_t n_sw_total = (int64_t)n_pw * ctx->vdd.size();
+    if (!ctx->map_valid) {
+        std::vector<int32_t> rnd(n_sw_total, -1), idx(n_sw_total, 0);
+        for (size_t r = 0; r < ctx->rounds.size(); ++r) {
+            const Round& R = ctx->rounds[r];
+            for (int64_t i = 0; i < R.n_sw; ++i) {
+                const int64_t sw = R.sws.empty() ? R.sw_first + i : R.sws[i];
+                rnd[sw] = (int32_t)r;
+                idx[sw] = (int32_t)i;
+            }
+        }
+        CK(ctx->d_swround.ensure(n_sw_total * 4));
+        CK(ctx->d_swindex.ensure(n_sw_total * 4));
+        CK(cudaMemcpy(ctx->d_swround.p, rnd.data(), n_sw_total * 4, cudaMemcpyHostToDevice));
+        CK(cudaMemcpy(ctx->d_swindex.p, idx.data(), n_sw_total * 4, cudaMemcpyHostToDevice));
+        ctx->map_valid = true;
+    }
+    return AVFS_OK;
+}
+
 static avfs_status gather(avfs_ctx* ctx, int32_t n_sig, const int32_t* sig, int64_t slot0, int64_t n_slots,
                           int32_t cap, uint8_t* init, int32_t* count, float* times) {
     if (!ctx->sim_done) return fail(ctx, AVFS_ERR_STATE, "simulate first");
@@ -1011,21 +1036,9 @@ static avfs_status gather(avfs_ctx* ctx, int32_t n_sig, const int32_t* sig, int6
     if (n_sig == 0 || n_slots == 0) return AVFS_OK;
     const int32_t n_pw = (int32_t)((ctx->n_pairs + 31) / 32);
     const int64_t n_sw_total = (int64_t)n_pw * ctx->vdd.size();
-    if (!ctx->map_valid) {
-        std::vector<int32_t> rnd(n_sw_total, -1), idx(n_sw_total, 0);
-        for (size_t r = 0; r < ctx->rounds.size(); ++r) {
-            const Round& R = ctx->rounds[r];
-            for (int64_t i = 0; i < R.n_sw; ++i) {
-                const int64_t sw = R.sws.empty() ? R.sw_first + i : R.sws[i];
-                rnd[sw] = (int32_t)r;
-                idx[sw] = (int32_t)i;
-            }
-        }
-        CK(ctx->d_swround.ensure(n_sw_total * 4));
-        CK(ctx->d_swindex.ensure(n_sw_total * 4));
-        CK(cudaMemcpy(ctx->d_swround.p, rnd.data(), n_sw_total * 4, cudaMemcpyHostToDevice));
-        CK(cudaMemcpy(ctx->d_swindex.p, idx.data(), n_sw_total * 4, cudaMemcpyHostToDevice));
-        ctx->map_valid = true;
+    {
+        avfs_status ms = ensure_round_map(ctx);
+        if (ms != AVFS_OK) return ms;
     }
     const size_t n = (size_t)n_sig * n_slots;
     CK(ctx->g_loc.ensure(n_sig * 4));
@@ -1082,6 +1095,85 @@ avfs_status avfs_get_waveforms(avfs_ctx* ctx, int32_t n_sig, const int32_t* sig,
     CHECK_CTX();
     if (!init || !count || (cap > 0 && !times)) return fail(ctx, AVFS_ERR_ARG, "null output");
     return gather(ctx, n_sig, sig, slot0, n_slots, cap, init, count, cap > 0 ? times : nullptr);
+}
+
+avfs_status avfs_capture(avfs_ctx* ctx, const float* t_clk, int32_t n_bins, float lo_ps, float width_ps,
+                         uint32_t* fail_pairs, uint32_t* fail_po, uint32_t* slack_hist, uint8_t* fail_bits) {
+    CHECK_CTX();
+    if (!ctx->sim_done) return fail(ctx, AVFS_ERR_STATE, "simulate first");
+    if (!t_clk || !fail_pairs) return fail(ctx, AVFS_ERR_ARG, "null t_clk / fail_pairs");
+    if (slack_hist && (n_bins < 1 || !(width_ps > 0))) return fail(ctx, AVFS_ERR_ARG, "bad histogram bins");
+    if (ctx->rounds.size() > 8) return fail(ctx, AVFS_ERR_STATE, "too many rounds");
+    avfs_status ms = ensure_round_map(ctx);
+    if (ms != AVFS_OK) return ms;
+    const int32_t V = (int32_t)ctx->vdd.size();
+    const int32_t n_po = (int32_t)ctx->po.size();
+    const int32_t n_pw = (int32_t)((ctx->n_pairs + 31) / 32);
+    const Round& R0 = ctx->rounds[0];
+    const int64_t n_sw = R0.n_sw, n_slots = ctx->sim_end - ctx->sim_first;
+    std::vector<uint32_t> loc(std::max(n_po, 1));
+    for (int32_t o = 0; o < n_po; ++o) {
+        const uint32_t l = ctx->loc[ctx->po[o]];
+        loc[o] = (l & LOC_KIND) == LOC_PI ? l : (LOC_PINNED | buffer_id(ctx, l));
+    }
+    const size_t nb = slack_hist ? (size_t)n_bins : 0;
+    // device scratch: loc | t_clk | slot_fail, slot_last | fail_po, fail_pairs, hist | fail_bits
+    CK(ctx->c_loc.ensure(loc.size() * 4));
+    CK(ctx->c_tclk.ensure((size_t)V * 4));
+    CK(ctx->c_slot.ensure((size_t)n_sw * 32 * 8));
+    const size_t out_words = (size_t)n_po * V + V + (size_t)V * nb;
+    CK(ctx->c_out.ensure(out_words * 4 + (size_t)n_slots + 16));
+    CK(cudaMemcpy(ctx->c_loc.p, loc.data(), loc.size() * 4, cudaMemcpyHostToDevice));
+    CK(cudaMemcpy(ctx->c_tclk.p, t_clk, (size_t)V * 4, cudaMemcpyHostToDevice));
+    CK(cudaMemsetAsync(ctx->c_slot.p, 0, (size_t)n_sw * 32 * 8, ctx->stream));
+    CK(cudaMemsetAsync(ctx->c_out.p, 0, out_words * 4, ctx->stream));
+    CaptureParams p{};
+    p.po_loc = ctx->c_loc.as<uint32_t>();
+    p.n_po = n_po;
+    p.n_vdd = V;
+    p.t_clk = ctx->c_tclk.as<float>();
+    p.sw_lo = R0.sw_first;
+    p.n_sw = n_sw;
+    p.n_pairs = ctx->n_pairs;
+    p.n_pw = n_pw;
+    p.slot_first = ctx->sim_first;
+    p.slot_end = ctx->sim_end;
+    p.p1t = ctx->d_p1t.as<uint32_t>();
+    p.p2t = ctx->d_p2t.as<uint32_t>();
+    p.sw_round = ctx->d_swround.as<int32_t>();
+    p.sw_index = ctx->d_swindex.as<int32_t>();
+    for (size_t r = 0; r < ctx->rounds.size(); ++r)
+        p.rounds[r] = GatherRound{ctx->arena[r].as<uint8_t>(), ctx->rounds[r].region_bytes, ctx->rounds[r].n_sw};
+    p.slot_fail = ctx->c_slot.as<uint32_t>();
+    p.slot_last = ctx->c_slot.as<uint32_t>() + (size_t)n_sw * 32;
+    p.fail_po = ctx->c_out.as<uint32_t>();
+    p.fail_pairs = p.fail_po + (size_t)n_po * V;
+    p.hist = slack_hist ? p.fail_pairs + V : nullptr;
+    p.n_bins = std::max(n_bins, 1);
+    p.lo = lo_ps;
+    p.width = width_ps > 0 ? width_ps : 1.0f;
+    p.fail_bits = fail_bits ? reinterpret_cast<uint8_t*>(p.fail_pairs + V + (size_t)V * nb) : nullptr;
+    CK(launch_capture(p, ctx->stream));
+    CK(cudaMemcpyAsync(fail_pairs, p.fail_pairs, (size_t)V * 4, cudaMemcpyDeviceToHost, ctx->stream));
+    if (fail_po && n_po) CK(cudaMemcpyAsync(fail_po, p.fail_po, (size_t)n_po * V * 4, cudaMemcpyDeviceToHost, ctx->stream));
+    if (slack_hist) CK(cudaMemcpyAsync(slack_hist, p.hist, (size_t)V * nb * 4, cudaMemcpyDeviceToHost, ctx->stream));
+    if (fail_bits) CK(cudaMemcpyAsync(fail_bits, p.fail_bits, (size_t)n_slots, cudaMemcpyDeviceToHost, ctx->stream));
+    CK(cudaStreamSynchronize(ctx->stream));
+    return AVFS_OK;
+}
+
+avfs_status avfs_get_switching_energy(avfs_ctx* ctx, double* out) {
+    CHECK_CTX();
+    if (!out) return fail(ctx, AVFS_ERR_ARG, "null output");
+    if (!ctx->sim_done) return fail(ctx, AVFS_ERR_STATE, "simulate first");
+    const int32_t V = (int32_t)ctx->vdd.size();
+    CK(ctx->d_energy.ensure((size_t)V * sizeof(double)));
+    CK(cudaMemsetAsync(ctx->d_energy.p, 0, (size_t)V * sizeof(double), ctx->stream));
+    CK(launch_energy(ctx->d_act.as<unsigned long long>(), ctx->d_cload.as<double>(), ctx->d_vdd.as<double>(), ctx->n_pi,
+                     ctx->n_gates, V, ctx->d_energy.as<double>(), ctx->stream));
+    CK(cudaMemcpyAsync(out, ctx->d_energy.p, (size_t)V * sizeof(double), cudaMemcpyDeviceToHost, ctx->stream));
+    CK(cudaStreamSynchronize(ctx->stream));
+    return AVFS_OK;
 }
 
 avfs_status avfs_get_stats(avfs_ctx* ctx, avfs_stats* st) {

@@ -133,4 +133,34 @@ struct GatherParams {
 };
 cudaError_t launch_gather(const GatherParams& p, cudaStream_t st);
 
+// NEXT-1 capture analysis over the kept PO waveforms
+struct CaptureParams {
+    const uint32_t* po_loc;     // [n_po] LOC_PI | pi, or LOC_PINNED | arena buffer
+    int32_t n_po;
+    int32_t n_vdd;
+    const float* t_clk;         // [n_vdd]
+    int64_t sw_lo, n_sw;        // simulated slot groups [sw_lo, sw_lo + n_sw)
+    int64_t n_pairs;
+    int32_t n_pw;
+    int64_t slot_first, slot_end;
+    const uint32_t* p1t;
+    const uint32_t* p2t;
+    const int32_t* sw_round;
+    const int32_t* sw_index;
+    GatherRound rounds[8];
+    uint32_t* slot_fail;        // [n_sw * 32]
+    uint32_t* slot_last;        // [n_sw * 32] float bits
+    uint32_t* fail_po;          // [n_po][n_vdd]
+    uint32_t* fail_pairs;       // [n_vdd]
+    uint32_t* hist;             // [n_vdd][n_bins] or null
+    int32_t n_bins;
+    float lo, width;
+    uint8_t* fail_bits;         // [slot_end - slot_first] or null
+};
+cudaError_t launch_capture(const CaptureParams& p, cudaStream_t st);
+
+// NEXT-4 switching energy: out[k] += 1/2 sum_g act[n_pi+g][k] c[g] v_k^2
+cudaError_t launch_energy(const unsigned long long* act, const double* c_load, const double* vdd, int32_t n_pi,
+                          int32_t n_gates, int32_t n_vdd, double* out, cudaStream_t st);
+
 }  // namespace avfs

@@ -711,4 +711,108 @@ cudaError_t launch_gather(const GatherParams& p, cudaStream_t st) {
     return cudaGetLastError();
 }
 
+// ---------------------------------------------------------------------------
+// NEXT-1: capture / test-response analysis.  One warp per (PO, slot group):
+// each lane samples its slot's PO waveform at the capture time of the slot's
+// operating point (value(t) = init xor #{t_i <= t} mod 2, reading C1) and
+// compares with the settled value.
+// ---------------------------------------------------------------------------
+__global__ void capture_kernel(const CaptureParams p) {
+    const int lane = threadIdx.x & 31;
+    const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    if (gw >= (int64_t)p.n_po * p.n_sw) return;
+    const int o = (int)(gw / p.n_sw);
+    const int64_t i = gw % p.n_sw;
+    const int64_t sw = p.sw_lo + i;
+    const int kv = (int)(sw / p.n_pw), pw = (int)(sw % p.n_pw);
+    const int64_t j = (int64_t)pw * 32 + lane;
+    const int64_t pub = (int64_t)kv * p.n_pairs + j;
+    const bool valid = j < p.n_pairs && pub >= p.slot_first && pub < p.slot_end;
+    const float T = p.t_clk[kv];
+    const uint32_t loc = p.po_loc[o];
+    uint32_t init = 0, n = 0, c = 0;
+    float last = 0.0f;
+    if ((loc & LOC_KIND) == LOC_PI) {
+        const uint32_t w1 = p.p1t[(int64_t)(loc & LOC_ID) * p.n_pw + pw];
+        const uint32_t w2 = p.p2t[(int64_t)(loc & LOC_ID) * p.n_pw + pw];
+        init = (w1 >> lane) & 1u;
+        n = ((w1 ^ w2) >> lane) & 1u;
+        c = (n && 0.0f <= T) ? 1u : 0u;
+    } else {
+        const int r = p.sw_round[sw];
+        const GatherRound R = p.rounds[r < 0 ? 0 : r];
+        const uint8_t* base = R.pinned + ((int64_t)(loc & LOC_ID) * R.n_sw + p.sw_index[sw]) * R.region_bytes;
+        const uint32_t h = reinterpret_cast<const uint32_t*>(base)[lane];
+        init = (h >> HDR_INIT_SHIFT) & 1u;
+        n = h & HDR_N;
+        const float* ev = reinterpret_cast<const float*>(base + 128) + ((h >> HDR_OFF_SHIFT) & HDR_OFF);
+        if (valid)
+            for (uint32_t e = 0; e < n; ++e) {
+                const float t = ev[e];
+                last = t;
+                c += (t <= T) ? 1u : 0u;
+            }
+    }
+    const bool fail = valid && (((init ^ c) & 1u) != ((init ^ n) & 1u));
+    const uint32_t fb = __ballot_sync(0xffffffffu, fail);
+    if (lane == 0 && fb) atomicAdd(p.fail_po + (int64_t)o * p.n_vdd + kv, (uint32_t)__popc(fb));
+    if (fail) atomicOr(p.slot_fail + i * 32 + lane, 1u);
+    if (valid && last > 0.0f) atomicMax(p.slot_last + i * 32 + lane, __float_as_uint(last));
+}
+
+// per simulated slot: fail count, fail bit, slack histogram
+__global__ void capture_finish_kernel(const CaptureParams p) {
+    const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (t >= p.n_sw * 32) return;
+    const int64_t i = t >> 5;
+    const int lane = (int)(t & 31);
+    const int64_t sw = p.sw_lo + i;
+    const int kv = (int)(sw / p.n_pw), pw = (int)(sw % p.n_pw);
+    const int64_t j = (int64_t)pw * 32 + lane;
+    const int64_t pub = (int64_t)kv * p.n_pairs + j;
+    if (!(j < p.n_pairs && pub >= p.slot_first && pub < p.slot_end)) return;
+    const uint32_t f = p.slot_fail[t];
+    if (f) atomicAdd(p.fail_pairs + kv, 1u);
+    if (p.fail_bits) p.fail_bits[pub - p.slot_first] = (uint8_t)f;
+    if (p.hist) {
+        const float slack = p.t_clk[kv] - __uint_as_float(p.slot_last[t]);
+        int b = (int)floorf((slack - p.lo) / p.width);
+        b = b < 0 ? 0 : (b >= p.n_bins ? p.n_bins - 1 : b);
+        atomicAdd(p.hist + (int64_t)kv * p.n_bins + b, 1u);
+    }
+}
+
+cudaError_t launch_capture(const CaptureParams& p, cudaStream_t st) {
+    const int64_t threads = (int64_t)p.n_po * p.n_sw * 32;
+    if (threads > 0) {
+        capture_kernel<<<(unsigned)((threads + 255) / 256), 256, 0, st>>>(p);
+        cudaError_t e = cudaGetLastError();
+        if (e != cudaSuccess) return e;
+    }
+    const int64_t t2 = p.n_sw * 32;
+    if (t2 > 0) capture_finish_kernel<<<(unsigned)((t2 + 255) / 256), 256, 0, st>>>(p);
+    return cudaGetLastError();
+}
+
+// NEXT-4: switching energy per operating point, warp-reduced double atomics
+__global__ void energy_kernel(const unsigned long long* __restrict__ act, const double* __restrict__ c_load,
+                              const double* __restrict__ vdd, int32_t n_pi, int32_t n_gates, int32_t n_vdd,
+                              double* out) {
+    const int64_t g = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    const double c = g < n_gates ? c_load[g] : 0.0;
+    for (int k = 0; k < n_vdd; ++k) {
+        double e = g < n_gates ? (double)act[(n_pi + g) * n_vdd + k] * c : 0.0;
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) e += __shfl_down_sync(0xffffffffu, e, o);
+        if ((threadIdx.x & 31) == 0 && e != 0.0) atomicAdd(out + k, 0.5 * e * vdd[k] * vdd[k]);
+    }
+}
+
+cudaError_t launch_energy(const unsigned long long* act, const double* c_load, const double* vdd, int32_t n_pi,
+                          int32_t n_gates, int32_t n_vdd, double* out, cudaStream_t st) {
+    if (n_gates <= 0) return cudaSuccess;
+    energy_kernel<<<(unsigned)((n_gates + 255) / 256), 256, 0, st>>>(act, c_load, vdd, n_pi, n_gates, n_vdd, out);
+    return cudaGetLastError();
+}
+
 }  // namespace avfs

