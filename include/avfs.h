@@ -133,6 +133,15 @@ avfs_status avfs_get_buffer_map(avfs_ctx *ctx, int32_t *loc);
 /* Operating points: n_vdd supply voltages in volts.             */
 avfs_status avfs_set_operating_points(avfs_ctx *ctx, int32_t n_vdd, const double *vdd_volts);
 
+/* NEXT-2 -- per-gate operating points (voltage islands; "gate- and circuit
+ * parameters P").  island_of_gate[n_gates] in [0, n_islands) (NULL:
+ * all 0); vdd_volts[n_points][n_islands]: operating point k supplies island i
+ * with vdd_volts[k][i].  Gate g's delays at point k use vdd[k][island[g]].
+ * avfs_set_operating_points(n, v) is the 1-island special case.  Call after
+ * the netlist is loaded (loading a netlist resets to one island).        */
+avfs_status avfs_set_voltage_islands(avfs_ctx *ctx, int32_t n_islands, const int32_t *island_of_gate,
+                                     int32_t n_points, const double *vdd_volts);
+
 /* ---------------------------------------------------------------- (3) */
 /* Two-pattern stimuli: p1, p2 are uint32 [n_pairs][ceil(n_pi/32)], bit
  * (i % 32) of word (i / 32) is PI i.  All PIs with p1 != p2 switch at
@@ -211,8 +220,9 @@ avfs_status avfs_capture(avfs_ctx *ctx, const float *t_clk, int32_t n_bins, floa
                          uint32_t *slack_hist, uint8_t *fail_bits);
 
 /* NEXT-4 -- switching energy per operating point (P:L37 power estimation):
- * out[k] = 1/2 sum_g act[g][k] * c_load(g) * v_k^2, in fJ (c_load in fF from
- * the netlist, v in V), summed over the simulated pairs.  Gate outputs only
+ * out[k] = 1/2 sum_g act[g][k] * c_load(g) * v(g,k)^2, in fJ (c_load in fF from
+ * the netlist, v(g,k) the gate's island voltage at point k, in V), summed over
+ * the simulated pairs.  Gate outputs only
  * (primary inputs are driven externally).  Computed on the device.        */
 avfs_status avfs_get_switching_energy(avfs_ctx *ctx, double *out_fJ);
 

@@ -43,11 +43,11 @@ def _load():
         lib.oracle_sta.restype = C.c_int
         lib.oracle_sta.argtypes = [C.c_int32, C.c_int32, P, P, P, P, P, P, P, C.c_int32, C.c_int32, P,
                                    C.c_double, C.c_double, C.c_double, C.c_double,
-                                   C.c_int32, P, C.c_double, P, P]
+                                   C.c_int32, P, C.c_double, P, C.c_int32, P, P]
         lib.oracle_simulate.restype = C.c_int
         lib.oracle_simulate.argtypes = [C.c_int32, C.c_int32, P, P, P, P, P, P, P, C.c_int32, C.c_int32, P,
                                         C.c_double, C.c_double, C.c_double, C.c_double,
-                                        C.c_int32, P, P, P, C.c_double,
+                                        C.c_int32, P, P, P, C.c_double, P, C.c_int32,
                                         C.c_int64, P, P, C.c_int32, P, C.c_int32,
                                         P, P, P, P, P, C.c_int32]
         lib.oracle_max_threads.restype = C.c_int
@@ -86,13 +86,22 @@ def _net_args(nl, lib):
     return keep, args
 
 
-def sta(nl, lib, vdd, quantum=0.0):
+def _islands(vdd, island):
+    """vdd [n_points] (one supply) or [n_points][n_isl] with island[gate]."""
+    v = _c(vdd, np.float64)
+    if v.ndim == 1:
+        return v, None, 1
+    isl = _c(island, np.int32)
+    return v, isl, int(v.shape[1])
+
+
+def sta(nl, lib, vdd, quantum=0.0, island=None):
     """Longest / shortest path arrival per (Vdd, signal): (arr_max, arr_min)."""
-    vdd = _c(vdd, np.float64)
+    vdd, isl, n_isl = _islands(vdd, island)
     amax = np.zeros((len(vdd), nl.n_signals))
     amin = np.zeros((len(vdd), nl.n_signals))
     keep, args = _net_args(nl, lib)
-    rc = _load().oracle_sta(*args, len(vdd), _p(vdd), float(quantum), _p(amax), _p(amin))
+    rc = _load().oracle_sta(*args, len(vdd), _p(vdd), float(quantum), _p(isl), n_isl, _p(amax), _p(amin))
     if rc:
         raise RuntimeError(f"oracle_sta failed: {rc}")
     return amax, amin
@@ -113,9 +122,10 @@ class OracleResult:
 
 
 def simulate(nl, lib, stim, vdd, slot_pair, slot_vdd, quantum=0.0, cap=8,
-             out_sig=None, threads=0) -> OracleResult:
-    """Simulate slots (pair slot_pair[s], Vdd index slot_vdd[s])."""
-    vdd = _c(vdd, np.float64)
+             out_sig=None, threads=0, island=None) -> OracleResult:
+    """Simulate slots (pair slot_pair[s], operating point slot_vdd[s]).
+    vdd: [n_points] volts, or [n_points][n_isl] with island[gate] (NEXT-2)."""
+    vdd, isl, n_isl = _islands(vdd, island)
     sp = _c(slot_pair, np.int64)
     sv = _c(slot_vdd, np.int32)
     n_slots = len(sp)
@@ -130,7 +140,7 @@ def simulate(nl, lib, stim, vdd, slot_pair, slot_vdd, quantum=0.0, cap=8,
     flags = np.zeros(1, np.int64)
     p1, p2 = _c(stim.p1, np.uint32), _c(stim.p2, np.uint32)
     keep, args = _net_args(nl, lib)
-    rc = _load().oracle_simulate(*args, stim.words, _p(p1), _p(p2), _p(vdd), float(quantum),
+    rc = _load().oracle_simulate(*args, stim.words, _p(p1), _p(p2), _p(vdd), float(quantum), _p(isl), n_isl,
                                  n_slots, _p(sp), _p(sv), n_out, _p(out_sig), int(cap),
                                  _p(count), _p(init), _p(times), _p(taint), _p(flags), int(threads))
     if rc:

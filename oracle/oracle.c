@@ -9,6 +9,10 @@
  * It shares no code, header, table or helper with the CUDA path
  * (paper_conf_date_schneiderw20_b200/), and never imports it.
  *
+ * Operating points may give one voltage per island (NEXT-2, per-gate
+ * parameters P:L155): vdd is then [point][n_isl] and gate g uses
+ * vdd[k][island[g]]; n_isl = 1 is the paper's single supply.
+ *
  * Functions (each cites the passage it follows):
  *   oracle_delay     -- Eq. (4), normalisations P:L117, Eq. (9) P:L135,
  *                       Horner/FMA P:L139.  Pinned by tests T1/T2/T3.
@@ -79,6 +83,8 @@ typedef struct {
     int32_t deg_v, deg_c;
     const double *beta;      /* [cell][4][2][deg_v+1][deg_c+1] */
     double v_min, v_max, c_min, c_max;
+    const int32_t *island;   /* [gate] voltage island (NEXT-2) or NULL: island 0 */
+    int32_t n_isl;           /* islands per operating point (vdd is [point][n_isl]) */
     /* derived */
     int32_t *topo;           /* gates in topological order */
     int64_t *fo_ptr;         /* fanout CSR per signal */
@@ -137,8 +143,10 @@ static void net_free(Net *n)
     free(n->topo); free(n->fo_ptr); free(n->fo_gate); free(n->fo_pin);
 }
 
-static double arc_delay(const Net *n, int32_t g, int32_t pin, int pol, double v, double quantum)
+/* vrow = the operating point's island voltages; the gate uses its island's (NEXT-2) */
+static double arc_delay(const Net *n, int32_t g, int32_t pin, int pol, const double *vrow, double quantum)
 {
+    const double v = vrow[n->island ? n->island[g] : 0];
     int32_t cell = n->gate_cell[g];
     size_t nb = (size_t)(n->deg_v + 1) * (size_t)(n->deg_c + 1);
     const double *b = n->beta + (((size_t)cell * 4 + (size_t)pin) * 2 + (size_t)pol) * nb;
@@ -161,10 +169,12 @@ int oracle_sta(int32_t n_pi, int32_t n_gates, const int32_t *gate_cell,
                int32_t deg_v, int32_t deg_c, const double *beta,
                double v_min, double v_max, double c_min, double c_max,
                int32_t n_vdd, const double *vdd, double quantum,
+               const int32_t *gate_island, int32_t n_isl,
                double *arr_max, double *arr_min)
 {
     Net n = {n_pi, n_gates, n_pi + n_gates, gate_cell, fanin_ptr, fanin_sig, d_nom, c_load,
-             cell_nin, cell_tt, deg_v, deg_c, beta, v_min, v_max, c_min, c_max, 0, 0, 0, 0};
+             cell_nin, cell_tt, deg_v, deg_c, beta, v_min, v_max, c_min, c_max,
+             gate_island, n_isl > 0 ? n_isl : 1, 0, 0, 0, 0};
     int rc = net_prepare(&n);
     if (rc) { net_free(&n); return rc; }
     for (int32_t k = 0; k < n_vdd; ++k) {
@@ -176,7 +186,7 @@ int oracle_sta(int32_t n_pi, int32_t n_gates, const int32_t *gate_cell,
             for (int64_t e = fanin_ptr[g]; e < fanin_ptr[g + 1]; ++e) {
                 int32_t pin = (int32_t)(e - fanin_ptr[g]);
                 for (int pol = 0; pol < 2; ++pol) {
-                    double d = arc_delay(&n, g, pin, pol, vdd[k], quantum);
+                    double d = arc_delay(&n, g, pin, pol, vdd + (size_t)k * n.n_isl, quantum);
                     double a = amax[fanin_sig[e]] + d, b = amin[fanin_sig[e]] + d;
                     if (a > mx) mx = a;
                     if (b < mn) mn = b;
@@ -268,13 +278,15 @@ int oracle_simulate(int32_t n_pi, int32_t n_gates, const int32_t *gate_cell,
                     double v_min, double v_max, double c_min, double c_max,
                     int32_t words, const uint32_t *p1, const uint32_t *p2,
                     const double *vdd, double quantum,
+                    const int32_t *gate_island, int32_t n_isl,
                     int64_t n_slots, const int64_t *slot_pair, const int32_t *slot_vdd,
                     int32_t n_out, const int32_t *out_sig, int32_t cap,
                     int32_t *count, uint8_t *init, double *times, uint8_t *taint,
                     int64_t *flags_out, int32_t n_threads)
 {
     Net n = {n_pi, n_gates, n_pi + n_gates, gate_cell, fanin_ptr, fanin_sig, d_nom, c_load,
-             cell_nin, cell_tt, deg_v, deg_c, beta, v_min, v_max, c_min, c_max, 0, 0, 0, 0};
+             cell_nin, cell_tt, deg_v, deg_c, beta, v_min, v_max, c_min, c_max,
+             gate_island, n_isl > 0 ? n_isl : 1, 0, 0, 0, 0};
     int rc = net_prepare(&n);
     if (rc) { net_free(&n); return rc; }
     const int32_t S = n.n_sig, G = n_gates;
@@ -311,7 +323,7 @@ int oracle_simulate(int32_t n_pi, int32_t n_gates, const int32_t *gate_cell,
 #pragma omp for schedule(dynamic, 1)
         for (int64_t s = 0; s < n_slots; ++s) {
             const int64_t j = slot_pair[s];
-            const double v = vdd[slot_vdd[s]];
+            const double *v = vdd + (size_t)slot_vdd[s] * n.n_isl;   /* island voltages */
             const uint32_t *w1 = p1 + (size_t)j * (size_t)words, *w2 = p2 + (size_t)j * (size_t)words;
             /* O3: static evaluation of p1 in topological order */
             for (int32_t i = 0; i < n_pi; ++i) val[i] = (uint8_t)get_bit(w1, i);

@@ -21,7 +21,7 @@ EXPORTS = [
     "avfs_create", "avfs_destroy", "avfs_last_error", "avfs_status_string", "avfs_version",
     "avfs_load_library", "avfs_load_netlist", "avfs_load_bench", "avfs_find_signal",
     "avfs_get_netlist_info", "avfs_get_levels", "avfs_get_buffer_map",
-    "avfs_set_operating_points", "avfs_set_stimuli", "avfs_set_slot_range",
+    "avfs_set_operating_points", "avfs_set_voltage_islands", "avfs_set_stimuli", "avfs_set_slot_range",
     "avfs_set_options", "avfs_default_options", "avfs_simulate", "avfs_sync",
     "avfs_get_activity", "avfs_get_latest_arrival", "avfs_get_final_values",
     "avfs_get_waveforms", "avfs_get_stats", "avfs_capture", "avfs_get_switching_energy",
@@ -86,6 +86,7 @@ def load_library(path: str = LIB_PATH):
             "avfs_get_levels": ([P, P], C.c_int),
             "avfs_get_buffer_map": ([P, P], C.c_int),
             "avfs_set_operating_points": ([P, I32, P], C.c_int),
+            "avfs_set_voltage_islands": ([P, I32, P, I32, P], C.c_int),
             "avfs_set_stimuli": ([P, I64, P, P, I32], C.c_int),
             "avfs_set_slot_range": ([P, I64, I64], C.c_int),
             "avfs_set_options": ([P, P], C.c_int),
@@ -211,6 +212,13 @@ class Context:
         v = _c(vdd, np.float64)
         self._ck(self.lib.avfs_set_operating_points(self.h, len(v), _p(v)))
         self.n_vdd = len(v)
+
+    def set_voltage_islands(self, island_of_gate, vdd_matrix):
+        """NEXT-2: vdd_matrix [n_points][n_islands] volts, island_of_gate [n_gates]."""
+        v = _c(vdd_matrix, np.float64)
+        isl = None if island_of_gate is None else _c(island_of_gate, np.int32)
+        self._ck(self.lib.avfs_set_voltage_islands(self.h, int(v.shape[1]), _p(isl), int(v.shape[0]), _p(v)))
+        self.n_vdd = int(v.shape[0])
 
     def set_stimuli(self, p1, p2):
         """p1, p2: numpy uint32 [n_pairs][words] (host) or torch CUDA tensors (device)."""

@@ -111,7 +111,10 @@ struct avfs_ctx {
     avfs_options opt{};
     std::vector<int32_t> probes;
 
-    std::vector<double> vdd;
+    std::vector<double> vdd;          // [n_points] first island's supply (sizes by point)
+    std::vector<double> vdd_all;      // [n_points][n_isl]
+    std::vector<int32_t> island;      // [n_gates] voltage island (NEXT-2)
+    int32_t n_isl = 1;
     int64_t n_pairs = 0;
     int32_t words = 0;
     bool stim_set = false;
@@ -119,7 +122,7 @@ struct avfs_ctx {
 
     // device state
     bool dev_net_valid = false, dev_vdd_valid = false;
-    DevBuf d_gates, d_ddesc, d_dtab, d_coef, d_cload, d_energy, c_loc, c_tclk, c_slot, c_out, d_level_ptr, d_vdd, d_p1, d_p2, d_p1t, d_p2t, d_act, d_latest, d_ovf,
+    DevBuf d_gates, d_ddesc, d_dtab, d_coef, d_cload, d_island, d_energy, c_loc, c_tclk, c_slot, c_out, d_level_ptr, d_vdd, d_p1, d_p2, d_p1t, d_p2t, d_act, d_latest, d_ovf,
         d_err, d_list[2], d_count, d_swround, d_swindex, g_loc, g_init, g_count, g_times, g_bad;
     std::vector<DevBuf> arena;        // per round: [buffer][slot group][region]
     int32_t* h_pinned = nullptr;      // small pinned host buffer (count, err)
@@ -336,6 +339,7 @@ avfs_status upload_netlist(avfs_ctx* ctx) {
                 ((ctx->is_po[ctx->n_pi + g] ? 1u : 0u) << 24);
         e.coef_off = ctx->coef_off[g];
         e.k = (uint32_t)k;
+        e.island = (uint32_t)ctx->island[g];
         for (int p = 0; p < k; ++p)
             for (int pol = 0; pol < 2; ++pol) e.dnom[2 * p + pol] = ctx->d_nom[(ctx->fanin_ptr[g] + p) * 2 + pol];
         for (int p = k; p < KMAX; ++p) e.dnom[2 * p] = e.dnom[2 * p + 1] = 1.0;
@@ -347,6 +351,8 @@ avfs_status upload_netlist(avfs_ctx* ctx) {
     CK(ctx->d_coef.ensure(std::max<size_t>(ctx->coef.size(), 1) * sizeof(double)));
     if (!ctx->coef.empty())
         CK(cudaMemcpy(ctx->d_coef.p, ctx->coef.data(), ctx->coef.size() * sizeof(double), cudaMemcpyHostToDevice));
+    CK(ctx->d_island.ensure((size_t)std::max<int32_t>(G, 1) * sizeof(int32_t)));
+    CK(cudaMemcpy(ctx->d_island.p, ctx->island.data(), (size_t)G * sizeof(int32_t), cudaMemcpyHostToDevice));
     CK(ctx->d_cload.ensure((size_t)std::max<int32_t>(G, 1) * sizeof(double)));
     CK(cudaMemcpy(ctx->d_cload.p, ctx->c_load.data(), (size_t)G * sizeof(double), cudaMemcpyHostToDevice));
     CK(ctx->d_level_ptr.ensure(ctx->level_ptr.size() * sizeof(int32_t)));
@@ -523,6 +529,12 @@ avfs_status avfs_load_netlist(avfs_ctx* ctx, int32_t n_pi, int32_t n_gates, cons
     if (c_load_fF) ctx->c_load.assign(c_load_fF, c_load_fF + n_gates);
     else ctx->c_load.assign(n_gates, 1.0);
     ctx->po.assign(po_sig, po_sig + n_po);
+    ctx->island.assign(n_gates, 0);
+    if (ctx->n_isl != 1 && !ctx->vdd.empty()) {     // back to one supply per operating point
+        ctx->n_isl = 1;
+        ctx->vdd_all = ctx->vdd;
+        ctx->dev_vdd_valid = false;
+    }
     ctx->net_loaded = false;
     avfs_status st = levelize(ctx);
     if (st != AVFS_OK) return st;
@@ -697,21 +709,38 @@ avfs_status avfs_get_buffer_map(avfs_ctx* ctx, int32_t* out) {
     return AVFS_OK;
 }
 
-avfs_status avfs_set_operating_points(avfs_ctx* ctx, int32_t n_vdd, const double* vdd) {
-    CHECK_CTX();
-    if (n_vdd < 1 || !vdd) return fail(ctx, AVFS_ERR_ARG, "need at least one operating point");
-    for (int32_t k = 0; k < n_vdd; ++k)
+static avfs_status set_points(avfs_ctx* ctx, int32_t n_isl, const int32_t* island, int32_t n_points,
+                              const double* vdd) {
+    if (n_points < 1 || n_isl < 1 || !vdd) return fail(ctx, AVFS_ERR_ARG, "need at least one operating point / island");
+    for (int64_t k = 0; k < (int64_t)n_points * n_isl; ++k)
         if (!std::isfinite(vdd[k])) return fail(ctx, AVFS_ERR_ARG, "non-finite Vdd");
-    ctx->vdd.assign(vdd, vdd + n_vdd);
-    ctx->dev_vdd_valid = false;
-    if (has_dev(ctx)) {
-        CK(cudaSetDevice(ctx->dev));
-        CK(ctx->d_vdd.ensure(n_vdd * sizeof(double)));
-        CK(cudaMemcpy(ctx->d_vdd.p, vdd, n_vdd * sizeof(double), cudaMemcpyHostToDevice));
-        ctx->dev_vdd_valid = true;
+    if (island) {
+        if (!ctx->net_loaded) return fail(ctx, AVFS_ERR_STATE, "load a netlist before assigning islands");
+        for (int32_t g = 0; g < ctx->n_gates; ++g)
+            if (island[g] < 0 || island[g] >= n_isl) return fail(ctx, AVFS_ERR_ARG, "gate %d: island out of range", g);
+        ctx->island.assign(island, island + ctx->n_gates);
+    } else if (ctx->net_loaded) {
+        ctx->island.assign(ctx->n_gates, 0);
     }
+    ctx->n_isl = n_isl;
+    ctx->vdd_all.assign(vdd, vdd + (size_t)n_points * n_isl);
+    ctx->vdd.resize(n_points);
+    for (int32_t k = 0; k < n_points; ++k) ctx->vdd[k] = vdd[(size_t)k * n_isl];
+    ctx->dev_vdd_valid = false;
+    ctx->dev_net_valid = false;          // island index lives in the delay descriptors
     invalidate_sim(ctx);
     return AVFS_OK;
+}
+
+avfs_status avfs_set_operating_points(avfs_ctx* ctx, int32_t n_vdd, const double* vdd) {
+    CHECK_CTX();
+    return set_points(ctx, 1, nullptr, n_vdd, vdd);
+}
+
+avfs_status avfs_set_voltage_islands(avfs_ctx* ctx, int32_t n_islands, const int32_t* island_of_gate,
+                                     int32_t n_points, const double* vdd_volts) {
+    CHECK_CTX();
+    return set_points(ctx, n_islands, island_of_gate, n_points, vdd_volts);
 }
 
 avfs_status avfs_set_stimuli(avfs_ctx* ctx, int64_t n_pairs, const uint32_t* p1, const uint32_t* p2,
@@ -861,6 +890,11 @@ avfs_status avfs_simulate(avfs_ctx* ctx, void* cuda_stream) {
     if (st != AVFS_OK) return st;
     st = upload_netlist(ctx);
     if (st != AVFS_OK) return st;
+    if (!ctx->dev_vdd_valid) {
+        CK(ctx->d_vdd.ensure(ctx->vdd_all.size() * sizeof(double)));
+        CK(cudaMemcpy(ctx->d_vdd.p, ctx->vdd_all.data(), ctx->vdd_all.size() * sizeof(double), cudaMemcpyHostToDevice));
+        ctx->dev_vdd_valid = true;
+    }
     invalidate_sim(ctx);
     const int64_t P = ctx->n_pairs;
     const int32_t V = (int32_t)ctx->vdd.size();
@@ -895,6 +929,7 @@ avfs_status avfs_simulate(avfs_ctx* ctx, void* cuda_stream) {
         dp.deg_v = ctx->deg_v;
         dp.vdd = ctx->d_vdd.as<double>();
         dp.n_vdd = V;
+        dp.n_isl = ctx->n_isl;
         dp.v_min = ctx->v_min;
         dp.v_max = ctx->v_max;
         dp.quantum = ctx->opt.quantum_ps;
@@ -1169,8 +1204,9 @@ avfs_status avfs_get_switching_energy(avfs_ctx* ctx, double* out) {
     const int32_t V = (int32_t)ctx->vdd.size();
     CK(ctx->d_energy.ensure((size_t)V * sizeof(double)));
     CK(cudaMemsetAsync(ctx->d_energy.p, 0, (size_t)V * sizeof(double), ctx->stream));
-    CK(launch_energy(ctx->d_act.as<unsigned long long>(), ctx->d_cload.as<double>(), ctx->d_vdd.as<double>(), ctx->n_pi,
-                     ctx->n_gates, V, ctx->d_energy.as<double>(), ctx->stream));
+    CK(launch_energy(ctx->d_act.as<unsigned long long>(), ctx->d_cload.as<double>(), ctx->d_vdd.as<double>(),
+                     ctx->d_island.as<int32_t>(), ctx->n_isl, ctx->n_pi, ctx->n_gates, V, ctx->d_energy.as<double>(),
+                     ctx->stream));
     CK(cudaMemcpyAsync(out, ctx->d_energy.p, (size_t)V * sizeof(double), cudaMemcpyDeviceToHost, ctx->stream));
     CK(cudaStreamSynchronize(ctx->stream));
     return AVFS_OK;

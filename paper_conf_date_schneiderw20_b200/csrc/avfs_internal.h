@@ -40,7 +40,8 @@ struct alignas(16) DelayDesc {
     double dnom[2 * KMAX];   // [pin][pol] nominal delay, ps
     uint32_t coef_off;       // offset (doubles) of the [pin][pol][deg_v+1] coefficient block
     uint32_t k;
-    uint32_t pad[2];
+    uint32_t island;         // voltage island (NEXT-2)
+    uint32_t pad;
 };
 static_assert(sizeof(DelayDesc) == 80, "DelayDesc layout");
 
@@ -49,8 +50,9 @@ struct DelayParams {
     int32_t n_gates;
     const double* __restrict__ coef;
     int32_t deg_v;
-    const double* __restrict__ vdd;          // [n_vdd] volts
+    const double* __restrict__ vdd;          // [n_vdd][n_isl] volts
     int32_t n_vdd;
+    int32_t n_isl;
     double v_min, v_max;
     double quantum;                          // 0: F mode
     float* dtab;                             // [n_vdd][n_gates][8] delays (binary32), ps
@@ -160,7 +162,8 @@ struct CaptureParams {
 cudaError_t launch_capture(const CaptureParams& p, cudaStream_t st);
 
 // NEXT-4 switching energy: out[k] += 1/2 sum_g act[n_pi+g][k] c[g] v_k^2
-cudaError_t launch_energy(const unsigned long long* act, const double* c_load, const double* vdd, int32_t n_pi,
-                          int32_t n_gates, int32_t n_vdd, double* out, cudaStream_t st);
+cudaError_t launch_energy(const unsigned long long* act, const double* c_load, const double* vdd,
+                          const int32_t* island, int32_t n_isl, int32_t n_pi, int32_t n_gates, int32_t n_vdd,
+                          double* out, cudaStream_t st);
 
 }  // namespace avfs

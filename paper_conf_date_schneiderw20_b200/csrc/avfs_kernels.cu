@@ -106,7 +106,8 @@ __global__ void delay_kernel(const DelayParams p) {
     const DelayDesc& D = p.dd[g];
     float out = 1.0f;
     if (e < 2 * (int)D.k) {
-        const double x = (p.vdd[kv] - p.v_min) / (p.v_max - p.v_min);      // phi_V
+        const double v = p.vdd[(size_t)kv * p.n_isl + D.island];           // gate's island supply (NEXT-2)
+        const double x = (v - p.v_min) / (p.v_max - p.v_min);                // phi_V
         const double* cf = p.coef + D.coef_off + e * (p.deg_v + 1);
         double f = cf[p.deg_v];
         for (int i = p.deg_v - 1; i >= 0; --i) f = fma(f, x, cf[i]);
@@ -796,22 +797,26 @@ cudaError_t launch_capture(const CaptureParams& p, cudaStream_t st) {
 
 // NEXT-4: switching energy per operating point, warp-reduced double atomics
 __global__ void energy_kernel(const unsigned long long* __restrict__ act, const double* __restrict__ c_load,
-                              const double* __restrict__ vdd, int32_t n_pi, int32_t n_gates, int32_t n_vdd,
-                              double* out) {
+                              const double* __restrict__ vdd, const int32_t* __restrict__ island, int32_t n_isl,
+                              int32_t n_pi, int32_t n_gates, int32_t n_vdd, double* out) {
     const int64_t g = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     const double c = g < n_gates ? c_load[g] : 0.0;
+    const int isl = g < n_gates ? island[g] : 0;
     for (int k = 0; k < n_vdd; ++k) {
-        double e = g < n_gates ? (double)act[(n_pi + g) * n_vdd + k] * c : 0.0;
+        const double v = vdd[(size_t)k * n_isl + isl];
+        double e = g < n_gates ? 0.5 * (double)act[(n_pi + g) * n_vdd + k] * c * v * v : 0.0;
 #pragma unroll
         for (int o = 16; o > 0; o >>= 1) e += __shfl_down_sync(0xffffffffu, e, o);
-        if ((threadIdx.x & 31) == 0 && e != 0.0) atomicAdd(out + k, 0.5 * e * vdd[k] * vdd[k]);
+        if ((threadIdx.x & 31) == 0 && e != 0.0) atomicAdd(out + k, e);
     }
 }
 
-cudaError_t launch_energy(const unsigned long long* act, const double* c_load, const double* vdd, int32_t n_pi,
-                          int32_t n_gates, int32_t n_vdd, double* out, cudaStream_t st) {
+cudaError_t launch_energy(const unsigned long long* act, const double* c_load, const double* vdd,
+                          const int32_t* island, int32_t n_isl, int32_t n_pi, int32_t n_gates, int32_t n_vdd,
+                          double* out, cudaStream_t st) {
     if (n_gates <= 0) return cudaSuccess;
-    energy_kernel<<<(unsigned)((n_gates + 255) / 256), 256, 0, st>>>(act, c_load, vdd, n_pi, n_gates, n_vdd, out);
+    energy_kernel<<<(unsigned)((n_gates + 255) / 256), 256, 0, st>>>(act, c_load, vdd, island, n_isl, n_pi, n_gates,
+                                                                     n_vdd, out);
     return cudaGetLastError();
 }
 

@@ -73,3 +73,34 @@ def test_switching_energy_matches_oracle_counts():
     assert np.allclose(got, want, rtol=1e-12, atol=0)
     assert np.all(np.diff(want / w.vdd ** 2) != 0) or True
     ctx.close()
+
+
+@pytest.mark.parametrize("quantum", [Q, 0.0])
+def test_voltage_islands_parity(quantum):
+    """NEXT-2: per-gate supplies (3 islands x 4 operating points) vs the oracle."""
+    from paper_conf_date_schneiderw20_b200 import Context, load_workload
+    from tests.parity import gpu_waveforms, compare, activity_ref
+    w = make_config(3, n_pairs=72, n_vdd=4, scale=0.05)
+    nl = w.netlist
+    rng = np.random.default_rng(11)
+    island = rng.integers(0, 3, size=nl.n_gates).astype(np.int32)
+    vdd = np.array([[0.6, 0.8, 1.1], [0.7, 0.7, 0.7], [1.0, 0.65, 0.9], [1.1, 1.1, 0.6]])
+    P, V = w.stimuli.n_pairs, vdd.shape[0]
+    j, k = oracle.all_slots(P, V)
+    ref = oracle.simulate(nl, w.library, w.stimuli, vdd, j, k, quantum=quantum, cap=64, island=island)
+    ctx = Context(0)
+    load_workload(ctx, nl, w.library, w.stimuli, vdd[:, 0])
+    ctx.set_voltage_islands(island, vdd)
+    ctx.set_options(capacity=8, quantum_ps=quantum, keep_all=True)
+    ctx.simulate()
+    init, cnt, times = gpu_waveforms(ctx, np.arange(nl.n_signals), 0, P * V, int(ref.count.max()) or 1)
+    compare(ref, init, cnt, times, quantum, "islands")
+    act = ctx.activity().astype(np.int64)
+    ra, ok = activity_ref(ref, V, nl.n_signals)
+    assert np.array_equal(act[ok], ra[ok])
+    e = ctx.switching_energy()
+    vg = vdd[:, island]                                  # [V][G]
+    want = 0.5 * (ra[nl.n_pi:].T * nl.c_load[None, :] * vg ** 2).sum(1)
+    if quantum > 0:
+        assert np.allclose(e, want, rtol=1e-12)
+    ctx.close()

@@ -328,3 +328,41 @@ def test_oracle_fmode_flags_are_rare_and_counted(oracle_mod):
     assert r.taint.mean() < 0.1
     rq = oracle_mod.simulate(w.netlist, w.library, w.stimuli, w.vdd, *oracle_mod.all_slots(32, 2), cap=0, quantum=Q)
     assert rq.flags == 0 and rq.taint.sum() == 0
+
+
+# ---------------------------------------------------------------- NEXT-2 islands
+def test_islands_chain_closed_form(oracle_mod):
+    """Per-gate supplies: each stage of a chain uses its own island's voltage."""
+    rng = np.random.default_rng(9)
+    n = 24
+    b = _Builder(1)
+    s = 0
+    kinds = rng.choice(["INV", "BUF"], size=n)
+    for kd in kinds:
+        s = b.gate(str(kd), s)
+    nl = b.build("chain", [s])
+    nl.d_nom = rng.uniform(2.0, 12.0, size=(n, 2))
+    lib = make_library(5, deg_v=3)
+    island = rng.integers(0, 3, size=n).astype(np.int32)
+    vdd = np.array([[0.6, 0.9, 1.1], [1.0, 0.7, 0.8]])
+    stim = Stimuli(1, pack_bits(np.array([[0]], np.uint8)), pack_bits(np.array([[1]], np.uint8)))
+    j, k = oracle_mod.all_slots(1, 2)
+    r = oracle_mod.simulate(nl, lib, stim, vdd, j, k, cap=2, island=island)
+    for kk in range(2):
+        t, val = 0.0, 1
+        for g in range(n):
+            val = 1 - val if kinds[g] == "INV" else val
+            t += poly_delay(lib, nl, g, 0, val, vdd[kk, island[g]])
+            assert abs(r.times[kk, 1 + g, 0] - t) <= 1e-9 * t
+
+
+def test_islands_equal_supplies_reduce_to_single_supply(oracle_mod):
+    nl = small_dag(41, G=300, n_pi=16, depth=12)
+    lib = make_library(7, deg_v=3)
+    stim = make_stimuli(8, nl.n_pi, 16)
+    vdd = np.array([0.65, 0.95])
+    island = (np.arange(nl.n_gates) % 4).astype(np.int32)
+    j, k = oracle_mod.all_slots(16, 2)
+    a = oracle_mod.simulate(nl, lib, stim, vdd, j, k, cap=32)
+    b = oracle_mod.simulate(nl, lib, stim, np.repeat(vdd[:, None], 4, axis=1), j, k, cap=32, island=island)
+    assert np.array_equal(a.count, b.count) and np.array_equal(a.times, b.times)
