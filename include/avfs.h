@@ -226,6 +226,20 @@ avfs_status avfs_capture(avfs_ctx *ctx, const float *t_clk, int32_t n_bins, floa
  * (primary inputs are driven externally).  Computed on the device.        */
 avfs_status avfs_get_switching_energy(avfs_ctx *ctx, double *out_fJ);
 
+/* NEXT-3 -- offline regression pre-process (Fig. 1 step C):
+ * fit the coefficients of Eq. (4) to n characterisation samples by ordinary
+ * least squares on the normal equation (Eq. 7/8), in FP64, host side.
+ *   v[n], c[n]   operating points (c may be NULL iff deg_c == 0)
+ *   y[n]         relative delay deviation d/d_nom - 1 (phi_D)
+ *   beta[(deg_v+1)(deg_c+1)]  output, row-major [i][j] (reading C9), the
+ *                layout avfs_load_library expects per (cell, pin, pol)
+ *   rms          output (may be NULL): root-mean-square residual in y
+ * AVFS_ERR_ARG: bad sizes / bounds, fewer samples than coefficients, or a
+ * rank-deficient design matrix.                                          */
+avfs_status avfs_fit_delay_polynomial(int64_t n, const double *v, const double *c, const double *y,
+                                      int32_t deg_v, int32_t deg_c, double v_min, double v_max,
+                                      double c_min_fF, double c_max_fF, double *beta, double *rms);
+
 typedef struct {
     int64_t evals;               /* gates x simulated slots                  */
     int64_t slots, slot_warps;   /* simulated slots / 32-slot groups         */

@@ -5,8 +5,8 @@ The product is the C-ABI library libavfs.so (include/avfs.h, csrc/); this
 package holds its thin ctypes binding and the multi-GPU slot sharding.  There
 is no CPU fallback: without the built library, Context() raises.
 """
-from .avfs import (AvfsError, Context, EXPORTS, LIB_PATH, load_library, load_workload)
+from .avfs import (AvfsError, Context, EXPORTS, LIB_PATH, fit_delay_polynomial, load_library, load_workload)
 from .parallel import shard_range, reduce_results
 
-__all__ = ["AvfsError", "Context", "EXPORTS", "LIB_PATH", "load_library", "load_workload",
+__all__ = ["AvfsError", "Context", "EXPORTS", "LIB_PATH", "fit_delay_polynomial", "load_library", "load_workload",
            "shard_range", "reduce_results"]

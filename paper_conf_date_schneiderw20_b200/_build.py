@@ -8,7 +8,7 @@ PKG = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(PKG)
 CSRC = os.path.join(PKG, "csrc")
 LIB = os.path.join(PKG, "libavfs.so")
-SOURCES = [os.path.join(CSRC, f) for f in ("avfs_host.cpp", "avfs_kernels.cu")]
+SOURCES = [os.path.join(CSRC, f) for f in ("avfs_host.cpp", "avfs_kernels.cu", "avfs_fit.cpp")]
 HEADERS = [os.path.join(CSRC, "avfs_internal.h"), os.path.join(ROOT, "include", "avfs.h")]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 FLAGS = ["-gencode", "arch=compute_100a,code=sm_100a", "-lineinfo", "-O3", "-std=c++17",

@@ -25,6 +25,7 @@ EXPORTS = [
     "avfs_set_options", "avfs_default_options", "avfs_simulate", "avfs_sync",
     "avfs_get_activity", "avfs_get_latest_arrival", "avfs_get_final_values",
     "avfs_get_waveforms", "avfs_get_stats", "avfs_capture", "avfs_get_switching_energy",
+    "avfs_fit_delay_polynomial",
 ]
 
 
@@ -100,6 +101,7 @@ def load_library(path: str = LIB_PATH):
             "avfs_get_stats": ([P, P], C.c_int),
             "avfs_capture": ([P, P, I32, C.c_float, C.c_float, P, P, P, P], C.c_int),
             "avfs_get_switching_energy": ([P, P], C.c_int),
+            "avfs_fit_delay_polynomial": ([I64, P, P, P, I32, I32, D, D, D, D, P, P], C.c_int),
         }
         for name, (args, res) in sig.items():
             f = getattr(lib, name)
@@ -314,6 +316,21 @@ class Context:
         st = avfs_stats()
         self._ck(self.lib.avfs_get_stats(self.h, C.byref(st)))
         return st.as_dict()
+
+
+def fit_delay_polynomial(v, c, y, deg_v, deg_c, v_min=0.55, v_max=1.1, c_min=0.5, c_max=128.0):
+    """NEXT-3: OLS fit of Eq. (4) (normal equation, Eq. 8).  Returns (beta [deg_v+1][deg_c+1], rms)."""
+    lib = load_library()
+    vv = _c(v, np.float64)
+    cc = None if c is None else _c(c, np.float64)
+    yy = _c(y, np.float64)
+    beta = np.zeros((deg_v + 1) * (deg_c + 1), np.float64)
+    rms = np.zeros(1, np.float64)
+    st = lib.avfs_fit_delay_polynomial(len(vv), _p(vv), _p(cc), _p(yy), int(deg_v), int(deg_c), float(v_min),
+                                       float(v_max), float(c_min), float(c_max), _p(beta), _p(rms))
+    if st:
+        raise AvfsError(st, "avfs_fit_delay_polynomial failed")
+    return beta.reshape(deg_v + 1, deg_c + 1), float(rms[0])
 
 
 def load_workload(ctx: Context, netlist, library, stimuli, vdd):
