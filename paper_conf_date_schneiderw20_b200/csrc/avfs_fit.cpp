@@ -40,13 +40,16 @@ extern "C" avfs_status avfs_fit_delay_polynomial(int64_t n, const double* v, con
             for (int e = 0; e <= a; ++e) A[(size_t)a * m + e] += row[a] * row[e];
         }
     }
-    // Cholesky A = L L^T (lower triangle of A holds X^T X)
+    // Cholesky A = L L^T (lower triangle of A holds X^T X); a pivot that
+    // vanishes relative to its column norm means a rank-deficient design
+    std::vector<double> diag(m);
+    for (int a = 0; a < m; ++a) diag[a] = A[(size_t)a * m + a];
     for (int a = 0; a < m; ++a) {
         for (int e = 0; e <= a; ++e) {
             double s = A[(size_t)a * m + e];
             for (int f = 0; f < e; ++f) s -= A[(size_t)a * m + f] * A[(size_t)e * m + f];
             if (a == e) {
-                if (!(s > 0)) return AVFS_ERR_ARG;       // rank deficient design
+                if (!(s > 1e-12 * diag[a])) return AVFS_ERR_ARG;   // rank deficient design
                 A[(size_t)a * m + a] = std::sqrt(s);
             } else {
                 A[(size_t)a * m + e] = s / A[(size_t)e * m + e];
