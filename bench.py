@@ -97,16 +97,52 @@ class ClockSampler:
                 "reasons": reasons, "samples": len(sm)}
 
 
+# AVFS_BENCH_SHARE_GPU=1: every rank uses cuda:0 and gloo collectives on CPU
+# tensors -- exercises the multi-rank path on a single-GPU box (testing only).
+SHARE_GPU = os.environ.get("AVFS_BENCH_SHARE_GPU", "0") == "1"
+
+
 def dist_setup(n_gpus):
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
-    local = int(os.environ.get("LOCAL_RANK", "0"))
+    local = 0 if SHARE_GPU else int(os.environ.get("LOCAL_RANK", "0"))
     if world > 1:
         import torch
         import torch.distributed as dist
-        torch.cuda.set_device(local)
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        if SHARE_GPU:
+            dist.init_process_group("gloo")
+        else:
+            torch.cuda.set_device(local)
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     return world, rank, local
+
+
+def _reduce(t, op):
+    """dist.reduce to rank 0 (on the collective's device)."""
+    import torch.distributed as dist
+    if SHARE_GPU:
+        c = t.cpu()
+        dist.reduce(c, dst=0, op=op)
+        t.copy_(c)
+    else:
+        dist.reduce(t, dst=0, op=op)
+
+
+def _max_over_ranks(x, dev):
+    import torch
+    import torch.distributed as dist
+    t = torch.tensor([x], dtype=torch.float64, device="cpu" if SHARE_GPU else dev)
+    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    return float(t.item())
+
+
+def host_cores() -> int:
+    """All cores this process may run on (torchrun sets OMP_NUM_THREADS=1; the
+    oracle runs on rank 0 only, so it takes every core explicitly)."""
+    try:
+        return len(os.sched_getaffinity(0))
+    except AttributeError:
+        return os.cpu_count() or 1
 
 
 def cpu_baseline(w, target_s=15.0):
@@ -114,7 +150,7 @@ def cpu_baseline(w, target_s=15.0):
     import oracle
     P, V = w.stimuli.n_pairs, len(w.vdd)
     rng = np.random.default_rng(12345)
-    threads = oracle.max_threads()
+    threads = host_cores()
 
     def run(n):
         s = np.sort(rng.choice(P * V, size=n, replace=False))
@@ -139,7 +175,7 @@ def run_reference(args, w, world, rank):
         return
     import oracle
     P, V = w.stimuli.n_pairs, len(w.vdd)
-    threads = oracle.max_threads()
+    threads = host_cores()
     rng = np.random.default_rng(777)
     # size each step so the whole --steps K --warmup W run stays within a few minutes
     probe = np.sort(rng.choice(P * V, size=max(threads, 4), replace=False))
@@ -232,8 +268,8 @@ def main():
             ctx.activity(act_dev)
             lat_dev.copy_(torch.from_numpy(ctx.latest_arrival()))
             with torch.cuda.stream(stream):
-                dist.reduce(act_dev, dst=0, op=dist.ReduceOp.SUM)
-                dist.reduce(lat_dev, dst=0, op=dist.ReduceOp.MAX)
+                _reduce(act_dev, dist.ReduceOp.SUM)          # the only collective
+                _reduce(lat_dev, dist.ReduceOp.MAX)
 
     for _ in range(args.warmup):
         step()
@@ -260,9 +296,7 @@ def main():
     t_total = float(np.sum(step_ms))
     if world > 1:
         import torch.distributed as dist
-        t = torch.tensor([t_total], device=dev)
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        t_total = float(t.item())
+        t_total = _max_over_ranks(t_total, dev)
         dist.barrier()
     stats = ctx.stats()
     evals_total = w.netlist.n_gates * total_slots
@@ -296,17 +330,14 @@ def main():
                 import torch.distributed as dist
                 ta = torch.from_numpy(a.view(np.int64)).to(dev)
                 tl = torch.from_numpy(lat).to(dev)
-                dist.reduce(ta, dst=0, op=dist.ReduceOp.SUM)
-                dist.reduce(tl, dst=0, op=dist.ReduceOp.MAX)
+                _reduce(ta, dist.ReduceOp.SUM)
+                _reduce(tl, dist.ReduceOp.MAX)
                 a = ta.cpu()
             if i > 0:
                 e2e_ms.append((time.perf_counter() - t0) * 1e3)
         te = float(np.sum(e2e_ms))
         if world > 1:
-            import torch.distributed as dist
-            t = torch.tensor([te], device=dev)
-            dist.all_reduce(t, op=dist.ReduceOp.MAX)
-            te = float(t.item())
+            te = _max_over_ranks(te, dev)
         e2e = {"value": evals_total * args.steps / (te / 1e3), "unit": UNIT,
                "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h}
 
