@@ -1,0 +1,20 @@
+"""Small end-to-end runs for compute-sanitizer (c17 keep-all, multiplier with reruns, random DAG)."""
+import os, sys
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import numpy as np
+from paper_conf_date_schneiderw20_b200 import Context, load_workload
+from workloads import make_config
+
+for cfg, kw in ((1, dict(n_pairs=64)), (2, dict(n_pairs=64, n_vdd=2)), (3, dict(n_pairs=64, n_vdd=2, scale=0.02))):
+    w = make_config(cfg, **kw)
+    for cap in (1, 8):
+        ctx = Context(0)
+        load_workload(ctx, w.netlist, w.library, w.stimuli, w.vdd)
+        ctx.set_options(capacity=cap, keep_all=(cfg == 1), max_rerun_rounds=4)
+        ctx.simulate()
+        a = ctx.activity()
+        ctx.waveforms(w.netlist.po_sig, 0, w.n_slots, cap=8)
+        ctx.capture(np.full(len(w.vdd), 50.0, np.float32))
+        ctx.switching_energy()
+        print(cfg, cap, int(a.sum()), ctx.stats()["rerun_rounds"], flush=True)
+        ctx.close()
