@@ -16,7 +16,7 @@ from tests.parity import gpu_run, gpu_waveforms, compare, activity_ref
 
 pytestmark = pytest.mark.gpu
 
-SAMPLES = {2: 64, 3: 48, 4: 32, 5: 6}
+SAMPLES = {2: 256, 3: 128, 4: 96, 5: 12}
 # config 5 is specified on 8 x B200: one GPU simulates one eighth of its slots
 SHARD = {5: (0, 8)}
 
@@ -33,17 +33,18 @@ def sample_slots(w, n):
     return np.sort(first + rng.choice(cnt, size=n, replace=False))
 
 
-@pytest.mark.parametrize("cfg", [2, 3, 4, pytest.param(5, marks=pytest.mark.slow)])
-def test_fullsize_sampled_po_parity(cfg):
+@pytest.mark.parametrize("cfg,quantum", [(2, 0.0), (3, 0.0), (4, 0.0), pytest.param(5, 0.0, marks=pytest.mark.slow),
+                                         (2, 2.0 ** -8), (4, 2.0 ** -8)])
+def test_fullsize_sampled_po_parity(cfg, quantum):
     w = make_config(cfg)
     nl = w.netlist
     first, cnt = slot_window(w)
-    ctx = gpu_run(w, keep_all=False, slot_range=(first, cnt))
+    ctx = gpu_run(w, keep_all=False, slot_range=(first, cnt), quantum=quantum)
     st = ctx.stats()
     assert st["evals"] == w.netlist.n_gates * cnt
     slots = sample_slots(w, SAMPLES[cfg])
     P = w.stimuli.n_pairs
-    ref = oracle.simulate(nl, w.library, w.stimuli, w.vdd, slots % P, slots // P, quantum=0.0,
+    ref = oracle.simulate(nl, w.library, w.stimuli, w.vdd, slots % P, slots // P, quantum=quantum,
                           cap=64, out_sig=nl.po_sig)
     cap = max(1, min(64, int(ref.count.max())))
     init = np.zeros((len(slots), len(nl.po_sig)), np.uint8)
@@ -53,7 +54,9 @@ def test_fullsize_sampled_po_parity(cfg):
         a, b, c = gpu_waveforms(ctx, nl.po_sig, int(s), 1, cap)
         init[i], cnt[i], times[i] = a[0], b[0], c[0]
     ref.times = ref.times[:, :, :cap]
-    r = compare(ref, init, cnt, np.minimum(times, np.float32(3e38)), 0.0, f"cfg{cfg}")
+    r = compare(ref, init, cnt, times, quantum, f"cfg{cfg}-q{quantum}")
+    if quantum > 0:
+        assert r["tainted"] == 0
     assert r["events"] > 0
     # latest arrival bounds the sampled PO transitions
     lat = ctx.latest_arrival()
