@@ -59,7 +59,7 @@ struct Round {
     int64_t n_sw = 0;
     int64_t sw_first = 0;            // pass 0: contiguous range
     std::vector<int32_t> sws;        // reruns: explicit list
-    int32_t capacity = 0, W = 0, cstage = 0, stage_words = 0;
+    int32_t capacity = 0, W = 0;
     int64_t region_bytes = 0;
     int32_t grid = 0;
 };
@@ -805,17 +805,13 @@ avfs_status avfs_sync(avfs_ctx* ctx) {
 }
 
 static avfs_status run_round(avfs_ctx* ctx, Round& R, int round_idx, const int32_t* d_sw_list, int32_t prev_W,
-                             int32_t prev_cstage, bool timed) {
+                             bool timed) {
     const bool persistent = (round_idx == 0);
     // launch bounds: sweep_kernel up to 1024 threads, level_kernel 512 threads
-    int wpc = ctx->opt.warps_per_cta > 0 ? ctx->opt.warps_per_cta : (persistent ? 32 : 16);
-    wpc = std::min(wpc, persistent ? 32 : 16);
-    // input staging budget per warp: min(max fan-in, 2) x W words (more -> overflow, rerun)
-    const int stage_words = std::min(ctx->kmax, 2) * R.W;
-    R.stage_words = stage_words;
-    int smem = sweep_smem_bytes(wpc, stage_words, R.cstage);
-    while (wpc > 1 && smem > 227 * 1024) smem = sweep_smem_bytes(--wpc, stage_words, R.cstage);
-    if (smem > 227 * 1024) return fail(ctx, AVFS_ERR_CAPACITY, "capacity %d needs %d B shared memory per warp", R.capacity, smem);
+    const int wmax = persistent ? AVFS_SWEEP_THREADS / 32 : 16;
+    int wpc = ctx->opt.warps_per_cta > 0 ? ctx->opt.warps_per_cta : wmax;
+    wpc = std::min(wpc, wmax);
+    const int smem = persistent ? sweep_smem_bytes(wpc) : level_smem_bytes(wpc);
     int bps = 0;
     if (persistent) CK(sweep_occupancy(wpc, smem, &bps));
     else CK(level_occupancy(wpc, smem, &bps));
@@ -851,18 +847,10 @@ static avfs_status run_round(avfs_ctx* ctx, Round& R, int round_idx, const int32
     p.arena = ctx->arena[round_idx].as<uint8_t>();
     p.region_bytes = R.region_bytes;
     p.W = R.W;
-    p.stage_words = stage_words;
-    p.cstage = R.cstage;
     p.prev_W = prev_W;
-    p.prev_cstage = prev_cstage;
-    p.prev_stage_words = prev_W ? std::min(ctx->kmax, 2) * prev_W : 0;
     p.act = ctx->d_act.as<unsigned long long>();
     p.latest = ctx->d_latest.as<unsigned int>();
     p.ovf = ctx->d_ovf.as<int32_t>();
-    {
-        const char* dg = getenv("AVFS_DYN_GRAB");
-        p.dyn_grab = dg ? atoi(dg) : 0;   // measured: static striding is as fast at 32 warps/CTA
-    }
     CK(launch_pi_regions(p, ctx->n_pi, ctx->stream));   // materialise the PI waveforms of this round
     ctx->stats.launches++;
     if (timed) CK(cudaEventRecord(ctx->ev0, ctx->stream));
@@ -951,9 +939,8 @@ avfs_status avfs_simulate(avfs_ctx* ctx, void* cuda_stream) {
     R0.sw_first = sw_lo;
     R0.capacity = ctx->opt.capacity;
     R0.W = 32 * R0.capacity;
-    R0.cstage = 2 * R0.capacity;
     R0.region_bytes = 128 + 4 * (int64_t)R0.W;
-    st = run_round(ctx, R0, 0, nullptr, 0, 0, ctx->opt.profile != 0);
+    st = run_round(ctx, R0, 0, nullptr, 0, ctx->opt.profile != 0);
     if (st != AVFS_OK) return st;
     ctx->rounds.push_back(R0);
     int cur = 0;
@@ -981,11 +968,10 @@ avfs_status avfs_simulate(avfs_ctx* ctx, void* cuda_stream) {
         CK(cudaMemcpy(Rn.sws.data(), ctx->d_list[cur].p, n_ovf * sizeof(int32_t), cudaMemcpyDeviceToHost));
         Rn.capacity = std::min(prev.capacity * 4, 1024);
         Rn.W = 32 * Rn.capacity;
-        Rn.cstage = 2 * Rn.capacity;
         Rn.region_bytes = 128 + 4 * (int64_t)Rn.W;
         ctx->stats.overflow_slot_warps += n_ovf;
         ctx->stats.rerun_rounds++;
-        st = run_round(ctx, Rn, r + 1, ctx->d_list[cur].as<int32_t>(), prev.W, prev.cstage, false);
+        st = run_round(ctx, Rn, r + 1, ctx->d_list[cur].as<int32_t>(), prev.W, false);
         if (st != AVFS_OK) return st;
         ctx->rounds.push_back(std::move(Rn));
         cur ^= 1;

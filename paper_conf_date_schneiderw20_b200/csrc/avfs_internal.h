@@ -6,6 +6,14 @@
 
 namespace avfs {
 
+// sweep CTA shape (compile-time; A/B knobs via -D)
+#ifndef AVFS_SWEEP_THREADS
+#define AVFS_SWEEP_THREADS 1024
+#endif
+#ifndef AVFS_SWEEP_MINB
+#define AVFS_SWEEP_MINB (AVFS_SWEEP_THREADS > 768 ? 1 : (AVFS_SWEEP_THREADS > 512 ? 2 : 3))
+#endif
+
 constexpr int KMAX = 4;            // max cell inputs (truth table is 16 bits)
 constexpr int MAX_DEG = 7;         // max polynomial degree per variable
 
@@ -83,11 +91,7 @@ struct SweepParams {
     uint8_t* arena;
     int64_t region_bytes;
     int32_t W;                              // event capacity per region (32*C)
-    int32_t stage_words;                    // per-warp input staging: min(max fan-in, 2) x W
-    int32_t cstage;                         // per-slot capacity (2*C)
-    int32_t prev_W, prev_cstage;            // previous round (0: first pass)
-    int32_t prev_stage_words;               // previous round's staging budget (0: first pass)
-    int32_t dyn_grab;                       // 1: warps take gates of a level from a shared counter
+    int32_t prev_W;                         // previous round's W (0: first pass)
     // outputs
     unsigned long long* act;                // [n_signals][n_vdd]
     unsigned int* latest;                   // [n_vdd] float bits (non-negative)
@@ -95,7 +99,8 @@ struct SweepParams {
 };
 
 // launch wrappers (avfs_kernels.cu)
-int sweep_smem_bytes(int warps_per_cta, int stage_words, int cstage);
+int sweep_smem_bytes(int warps_per_cta);
+int level_smem_bytes(int warps_per_cta);
 cudaError_t sweep_occupancy(int warps_per_cta, int smem, int* blocks_per_sm);
 cudaError_t launch_delays(const DelayParams& p, cudaStream_t st);
 cudaError_t launch_sweep(const SweepParams& p, int grid, int warps_per_cta, cudaStream_t st);

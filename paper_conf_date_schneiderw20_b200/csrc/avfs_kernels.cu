@@ -15,15 +15,14 @@
 //                           processing); warp w evaluates gates w, w+nw, ...
 //                           of the level for the 32 slots (the
 //                           horizontal plane = one gate, all slots).  Per
-//                           gate: FP64 Horner delays lane-parallel (P:L139,
-//                           P:L152-L160 steps 1-5, Eq. 9), coalesced header
-//                           loads, cp.async 16-B staging of the compact input
-//                           event lists into shared memory, per-slot k-way
-//                           merge with the inertial filter (reading
-//                           C3-C6), compaction of the outputs through shared
-//                           memory, 128-bit stores, warp-ballot overflow
-//                           detection and activity / latest-arrival
-//                           reductions (P:L141 step 4).
+//                           gate: delays from the FP64 delay table (P:L139,
+//                           Eq. 9), coalesced header loads, an
+//                           event-parallel merge + inertial filter (P:L148,
+//                           readings C3-C6) built from warp ballots, compact
+//                           stores, capacity check, activity and
+//                           latest-arrival reductions (P:L141 step 4).
+//   level_kernel        H7  the same evaluation, one launch per level, for
+//                           the overflow reruns.
 //   compact_kernel      H7  list of overflowed slot groups for the rerun.
 //   gather_kernel       H9  readback of kept waveforms.
 #include <cuda_runtime.h>
@@ -38,54 +37,528 @@ namespace avfs {
 __device__ __forceinline__ uint32_t ld_u32(const void* p) {
     return __ldcg(reinterpret_cast<const unsigned int*>(p));
 }
+__device__ __forceinline__ float ld_f32(const void* p) { return __ldcg(reinterpret_cast<const float*>(p)); }
 
-__device__ __forceinline__ void cp_async16(void* smem, const void* gmem) {
-    uint32_t s = static_cast<uint32_t>(__cvta_generic_to_shared(smem));
-    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"(s), "l"(gmem) : "memory");
+__device__ __forceinline__ uint32_t lanemask_lt() {
+    uint32_t m;
+    asm("mov.u32 %0, %%lanemask_lt;" : "=r"(m));
+    return m;
 }
-__device__ __forceinline__ void cp_async16_a(uint32_t s, const void* gmem) {
-    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;\n" ::"r"(s), "l"(gmem) : "memory");
-}
-// TMA bulk copy global -> shared, completion signalled on an mbarrier (tx bytes)
-__device__ __forceinline__ void tma_bulk_g2s(uint32_t dst, const void* src, uint32_t bytes, uint32_t bar) {
-    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];\n"
-                 ::"r"(dst), "l"(src), "r"(bytes), "r"(bar) : "memory");
-}
-__device__ __forceinline__ void mbar_init(uint32_t bar) {
-    asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;\n" ::"r"(bar) : "memory");
-    asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
-}
-__device__ __forceinline__ void mbar_expect_tx(uint32_t bar, uint32_t bytes) {
-    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;\n" ::"r"(bar), "r"(bytes) : "memory");
-}
-__device__ __forceinline__ void mbar_wait(uint32_t bar, uint32_t phase) {
-    asm volatile(
-        "{\n .reg .pred P;\n WAIT_%=:\n"
-        " mbarrier.try_wait.parity.shared::cta.b64 P, [%0], %1;\n"
-        " @!P bra WAIT_%=;\n}\n" ::"r"(bar), "r"(phase) : "memory");
-}
-__device__ __forceinline__ void fence_proxy_async_smem() {
-    asm volatile("fence.proxy.async.shared::cta;\n" ::: "memory");
-}
-__device__ __forceinline__ void fence_proxy_async_global() {
-    asm volatile("fence.proxy.async.global;\n" ::: "memory");
-}
-__device__ __forceinline__ void cp_async_wait_all() {
-    asm volatile("cp.async.wait_all;\n" ::: "memory");
-}
-__device__ __forceinline__ void st_global_v4(void* p, float4 v) {
-    asm volatile("st.global.v4.f32 [%0], {%1, %2, %3, %4};\n" ::"l"(p), "f"(v.x), "f"(v.y), "f"(v.z),
-                 "f"(v.w)
-                 : "memory");
+__device__ __forceinline__ uint32_t lanemask_le() {
+    uint32_t m;
+    asm("mov.u32 %0, %%lanemask_le;" : "=r"(m));
+    return m;
 }
 
-__device__ __forceinline__ uint32_t warp_incl_scan(uint32_t v, int lane) {
+// inclusive warp prefix sum; the shuffle's in-range predicate guards the add
+__device__ __forceinline__ uint32_t warp_incl_scan(uint32_t v, int) {
 #pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
-        uint32_t u = __shfl_up_sync(0xffffffffu, v, o);
-        if (lane >= o) v += u;
-    }
+    for (int o = 1; o < 32; o <<= 1)
+        asm("{\n .reg .pred p;\n .reg .b32 u;\n"
+            " shfl.sync.up.b32 u|p, %0, %1, 0, 0xffffffff;\n"
+            " @p add.u32 %0, %0, u;\n}\n" : "+r"(v) : "r"(o));
     return v;
+}
+
+#define AVFS_INF __int_as_float(0x7f800000)
+#define FULL 0xffffffffu
+
+// ---------------------------------------------------------------------------
+// Gate evaluation for one gate x one 32-slot group.
+//
+// Lane l = slot l.  The K input header words (staged rows in shared memory,
+// or one coalesced 128-B row each) give per slot the event counts n_q, the
+// offsets of the event lists, the initial input values and hence the
+// initial output y0 = TT(inputs) (reading C1).  m = sum_q n_q bounds the
+// slot's output events; its warp prefix sum places slot l's outputs at
+// offset base(l) of the output region (the header stores offset and count).
+// Each lane then merges its K sorted lists (ties: ascending pin, reading C5)
+// for exactly max_l m(l) steps, evaluating the truth table after every input
+// event and applying the inertial filter (reading C3: a change whose
+// time precedes the pending output cancels it, reading C4: no reschedule on
+// confirming events); surviving outputs t + d(pin, polarity) (Eq. 9 delays)
+// are stored as they are pushed -- only the last one can later be cancelled,
+// and the next push overwrites it.
+//
+// Capacity: the region of a 32-slot group holds W = 32 C times; a gate-warp
+// whose inputs carry more than W events in total (an upper bound of its
+// outputs) is poisoned and the slot group rerun at 4C (reading C17).
+// ---------------------------------------------------------------------------
+
+struct Env {
+    uint8_t* row;                  // arena + i * region_bytes
+    uint32_t stride;               // bytes between buffers = n_sw * region_bytes (< 4 GiB, checked on host)
+    int64_t i;                     // index of the slot group in the round (overflow flag)
+    int kv, lane;
+    unsigned long long* act_kv;    // &act[0][kv]
+};
+
+__device__ __forceinline__ uint8_t* region(uint32_t buf, const Env& E) {
+    return E.row + (uint64_t)buf * (uint64_t)E.stride;
+}
+
+__device__ __forceinline__ uint32_t smem_u32(const void* p) {
+    return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+__device__ __forceinline__ float lds_f32(uint32_t a) {
+    float v;
+    asm volatile("ld.shared.f32 %0, [%1];" : "=f"(v) : "r"(a));
+    return v;
+}
+__device__ __forceinline__ uint32_t lds_u32(uint32_t a) {
+    uint32_t v;
+    asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v) : "r"(a));
+    return v;
+}
+__device__ __forceinline__ void cp_async16(uint32_t dst, const void* src) {
+    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(dst), "l"(src) : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+__device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_all;" ::: "memory"); }
+
+constexpr int EV_STAGE = 256;   // staged event words per gate (EV_STAGE / K' per input)
+
+// Where a gate's inputs are: header rows (4 x 32 words) and, if they fit, the
+// inputs' compact event lists staged in shared memory by the sweep pipeline.
+struct Staged {
+    bool hdr, ev;
+    uint32_t hdr_s;       // shared address of header row 0 (row q at + 128 q)
+    uint32_t ev_s[1];     // shared address of the staged events (input q at + 4 EV_STAGE q / K')
+    uint32_t dly_s;       // shared address of the gate's 8 delays [pin][pol]
+};
+__device__ __forceinline__ float4 lds_f32x4(uint32_t a) {
+    float4 v;
+    asm volatile("ld.shared.v4.f32 {%0, %1, %2, %3}, [%4];" : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w) : "r"(a));
+    return v;
+}
+
+// Lane-serial merge + inertial filter of one slot.  Input q's list: n[q]
+// events from ev[q] (shared-memory addresses if STAGED, else global
+// pointers); outputs go to out[0..).  Runs exactly `steps` (= the warp's max
+// m) steps; lanes with fewer events idle through the rest.  Returns the
+// output count.  One step: take the earliest head (ties: lower pin), flip
+// that pin, evaluate the truth table, and apply the filter.
+struct MergeIn {
+    uint64_t ev[KMAX];
+    int n[KMAX];
+    uint32_t bits, proj, tt, dly_s;
+    float4 d01;           // delays of pins 0, 1: {p0 fall, p0 rise, p1 fall, p1 rise}
+};
+
+template <bool STAGED>
+__device__ __forceinline__ float ld_ev(uint64_t a) {
+    return STAGED ? lds_f32((uint32_t)a) : ld_f32(reinterpret_cast<const void*>(a));
+}
+
+// Address arithmetic of the list walk: 32-bit shared-memory addresses when
+// STAGED, 64-bit global pointers otherwise.
+template <bool STAGED> struct EvAddr { typedef uint64_t T; };
+template <> struct EvAddr<true> { typedef uint32_t T; };
+
+template <int K, bool STAGED>
+__device__ __forceinline__ uint32_t merge_slot(const MergeIn& M, float* out, uint32_t steps) {
+    typedef typename EvAddr<STAGED>::T A;
+    uint32_t bits = M.bits, proj = M.proj;
+    const uint32_t tt = M.tt;
+    float* op = out;                             // next output slot (only the last output can be cancelled)
+    float tl = -AVFS_INF;
+    auto step = [&](float t, bool live, uint32_t y, float d) {
+        const float co = t + d;
+        const bool change = live && y != proj;
+        const bool cancel = change && tl > t;
+        const bool push = change && !cancel;
+        if (push) __stcg(op, co);
+        op += push ? 1 : (cancel ? -1 : 0);
+        tl = push ? co : (cancel ? -AVFS_INF : tl);
+        proj = y;
+    };
+    if (K == 1) {
+        A a = (A)M.ev[0];
+        const A e = a + 4 * (uint32_t)M.n[0];
+        float h = a < e ? ld_ev<STAGED>(a) : AVFS_INF;
+#pragma unroll 1
+        for (uint32_t it = 0; it < steps; ++it) {
+            const float t = h;
+            a += 4;
+            h = a < e ? ld_ev<STAGED>(a) : AVFS_INF;
+            const bool live = t < AVFS_INF;
+            bits ^= live ? 1u : 0u;
+            const uint32_t y = (tt >> bits) & 1u;
+            step(t, live, y, y ? M.d01.y : M.d01.x);
+        }
+    } else if (K == 2) {
+        A a0 = (A)M.ev[0], a1 = (A)M.ev[1];
+        const A e0 = a0 + 4 * (uint32_t)M.n[0], e1 = a1 + 4 * (uint32_t)M.n[1];
+        float h0 = a0 < e0 ? ld_ev<STAGED>(a0) : AVFS_INF;
+        float h1 = a1 < e1 ? ld_ev<STAGED>(a1) : AVFS_INF;
+        a0 += 4;
+        a1 += 4;
+#pragma unroll 1
+        for (uint32_t it = 0; it < steps; ++it) {
+            const bool p = h1 < h0;             // ties: pin 0 first
+            const float t = p ? h1 : h0;
+            const A a = p ? a1 : a0;
+            const float nx = a < (p ? e1 : e0) ? ld_ev<STAGED>(a) : AVFS_INF;
+            h1 = p ? nx : h1;
+            h0 = p ? h0 : nx;
+            a1 = p ? a + 4 : a1;
+            a0 = p ? a0 : a + 4;
+            const bool live = t < AVFS_INF;
+            bits ^= live ? (p ? 2u : 1u) : 0u;
+            const uint32_t y = (tt >> bits) & 1u;
+            step(t, live, y, p ? (y ? M.d01.w : M.d01.z) : (y ? M.d01.y : M.d01.x));
+        }
+    } else {
+        float h[K];
+        A a[K], e[K];
+#pragma unroll
+        for (int q = 0; q < K; ++q) {
+            a[q] = (A)M.ev[q];
+            e[q] = a[q] + 4 * (uint32_t)M.n[q];
+            h[q] = a[q] < e[q] ? ld_ev<STAGED>(a[q]) : AVFS_INF;
+            a[q] += 4;
+        }
+#pragma unroll 1
+        for (uint32_t it = 0; it < steps; ++it) {
+            float t = h[0];
+            int pm = 0;
+#pragma unroll
+            for (int q = 1; q < K; ++q) {
+                const bool lt = h[q] < t;
+                t = lt ? h[q] : t;
+                pm = lt ? q : pm;
+            }
+            A ap = a[0], ep = e[0];
+#pragma unroll
+            for (int q = 1; q < K; ++q)
+                if (pm == q) { ap = a[q]; ep = e[q]; }
+            const float nx = ap < ep ? ld_ev<STAGED>(ap) : AVFS_INF;
+#pragma unroll
+            for (int q = 0; q < K; ++q)
+                if (pm == q) { h[q] = nx; a[q] = ap + 4; }
+            const bool live = t < AVFS_INF;
+            bits ^= live ? (1u << pm) : 0u;
+            const uint32_t y = (tt >> bits) & 1u;
+            step(t, live, y, lds_f32(M.dly_s + 8 * pm + 4 * y));
+        }
+    }
+    return (uint32_t)(op - out);
+}
+
+template <int K>
+__device__ __forceinline__ void eval_gate(const SweepParams& p, const Env& E, const uint4 ins, const uint4 hd,
+                                          const Staged& S) {
+    const int lane = E.lane;
+    const uint32_t out_loc = hd.x, sig = hd.y;
+    const uint32_t tt = hd.z & 0xffffu;
+    const uint32_t in_loc[KMAX] = {ins.x, ins.y, ins.z, ins.w};
+    uint32_t hw[KMAX];
+#pragma unroll
+    for (int q = 0; q < K; ++q)
+        hw[q] = S.hdr ? lds_u32(S.hdr_s + 128 * q + 4 * lane)
+                      : __ldcg(reinterpret_cast<const uint32_t*>(region(in_loc[q], E)) + lane);
+    int n[KMAX] = {0, 0, 0, 0};
+    uint32_t bits = 0, orh = 0;
+    int m = 0;
+#pragma unroll
+    for (int q = 0; q < K; ++q) {
+        n[q] = (int)(hw[q] & HDR_N);
+        bits |= ((hw[q] >> HDR_INIT_SHIFT) & 1u) << q;
+        orh |= hw[q];
+        m += n[q];
+    }
+    const uint32_t y0 = (tt >> bits) & 1u;
+    uint8_t* ro = region(out_loc, E);
+    uint32_t* ro_hdr = reinterpret_cast<uint32_t*>(ro);
+    const bool first_pass = (p.prev_W == 0);
+    // one warp reduction: upstream poison / previous-capacity flags, any input event
+    const uint32_t R = __reduce_or_sync(FULL, (orh & (HDR_POISON | HDR_PREV)) | (m != 0 ? 1u : 0u));
+    if (R & HDR_POISON) {                               // upstream overflow: nothing valid here
+        __stcg(ro_hdr + lane, HDR_POISON | HDR_PREV | (y0 << HDR_INIT_SHIFT));
+        return;
+    }
+    const bool any_prev = first_pass || (R & HDR_PREV);
+    if (!(R & 1u)) {                                    // no input event in any slot: constant output
+        __stcg(ro_hdr + lane, (y0 << HDR_INIT_SHIFT) | (any_prev ? HDR_PREV : 0u));
+        return;
+    }
+    const uint32_t incl = warp_incl_scan((uint32_t)m, lane);
+    const uint32_t total_in = __shfl_sync(FULL, incl, 31);
+    const uint32_t base = incl - (uint32_t)m;
+    const uint32_t maxm = __reduce_max_sync(FULL, (uint32_t)m);
+    // capacity (reading C17): the inputs' events bound the outputs
+    const bool ovf = total_in > (uint32_t)p.W || maxm > HDR_N;
+    const bool prev = any_prev || total_in > (uint32_t)p.prev_W;
+    if (ovf) {
+        __stcg(ro_hdr + lane, HDR_POISON | (prev ? HDR_PREV : 0u) | (y0 << HDR_INIT_SHIFT));
+        if (lane == 0) p.ovf[p.i_base + E.i] = 1;
+        return;
+    }
+    float* out = reinterpret_cast<float*>(ro + 128) + base;
+    MergeIn M;
+    M.bits = bits;
+    M.proj = y0;
+    M.tt = tt;
+    M.dly_s = S.dly_s;
+    if (K <= 2) M.d01 = lds_f32x4(S.dly_s);
+#pragma unroll
+    for (int q = 0; q < KMAX; ++q) M.n[q] = n[q];
+    uint32_t my_n;
+    if (S.ev) {
+#pragma unroll
+        for (int q = 0; q < K; ++q)
+            M.ev[q] = S.ev_s[0] + (uint32_t)(4 * EV_STAGE / (K > 2 ? 4 : K)) * q + 4 * ((hw[q] >> HDR_OFF_SHIFT) & HDR_OFF);
+        my_n = merge_slot<K, true>(M, out, maxm);
+    } else {
+#pragma unroll
+        for (int q = 0; q < K; ++q)
+            M.ev[q] = reinterpret_cast<uint64_t>(region(in_loc[q], E) + 128) + 4 * ((hw[q] >> HDR_OFF_SHIFT) & HDR_OFF);
+        my_n = merge_slot<K, false>(M, out, maxm);
+    }
+    __stcg(ro_hdr + lane, my_n | (base << HDR_OFF_SHIFT) | (y0 << HDR_INIT_SHIFT) | (prev ? HDR_PREV : 0u));
+    // activity (reading C15) and latest PO arrival (P:L207): counted once per
+    // slot across overflow rounds (where prev && !ovf)
+    if (prev) {
+        const uint32_t total = __reduce_add_sync(FULL, my_n);
+        if (lane == 0 && total) atomicAdd(E.act_kv + (size_t)sig * (uint32_t)p.n_vdd, (unsigned long long)total);
+        if (hd.z & (1u << 24)) {
+            const float last = my_n ? __ldcg(out + my_n - 1) : 0.0f;
+            const uint32_t mx = __reduce_max_sync(FULL, __float_as_uint(last));
+            if (lane == 0 && mx) atomicMax(p.latest + E.kv, mx);
+        }
+    }
+}
+
+__device__ __forceinline__ void eval_dispatch(const SweepParams& p, const Env& E, const uint4 ins, const uint4 hd,
+                                              const Staged& S) {
+    switch ((hd.z >> 16) & 0xffu) {
+        case 1: eval_gate<1>(p, E, ins, hd, S); break;
+        case 2: eval_gate<2>(p, E, ins, hd, S); break;
+        case 3: eval_gate<3>(p, E, ins, hd, S); break;
+        default: eval_gate<4>(p, E, ins, hd, S); break;
+    }
+}
+
+__device__ __forceinline__ void slot_group(const SweepParams& p, int64_t i, int lane, Env& E) {
+    const int64_t sw = p.sw_list ? (int64_t)p.sw_list[i] : p.sw_first + i;
+    E.kv = (int)(sw / p.n_pw);
+    E.i = i;
+    E.lane = lane;
+    E.act_kv = p.act + E.kv;
+    E.row = p.arena + (p.i_base + i) * p.region_bytes;
+}
+
+// Per-warp shared memory (words): two descriptor windows of DW gates
+// (GateDesc 8 words each, then the gates' delays 8 words each), a header ring
+// 4 x 128 (4 input rows of 32 header words), an event ring 2 x EV_STAGE
+// (input q of a K-input gate owns EV_STAGE / K' words, K' = K rounded up to a
+// power of two), staged flags.
+constexpr int DW = 16;                                // gates per descriptor window
+constexpr int OFF_DESC = 0, OFF_HDR = OFF_DESC + 2 * 16 * DW, OFF_EV = OFF_HDR + 4 * 128,
+              OFF_META = OFF_EV + 2 * EV_STAGE;
+constexpr int WARP_SMEM_WORDS = OFF_META + 4;
+constexpr int LEVEL_SMEM_WORDS = 8;                   // delays of the current gate
+
+__device__ __forceinline__ float* warp_smem(int warp, int words) {
+    extern __shared__ __align__(16) float smem[];
+    return smem + 4 + (size_t)warp * words;
+}
+
+// Persistent level sweep (pass 0): one CTA owns one 32-slot group at a time
+// and walks all levels with a CTA barrier between levels.  Warp w
+// evaluates a contiguous block of each level's gates through a software
+// pipeline of asynchronous copies into shared memory (cp.async): descriptors
+// and delays arrive 16 gates at a time; at gate j the warp fetches the input
+// header rows of gate j+2 and the input event lists of gate j+1, so the
+// evaluation of gate j never waits for DRAM.  Event lists larger than the
+// stage are read from L2 by the evaluation instead.
+__global__ void __launch_bounds__(AVFS_SWEEP_THREADS, AVFS_SWEEP_MINB) sweep_kernel(const SweepParams p) {
+    const int lane = threadIdx.x & 31;
+    const int warp = threadIdx.x >> 5;
+    const int nw = blockDim.x >> 5;
+    Env E;
+    float* ws = warp_smem(warp, WARP_SMEM_WORDS);
+    const uint32_t s_desc = smem_u32(ws + OFF_DESC), s_hdr = smem_u32(ws + OFF_HDR), s_evr = smem_u32(ws + OFF_EV);
+    uint32_t* meta = reinterpret_cast<uint32_t*>(ws + OFF_META);
+    E.stride = (uint32_t)(p.pin_n_sw * p.region_bytes);
+    const uint4* gd = reinterpret_cast<const uint4*>(p.gates);
+    for (int64_t i = blockIdx.x; i < p.n_sw; i += gridDim.x) {
+        slot_group(p, i, lane, E);
+        const float4* dt = p.dtab + (int64_t)E.kv * p.n_gates * 2;
+        for (int L = 0; L < p.depth; ++L) {
+            const int ls = __ldg(p.level_ptr + L), le = __ldg(p.level_ptr + L + 1);
+            const int B = (le - ls + nw - 1) / nw;
+            const int g0 = ls + warp * B;
+            const int nj = max(0, min(B, le - g0));
+            // descriptor window k (gates g0 + 16k ..): lane copies 16 B of the
+            // descriptors (lanes 0..31 = 16 gates x 2) and 16 B of the delays
+            auto issue_win = [&](int k) {
+                const int g = g0 + DW * k + (lane >> 1);
+                const uint32_t w = s_desc + 4 * 16 * DW * (k & 1) + 16 * lane;
+                if (g < le) {
+                    cp_async16(w, gd + 2 * g + (lane & 1));
+                    cp_async16(w + 4 * 8 * DW, dt + 2 * g + (lane & 1));
+                }
+            };
+            auto desc_at = [&](int j) { return s_desc + 4 * 16 * DW * ((j / DW) & 1) + 32 * (j % DW); };
+            auto issue_hdr = [&](int j) {
+                const uint32_t d = desc_at(j);
+                const uint32_t q = (uint32_t)lane >> 3;
+                if (q < ((lds_u32(d + 24) >> 16) & 0xffu))
+                    cp_async16(s_hdr + 512 * (j & 3) + 128 * q + 16 * (lane & 7),
+                               region(lds_u32(d + 4 * q), E) + 16 * (lane & 7));
+            };
+            // input q's events (extent = lane 31's offset + count) -> slot q of
+            // the stage (EV_STAGE / K' words, 32 / K' lanes per input, <= 2
+            // chunks of 16 B per lane); staged only if every input fits
+            auto issue_ev = [&](int j) {
+                const uint32_t d = desc_at(j);
+                const uint32_t k = (lds_u32(d + 24) >> 16) & 0xffu;
+                const uint32_t sh = k > 2 ? 2u : (k > 1 ? 1u : 0u);      // log2 K'
+                const uint32_t q = (uint32_t)lane >> (5 - sh), sub = (uint32_t)lane & (31u >> sh);
+                uint32_t c = 0;
+                if (q < k) {
+                    const uint32_t w = lds_u32(s_hdr + 512 * (j & 3) + 128 * q + 124);
+                    c = (((w >> HDR_OFF_SHIFT) & HDR_OFF) + (w & HDR_N) + 3) >> 2;
+                }
+                const uint32_t cap = (uint32_t)(EV_STAGE / 4) >> sh;   // chunks per input
+                const bool staged = __all_sync(FULL, c <= cap);
+                if (lane == 0) meta[j & 1] = staged ? 1u : 0u;
+                if (staged && sub < c) {
+                    const uint8_t* src = region(lds_u32(d + 4 * q), E) + 128 + 16 * sub;
+                    const uint32_t dst = s_evr + 4 * EV_STAGE * (j & 1) + (4 * EV_STAGE >> sh) * q + 16 * sub;
+                    cp_async16(dst, src);
+                    const uint32_t st = 512u >> sh;                     // bytes covered by one pass of the lanes
+                    if (sub + (32u >> sh) < c) cp_async16(dst + st, src + st);
+                }
+            };
+            if (nj > 0) {
+                // prologue: descriptor windows 0, 1; header rows 0, 1; events of gate 0
+                issue_win(0);
+                if (nj > DW) issue_win(1);
+                cp_async_commit();
+                cp_async_wait_all();
+                __syncwarp();
+                issue_hdr(0);
+                if (nj > 1) issue_hdr(1);
+                cp_async_commit();
+                cp_async_wait_all();
+                __syncwarp();
+                issue_ev(0);
+                cp_async_commit();
+#pragma unroll 1
+                for (int j = 0; j < nj; ++j) {
+                    cp_async_wait_all();
+                    __syncwarp();
+                    if (j % DW == 0 && j > 0 && j + DW < nj) issue_win(j / DW + 1);
+                    if (j + 2 < nj) issue_hdr(j + 2);
+                    if (j + 1 < nj) issue_ev(j + 1);
+                    cp_async_commit();
+                    const uint32_t d = desc_at(j);
+                    const uint4* dv = reinterpret_cast<const uint4*>(ws + OFF_DESC + 16 * DW * ((j / DW) & 1) + 8 * (j % DW));
+                    Staged S;
+                    S.hdr = true;
+                    S.hdr_s = s_hdr + 512 * (j & 3);
+                    S.ev = meta[j & 1] != 0;
+                    S.dly_s = d + 4 * 8 * DW;
+                    S.ev_s[0] = s_evr + 4 * EV_STAGE * (j & 1);
+                    eval_dispatch(p, E, dv[0], dv[1], S);
+                }
+            }
+            __syncthreads();   // this level's stores -> the next levels' loads
+        }
+    }
+}
+
+// Level-parallel variant for overflow reruns (few slot groups): one launch per
+// level, warps take (gate, slot group) items of the level grid-wide.
+__global__ void __launch_bounds__(512, 2) level_kernel(const SweepParams p, int L) {
+    const int lane = threadIdx.x & 31;
+    const int warp = threadIdx.x >> 5;
+    Env E;
+    float* ws = warp_smem(warp, LEVEL_SMEM_WORDS);
+    E.stride = (uint32_t)(p.pin_n_sw * p.region_bytes);
+    const uint4* gd = reinterpret_cast<const uint4*>(p.gates);
+    Staged S;
+    S.hdr = false;
+    S.ev = false;
+    S.dly_s = smem_u32(ws);
+    const int g0 = __ldg(p.level_ptr + L);
+    const int64_t items = (int64_t)(__ldg(p.level_ptr + L + 1) - g0) * p.n_sw;
+    const int64_t gw = (int64_t)blockIdx.x * (blockDim.x >> 5) + warp;
+    const int64_t nwarps = (int64_t)gridDim.x * (blockDim.x >> 5);
+    for (int64_t it = gw; it < items; it += nwarps) {
+        const int gi = g0 + (int)(it / p.n_sw);
+        const int64_t i = it % p.n_sw;
+        slot_group(p, i, lane, E);
+        const float* dt = reinterpret_cast<const float*>(p.dtab) + ((int64_t)E.kv * p.n_gates + gi) * 8;
+        __syncwarp();
+        if (lane < 8) ws[lane] = __ldg(dt + lane);
+        __syncwarp();
+        eval_dispatch(p, E, __ldg(gd + 2 * gi), __ldg(gd + 2 * gi + 1), S);
+    }
+}
+
+// Materialise PI waveforms of a round's slot groups (reading C2: one event at
+// t = 0 iff p1 != p2) as regions of buffers 0..n_pi-1: one warp per (PI, group).
+__global__ void pi_regions_kernel(const SweepParams p, int32_t n_pi) {
+    const int lane = threadIdx.x & 31;
+    const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    if (gw >= (int64_t)n_pi * p.pin_n_sw) return;
+    const int pi = (int)(gw / p.pin_n_sw);
+    const int64_t i = gw % p.pin_n_sw;
+    const int64_t sw = p.sw_list ? (int64_t)p.sw_list[i] : p.sw_first + i;
+    const int kv = (int)(sw / p.n_pw), pw = (int)(sw % p.n_pw);
+    const int64_t j = (int64_t)pw * 32 + lane;
+    const int64_t pub = (int64_t)kv * p.n_pairs + j;
+    const bool valid = j < p.n_pairs && pub >= p.slot_first && pub < p.slot_end;
+    const uint32_t mask = __ballot_sync(0xffffffffu, valid);
+    const uint32_t w1 = p.p1t[(int64_t)pi * p.n_pw + pw] & mask;
+    const uint32_t w2 = p.p2t[(int64_t)pi * p.n_pw + pw] & mask;
+    const uint32_t tog = w1 ^ w2;
+    const uint32_t n = (tog >> lane) & 1u;
+    const uint32_t off = __popc(tog & ((1u << lane) - 1u));
+    uint8_t* r = p.arena + ((int64_t)pi * p.pin_n_sw + i) * p.region_bytes;
+    reinterpret_cast<uint32_t*>(r)[lane] = n | (off << HDR_OFF_SHIFT) | (((w1 >> lane) & 1u) << HDR_INIT_SHIFT);
+    reinterpret_cast<float*>(r + 128)[lane] = 0.0f;
+}
+
+cudaError_t launch_pi_regions(const SweepParams& p, int32_t n_pi, cudaStream_t st) {
+    const int64_t threads = (int64_t)n_pi * p.pin_n_sw * 32;
+    if (threads == 0) return cudaSuccess;
+    pi_regions_kernel<<<(unsigned)((threads + 255) / 256), 256, 0, st>>>(p, n_pi);
+    return cudaGetLastError();
+}
+
+int sweep_smem_bytes(int warps_per_cta) { return 16 + warps_per_cta * WARP_SMEM_WORDS * 4; }
+int level_smem_bytes(int warps_per_cta) { return 16 + warps_per_cta * LEVEL_SMEM_WORDS * 4; }
+
+cudaError_t sweep_occupancy(int warps_per_cta, int smem, int* blocks_per_sm) {
+    cudaError_t e = cudaFuncSetAttribute(sweep_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+    if (e != cudaSuccess) return e;
+    return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, sweep_kernel, warps_per_cta * 32, smem);
+}
+
+cudaError_t launch_sweep(const SweepParams& p, int grid, int warps_per_cta, cudaStream_t st) {
+    const int smem = sweep_smem_bytes(warps_per_cta);
+    cudaError_t e = cudaFuncSetAttribute(sweep_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+    if (e != cudaSuccess) return e;
+    sweep_kernel<<<grid, warps_per_cta * 32, smem, st>>>(p);
+    return cudaGetLastError();
+}
+
+cudaError_t level_occupancy(int warps_per_cta, int smem, int* blocks_per_sm) {
+    cudaError_t e = cudaFuncSetAttribute(level_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+    if (e != cudaSuccess) return e;
+    return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, level_kernel, warps_per_cta * 32, smem);
+}
+
+cudaError_t launch_level(const SweepParams& p, int level, int grid, int warps_per_cta, cudaStream_t st) {
+    const int smem = level_smem_bytes(warps_per_cta);
+    cudaError_t e = cudaFuncSetAttribute(level_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+    if (e != cudaSuccess) return e;
+    level_kernel<<<grid, warps_per_cta * 32, smem, st>>>(p, level);
+    return cudaGetLastError();
 }
 
 // ---------------------------------------------------------------------------
@@ -123,444 +596,6 @@ cudaError_t launch_delays(const DelayParams& p, cudaStream_t st) {
     const int64_t n = (int64_t)p.n_vdd * p.n_gates * 8;
     if (n == 0) return cudaSuccess;
     delay_kernel<<<(unsigned)((n + 255) / 256), 256, 0, st>>>(p);
-    return cudaGetLastError();
-}
-
-// ---------------------------------------------------------------------------
-// Per-slot merge of the K sorted input event lists of a gate with the inertial
-// filter (reading C3: the pending last output event is cancelled iff
-// it lies strictly after the input event; C4: no reschedule on confirming
-// events; C5: ties in time are taken in ascending pin order).  Branch-free
-// bodies; the element after each head is prefetched from shared memory one
-// step ahead.  Returns the exact output count; the first `cstage` surviving
-// events are left in shared memory rows s_out[i][lane].
-// ---------------------------------------------------------------------------
-__device__ __forceinline__ float lds_f32(uint32_t addr) {
-    float v;
-    asm volatile("ld.shared.f32 %0, [%1];\n" : "=f"(v) : "r"(addr));
-    return v;
-}
-__device__ __forceinline__ void sts_f32(uint32_t addr, float v) {
-    asm volatile("st.shared.f32 [%0], %1;\n" ::"r"(addr), "f"(v) : "memory");
-}
-
-#define AVFS_INF __int_as_float(0x7f800000)
-
-// filter step shared by all merges: one input event at time t whose pin flip
-// gives evaluated output y; d_r / d_f = the pin's rise / fall delays.
-struct OutState {
-    int n;          // surviving output events
-    float tl;       // time of the last surviving event (-inf if it is <= every later input)
-    uint32_t proj;  // projected output value
-};
-
-__device__ __forceinline__ void filter_step(OutState& o, float t, uint32_t y, float d_r, float d_f,
-                                            uint32_t s_out_lane, int cstage) {
-    const bool change = y != o.proj;
-    const bool cancel = change && (o.tl > t);   // pending output lies after t: pulse filtered
-    const bool push = change && !cancel;
-    const float tn = t + (y ? d_r : d_f);
-    // unconditional store to the next free row (clamped): harmless unless pushed
-    sts_f32(s_out_lane + 128u * (uint32_t)min(o.n, cstage), tn);
-    o.n += push ? 1 : (cancel ? -1 : 0);
-    o.tl = push ? tn : (cancel ? -AVFS_INF : o.tl);   // after a cancel the last event is <= t
-    o.proj = y;
-}
-
-// one input (BUF / INV / any 1-input cell)
-__device__ __forceinline__ int merge1(uint32_t s_in, int c, int n, float d_f, float d_r, uint32_t tt,
-                                     uint32_t bits, uint32_t proj, uint32_t s_out_lane, int cstage) {
-    const int e = c + n;
-    const float a0 = lds_f32(s_in + 4u * (uint32_t)c);
-    const float a1 = lds_f32(s_in + 4u * (uint32_t)(c + 1));
-    float h = n > 0 ? a0 : AVFS_INF;
-    float nh = n > 1 ? a1 : AVFS_INF;
-    OutState o{0, -AVFS_INF, proj};
-    while (h < AVFS_INF) {
-        const float t = h;
-        ++c;
-        const float raw = lds_f32(s_in + 4u * (uint32_t)(c + 1));
-        h = nh;
-        nh = (c + 1 < e) ? raw : AVFS_INF;
-        bits ^= 1u;
-        filter_step(o, t, (tt >> bits) & 1u, d_r, d_f, s_out_lane, cstage);
-    }
-    return o.n;
-}
-
-// two inputs, hand-specialised (62 % of gates on the random DAGs)
-__device__ __forceinline__ int merge2(uint32_t s_in, int c0, int n0, int c1, int n1,
-                                     const float (&dl)[8], uint32_t tt, uint32_t bits, uint32_t proj,
-                                     uint32_t s_out_lane, int cstage) {
-    const int e0 = c0 + n0, e1 = c1 + n1;
-    float h0, h1, nh0, nh1;
-    {
-        const float a = lds_f32(s_in + 4u * (uint32_t)c0), b = lds_f32(s_in + 4u * (uint32_t)(c0 + 1));
-        const float x = lds_f32(s_in + 4u * (uint32_t)c1), z = lds_f32(s_in + 4u * (uint32_t)(c1 + 1));
-        h0 = n0 > 0 ? a : AVFS_INF;
-        nh0 = n0 > 1 ? b : AVFS_INF;
-        h1 = n1 > 0 ? x : AVFS_INF;
-        nh1 = n1 > 1 ? z : AVFS_INF;
-    }
-    OutState o{0, -AVFS_INF, proj};
-    for (;;) {
-        const bool p1 = h1 < h0;                 // ties: pin 0 first
-        const float t = p1 ? h1 : h0;
-        if (!(t < AVFS_INF)) break;
-        const int cn = (p1 ? c1 : c0) + 1;
-        const int en = p1 ? e1 : e0;
-        const float raw = lds_f32(s_in + 4u * (uint32_t)(cn + 1));
-        const float hn = p1 ? nh1 : nh0;
-        const float nn = (cn + 1 < en) ? raw : AVFS_INF;
-        if (p1) { h1 = hn; nh1 = nn; c1 = cn; } else { h0 = hn; nh0 = nn; c0 = cn; }
-        bits ^= p1 ? 2u : 1u;
-        filter_step(o, t, (tt >> bits) & 1u, p1 ? dl[3] : dl[1], p1 ? dl[2] : dl[0], s_out_lane, cstage);
-    }
-    return o.n;
-}
-
-// generic K (3 and 4 inputs)
-template <int K>
-__device__ __forceinline__ int merge_k(uint32_t s_in, const int (&cb)[KMAX], const int (&n)[KMAX],
-                                       const float (&dl)[8], uint32_t tt, uint32_t bits,
-                                       uint32_t proj, uint32_t s_out_lane, int cstage) {
-    float h[K], nh[K];
-    int c[K], e[K];
-#pragma unroll
-    for (int q = 0; q < K; ++q) {
-        c[q] = cb[q];
-        e[q] = cb[q] + n[q];
-        const float a0 = lds_f32(s_in + 4u * (uint32_t)c[q]);
-        const float a1 = lds_f32(s_in + 4u * (uint32_t)(c[q] + 1));
-        h[q] = n[q] > 0 ? a0 : AVFS_INF;
-        nh[q] = n[q] > 1 ? a1 : AVFS_INF;
-    }
-    OutState o{0, -AVFS_INF, proj};
-    for (;;) {
-        float t = h[0];
-        int pm = 0;
-#pragma unroll
-        for (int q = 1; q < K; ++q) {
-            const bool lt = h[q] < t;
-            t = lt ? h[q] : t;
-            pm = lt ? q : pm;
-        }
-        if (!(t < AVFS_INF)) break;
-        int cn = c[0], en = e[0];
-        float hn = nh[0], dfp = dl[0], drp = dl[1];
-#pragma unroll
-        for (int q = 1; q < K; ++q)
-            if (pm == q) { cn = c[q]; en = e[q]; hn = nh[q]; dfp = dl[2 * q]; drp = dl[2 * q + 1]; }
-        ++cn;
-        const float raw = lds_f32(s_in + 4u * (uint32_t)(cn + 1));
-        const float nn = (cn + 1 < en) ? raw : AVFS_INF;
-#pragma unroll
-        for (int q = 0; q < K; ++q)
-            if (pm == q) { c[q] = cn; h[q] = hn; nh[q] = nn; }
-        bits ^= 1u << pm;
-        filter_step(o, t, (tt >> bits) & 1u, drp, dfp, s_out_lane, cstage);
-    }
-    return o.n;
-}
-
-// Where one warp's 32 slots live for the gate being evaluated.  All regions
-// of a round live in one arena [buffer][slot group][region] (buffers: PIs,
-// kept signals, scratch), so a region address is one multiply-add.
-struct Env {
-    uint8_t* row;                  // arena + i * region_bytes
-    uint32_t stride;               // bytes between buffers = n_sw * region_bytes (< 4 GiB, checked on host)
-    int64_t i;                     // index of the slot group in the round (overflow flag)
-    int kv, lane;
-    uint32_t s_in_a;               // per-warp input staging (shared window address)
-    uint32_t s_out_a;              // per-warp output rows + 4*lane
-    uint32_t bar;                  // per-warp mbarrier for the TMA staging
-    uint32_t phase;                // its current parity
-    unsigned long long* act_kv;    // &act[0][kv]
-};
-
-__device__ __forceinline__ uint8_t* region(uint32_t buf, const Env& E) {
-    return E.row + (uint64_t)buf * (uint64_t)E.stride;
-}
-
-// One gate for one 32-slot group: input headers,
-// compact staging, merge/filter, output compaction, reductions.
-template <int K>
-__device__ __forceinline__ void eval_gate(const SweepParams& p, Env& E, const uint4 ins, const uint4 hd,
-                                          const float (&dl)[8]) {
-    const int lane = E.lane;
-    const uint32_t out_loc = hd.x, sig = hd.y;
-    const uint32_t tt = hd.z & 0xffffu;
-    const uint32_t in_loc[KMAX] = {ins.x, ins.y, ins.z, ins.w};
-    // all input header loads first (one coalesced 128-B row per input)
-    const uint8_t* rg[KMAX];
-    uint32_t hw[KMAX];
-#pragma unroll
-    for (int q = 0; q < K; ++q) {
-        rg[q] = region(in_loc[q], E);
-        hw[q] = __ldcg(reinterpret_cast<const uint32_t*>(rg[q]) + lane);
-    }
-    int n[KMAX], cb[KMAX];
-    uint32_t bits = 0, pois = 0, prevp = 0;
-    int sum = 0;
-#pragma unroll
-    for (int q = 0; q < KMAX; ++q) {
-        n[q] = 0;
-        cb[q] = 0;
-        if (q < K) {
-            const uint32_t h = hw[q];
-            n[q] = (int)(h & HDR_N);
-            cb[q] = (int)((h >> HDR_OFF_SHIFT) & HDR_OFF);
-            bits |= ((h >> HDR_INIT_SHIFT) & 1u) << q;
-            pois |= h;
-            prevp |= h;
-            sum += n[q];
-        }
-    }
-    const uint32_t y0 = (tt >> bits) & 1u;
-    uint8_t* ro = region(out_loc, E);
-    uint32_t* ro_hdr = reinterpret_cast<uint32_t*>(ro);
-    const bool first_pass = (p.prev_W == 0);
-    const bool any_prev = first_pass || __any_sync(0xffffffffu, (prevp & HDR_PREV) != 0);
-    if (__any_sync(0xffffffffu, (pois & HDR_POISON) != 0)) {   // upstream overflow: nothing valid here
-        __stcg(ro_hdr + lane, HDR_POISON | HDR_PREV | (y0 << HDR_INIT_SHIFT));
-        return;
-    }
-    if (!__any_sync(0xffffffffu, sum != 0)) {                   // no input event in any slot: constant output
-        __stcg(ro_hdr + lane, (y0 << HDR_INIT_SHIFT) | (any_prev ? HDR_PREV : 0u));
-        return;
-    }
-    // stage each input's compact event list into shared memory with one TMA
-    // bulk copy per input (extent = lane 31's offset + count), one mbarrier
-    int stage_base = 0;
-    {
-        int base = 0;
-        int ext[KMAX];
-#pragma unroll
-        for (int q = 0; q < K; ++q) {
-            ext[q] = __shfl_sync(0xffffffffu, cb[q] + n[q], 31);
-            ext[q] = (ext[q] + 3) & ~3;
-            cb[q] += base;
-            base += ext[q];
-        }
-        if (base > p.stage_words) {                    // inputs exceed this capacity's staging: rerun
-            __stcg(ro_hdr + lane, HDR_POISON | HDR_PREV | (y0 << HDR_INIT_SHIFT));
-            if (lane == 0) p.ovf[p.i_base + E.i] = 1;
-            return;
-        }
-        stage_base = base;
-        if (base > 0) {
-            if (lane == 0) {
-                fence_proxy_async_smem();              // earlier generic reads of the staging area
-                mbar_expect_tx(E.bar, 4u * (uint32_t)base);
-                uint32_t dst = E.s_in_a;
-#pragma unroll
-                for (int q = 0; q < K; ++q) {
-                    if (ext[q] > 0) tma_bulk_g2s(dst, rg[q] + 128, 4u * (uint32_t)ext[q], E.bar);
-                    dst += 4u * (uint32_t)ext[q];
-                }
-            }
-            mbar_wait(E.bar, E.phase);
-            E.phase ^= 1u;
-        }
-    }
-    int n_out;
-    if (K == 1) {
-        n_out = merge1(E.s_in_a, cb[0], n[0], dl[0], dl[1], tt, bits, y0, E.s_out_a, p.cstage);
-    } else if (K == 2) {
-        n_out = merge2(E.s_in_a, cb[0], n[0], cb[1], n[1], dl, tt, bits, y0, E.s_out_a, p.cstage);
-    } else {
-        n_out = merge_k<K>(E.s_in_a, cb, n, dl, tt, bits, y0, E.s_out_a, p.cstage);
-    }
-    // output: scan, overflow ballot, compact stores row by row (warp-uniform loop)
-    const uint32_t incl = warp_incl_scan((uint32_t)n_out, lane);
-    const uint32_t total = __shfl_sync(0xffffffffu, incl, 31);
-    const uint32_t excl = incl - (uint32_t)n_out;
-    const bool ovf = __any_sync(0xffffffffu, n_out > p.cstage) || total > (uint32_t)p.W;
-    bool prev = true;
-    if (!first_pass)
-        prev = any_prev || stage_base > p.prev_stage_words || __any_sync(0xffffffffu, n_out > p.prev_cstage) ||
-               total > (uint32_t)p.prev_W;
-    if (!ovf) {
-        const int rows = (int)__reduce_max_sync(0xffffffffu, (uint32_t)n_out);
-        float* dst = reinterpret_cast<float*>(ro + 128) + excl;
-        for (int r = 0; r < rows; ++r) {
-            const float v = lds_f32(E.s_out_a + 128u * (uint32_t)r);
-            if (r < n_out) __stcg(dst + r, v);
-        }
-    } else if (lane == 0) {
-        p.ovf[p.i_base + E.i] = 1;
-    }
-    __stcg(ro_hdr + lane, (uint32_t)min(n_out, (int)HDR_N) | ((excl & HDR_OFF) << HDR_OFF_SHIFT) |
-                              (y0 << HDR_INIT_SHIFT) | (ovf ? HDR_POISON : 0u) | (prev ? HDR_PREV : 0u));
-    // activity (reading C15) and latest PO arrival (P:L207): counted once per
-    // slot across overflow rounds (where prev && !ovf)
-    if (!ovf && prev) {
-        if (lane == 0 && total) atomicAdd(E.act_kv + (size_t)sig * (uint32_t)p.n_vdd, (unsigned long long)total);
-        if (hd.z & (1u << 24)) {
-            const float last = n_out ? lds_f32(E.s_out_a + 128u * (uint32_t)(n_out - 1)) : 0.0f;
-            const uint32_t m = __reduce_max_sync(0xffffffffu, __float_as_uint(last));
-            if (lane == 0 && m) atomicMax(p.latest + E.kv, m);
-        }
-    }
-    __syncwarp();
-}
-
-__device__ __forceinline__ void eval_dispatch(const SweepParams& p, Env& E, const uint4 ins, const uint4 hd,
-                                              const float4 d0, const float4 d1) {
-    const float dl[8] = {d0.x, d0.y, d0.z, d0.w, d1.x, d1.y, d1.z, d1.w};
-    switch ((hd.z >> 16) & 0xffu) {
-        case 1: eval_gate<1>(p, E, ins, hd, dl); break;
-        case 2: eval_gate<2>(p, E, ins, hd, dl); break;
-        case 3: eval_gate<3>(p, E, ins, hd, dl); break;
-        default: eval_gate<4>(p, E, ins, hd, dl); break;
-    }
-}
-
-__device__ __forceinline__ void slot_group(const SweepParams& p, int64_t i, int lane, Env& E) {
-    const int64_t sw = p.sw_list ? (int64_t)p.sw_list[i] : p.sw_first + i;
-    E.kv = (int)(sw / p.n_pw);
-    E.i = i;
-    E.lane = lane;
-    E.act_kv = p.act + E.kv;
-    E.row = p.arena + (p.i_base + i) * p.region_bytes;
-}
-
-__device__ __forceinline__ void warp_smem(const SweepParams& p, int warp, int lane, Env& E) {
-    extern __shared__ __align__(16) float smem[];
-    float* s_in = smem + 4 + (size_t)warp * (size_t)(p.stage_words + 16 + 32 * (p.cstage + 1));
-    E.s_in_a = static_cast<uint32_t>(__cvta_generic_to_shared(s_in));
-    E.s_out_a = E.s_in_a + 4u * (uint32_t)(p.stage_words + 16) + 4u * (uint32_t)lane;
-    E.bar = E.s_in_a + 4u * (uint32_t)(p.stage_words + 14);   // 8-B aligned, past any over-read
-    E.phase = 0;
-    if (lane == 0) mbar_init(E.bar);
-    __syncwarp();
-}
-
-// Persistent level sweep (pass 0): one CTA owns one 32-slot group at a time
-// and walks all levels with a CTA barrier between levels.
-__global__ void __launch_bounds__(1024, 1) sweep_kernel(const SweepParams p) {
-    extern __shared__ __align__(16) float smem[];
-    int* ctr = reinterpret_cast<int*>(smem);             // two level counters (16-B header)
-    const int lane = threadIdx.x & 31;
-    const int warp = threadIdx.x >> 5;
-    const int nw = blockDim.x >> 5;
-    Env E;
-    warp_smem(p, warp, lane, E);
-    E.stride = (uint32_t)(p.pin_n_sw * p.region_bytes);
-    const uint4* gd = reinterpret_cast<const uint4*>(p.gates);
-    for (int64_t i = blockIdx.x; i < p.n_sw; i += gridDim.x) {
-        slot_group(p, i, lane, E);
-        const float4* dt = p.dtab + (int64_t)E.kv * p.n_gates * 2;
-        if (threadIdx.x == 0) ctr[0] = __ldg(p.level_ptr);
-        __syncthreads();
-        for (int L = 0; L < p.depth; ++L) {
-            const int g_end = __ldg(p.level_ptr + L + 1);
-            if (p.dyn_grab) {
-                // warps take gates of the level from a shared counter (load balance)
-                int* c = ctr + (L & 1);
-                for (;;) {
-                    int gi = 0;
-                    if (lane == 0) gi = atomicAdd(c, 1);
-                    gi = __shfl_sync(0xffffffffu, gi, 0);
-                    if (gi >= g_end) break;
-                    eval_dispatch(p, E, __ldg(gd + 2 * gi), __ldg(gd + 2 * gi + 1), __ldg(dt + 2 * gi),
-                                  __ldg(dt + 2 * gi + 1));
-                }
-                if (threadIdx.x == 0 && L + 1 < p.depth) ctr[(L + 1) & 1] = g_end;
-            } else {
-                for (int gi = __ldg(p.level_ptr + L) + warp; gi < g_end; gi += nw)
-                    eval_dispatch(p, E, __ldg(gd + 2 * gi), __ldg(gd + 2 * gi + 1), __ldg(dt + 2 * gi),
-                                  __ldg(dt + 2 * gi + 1));
-            }
-            fence_proxy_async_global();   // this level's stores -> next levels' TMA reads
-            __syncthreads();
-        }
-    }
-}
-
-// Level-parallel variant for overflow reruns (few slot groups): one launch per
-// level, warps take (gate, slot group) items of the level grid-wide.
-__global__ void __launch_bounds__(512, 2) level_kernel(const SweepParams p, int L) {
-    const int lane = threadIdx.x & 31;
-    const int warp = threadIdx.x >> 5;
-    Env E;
-    warp_smem(p, warp, lane, E);
-    E.stride = (uint32_t)(p.pin_n_sw * p.region_bytes);
-    const uint4* gd = reinterpret_cast<const uint4*>(p.gates);
-    const int g0 = __ldg(p.level_ptr + L);
-    const int64_t items = (int64_t)(__ldg(p.level_ptr + L + 1) - g0) * p.n_sw;
-    const int64_t gw = (int64_t)blockIdx.x * (blockDim.x >> 5) + warp;
-    const int64_t nwarps = (int64_t)gridDim.x * (blockDim.x >> 5);
-    for (int64_t it = gw; it < items; it += nwarps) {
-        const int gi = g0 + (int)(it / p.n_sw);
-        const int64_t i = it % p.n_sw;
-        slot_group(p, i, lane, E);
-        const float4* dt = p.dtab + (int64_t)E.kv * p.n_gates * 2;
-        eval_dispatch(p, E, __ldg(gd + 2 * gi), __ldg(gd + 2 * gi + 1), __ldg(dt + 2 * gi), __ldg(dt + 2 * gi + 1));
-    }
-    fence_proxy_async_global();   // stores -> next launch's TMA reads
-}
-
-// Materialise PI waveforms of a round's slot groups (reading C2: one event at
-// t = 0 iff p1 != p2) as regions of buffers 0..n_pi-1: one warp per (PI, group).
-__global__ void pi_regions_kernel(const SweepParams p, int32_t n_pi) {
-    const int lane = threadIdx.x & 31;
-    const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-    if (gw >= (int64_t)n_pi * p.pin_n_sw) return;
-    const int pi = (int)(gw / p.pin_n_sw);
-    const int64_t i = gw % p.pin_n_sw;
-    const int64_t sw = p.sw_list ? (int64_t)p.sw_list[i] : p.sw_first + i;
-    const int kv = (int)(sw / p.n_pw), pw = (int)(sw % p.n_pw);
-    const int64_t j = (int64_t)pw * 32 + lane;
-    const int64_t pub = (int64_t)kv * p.n_pairs + j;
-    const bool valid = j < p.n_pairs && pub >= p.slot_first && pub < p.slot_end;
-    const uint32_t mask = __ballot_sync(0xffffffffu, valid);
-    const uint32_t w1 = p.p1t[(int64_t)pi * p.n_pw + pw] & mask;
-    const uint32_t w2 = p.p2t[(int64_t)pi * p.n_pw + pw] & mask;
-    const uint32_t tog = w1 ^ w2;
-    const uint32_t n = (tog >> lane) & 1u;
-    const uint32_t off = __popc(tog & ((1u << lane) - 1u));
-    uint8_t* r = p.arena + ((int64_t)pi * p.pin_n_sw + i) * p.region_bytes;
-    reinterpret_cast<uint32_t*>(r)[lane] = n | (off << HDR_OFF_SHIFT) | (((w1 >> lane) & 1u) << HDR_INIT_SHIFT);
-    reinterpret_cast<float*>(r + 128)[lane] = 0.0f;
-}
-
-cudaError_t launch_pi_regions(const SweepParams& p, int32_t n_pi, cudaStream_t st) {
-    const int64_t threads = (int64_t)n_pi * p.pin_n_sw * 32;
-    if (threads == 0) return cudaSuccess;
-    pi_regions_kernel<<<(unsigned)((threads + 255) / 256), 256, 0, st>>>(p, n_pi);
-    return cudaGetLastError();
-}
-
-int sweep_smem_bytes(int warps_per_cta, int stage_words, int cstage) {
-    return 16 + warps_per_cta * (stage_words + 16 + 32 * (cstage + 1)) * 4;
-}
-
-cudaError_t sweep_occupancy(int warps_per_cta, int smem, int* blocks_per_sm) {
-    cudaError_t e = cudaFuncSetAttribute(sweep_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
-    if (e != cudaSuccess) return e;
-    return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, sweep_kernel, warps_per_cta * 32, smem);
-}
-
-cudaError_t launch_sweep(const SweepParams& p, int grid, int warps_per_cta, cudaStream_t st) {
-    const int smem = sweep_smem_bytes(warps_per_cta, p.stage_words, p.cstage);
-    cudaError_t e = cudaFuncSetAttribute(sweep_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
-    if (e != cudaSuccess) return e;
-    sweep_kernel<<<grid, warps_per_cta * 32, smem, st>>>(p);
-    return cudaGetLastError();
-}
-
-cudaError_t level_occupancy(int warps_per_cta, int smem, int* blocks_per_sm) {
-    cudaError_t e = cudaFuncSetAttribute(level_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
-    if (e != cudaSuccess) return e;
-    return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, level_kernel, warps_per_cta * 32, smem);
-}
-
-cudaError_t launch_level(const SweepParams& p, int level, int grid, int warps_per_cta, cudaStream_t st) {
-    const int smem = sweep_smem_bytes(warps_per_cta, p.stage_words, p.cstage);
-    cudaError_t e = cudaFuncSetAttribute(level_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
-    if (e != cudaSuccess) return e;
-    level_kernel<<<grid, warps_per_cta * 32, smem, st>>>(p, level);
     return cudaGetLastError();
 }
 
