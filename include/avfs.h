@@ -155,17 +155,25 @@ avfs_status avfs_set_stimuli(avfs_ctx *ctx, int64_t n_pairs, const uint32_t *p1,
 avfs_status avfs_set_slot_range(avfs_ctx *ctx, int64_t first_slot, int64_t n_slots);
 
 typedef struct {
-    int32_t capacity;          /* C: transitions per slot on average within a
-                                  32-slot warp region (region holds 32*C
-                                  times), and 2*C per single slot.  >= 1.   */
+    int32_t capacity;          /* C: in-place event capacity of a 32-slot
+                                  region, 32*C binary32 times.  A gate-warp
+                                  whose inputs carry more than 32*C events
+                                  stores its outputs in the round's spill
+                                  heap instead (address in the region).  >= 1 */
     double quantum_ps;         /* 0: F mode; q > 0: Q mode, d' <- q rint(d'/q)
                                   (reading C12)                             */
     int32_t n_probe;           /* internal signals kept for readback        */
     const int32_t *probe_sig;  /* [n_probe], copied                          */
     int32_t keep_all;          /* 1: every gate output is kept (parity runs) */
-    int32_t max_rerun_rounds;  /* overflow reruns at 4x capacity; default 3  */
+    int32_t max_rerun_rounds;  /* overflow reruns; default 3.  Overflow = spill
+                                  heap exhausted (rerun with a heap twice the
+                                  requested size) or, with spill disabled,
+                                  more than 32*C events (rerun at 4C)       */
     int32_t warps_per_cta;     /* 0: default (8)                              */
     int32_t profile;           /* 1: time the sweep kernel with CUDA events  */
+    int64_t spill_bytes;       /* pass-0 spill heap: 0 = auto (arena/4, at
+                                  least 256 MiB, within free memory); > 0 =
+                                  this many bytes; < 0 = no spill heap     */
 } avfs_options;
 avfs_status avfs_set_options(avfs_ctx *ctx, const avfs_options *opt);
 avfs_status avfs_default_options(avfs_options *opt);
@@ -251,6 +259,8 @@ typedef struct {
     int32_t grid, warps_per_cta, n_scratch_buffers, n_pinned;
     double sim_ms;               /* host wall time of the last simulate      */
     double sweep_ms;             /* CUDA-event time of pass-0 sweep (profile=1) */
+    int64_t spill_bytes;         /* spill-heap bytes used by the kept rounds  */
+    int64_t spill_heap_bytes;    /* spill-heap bytes allocated (all rounds)   */
 } avfs_stats;
 avfs_status avfs_get_stats(avfs_ctx *ctx, avfs_stats *st);
 

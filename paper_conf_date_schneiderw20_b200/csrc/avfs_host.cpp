@@ -62,6 +62,9 @@ struct Round {
     int32_t capacity = 0, W = 0;
     int64_t region_bytes = 0;
     int32_t grid = 0;
+    int64_t spill_want = 0;          // requested heap words (0: no spill heap)
+    int64_t spill_words = 0;         // heap words allocated for this round
+    int64_t spill_req = 0;           // words requested by the round's gate-warps (incl. failed)
 };
 
 }  // namespace
@@ -123,8 +126,10 @@ struct avfs_ctx {
     // device state
     bool dev_net_valid = false, dev_vdd_valid = false;
     DevBuf d_gates, d_ddesc, d_dtab, d_coef, d_cload, d_island, d_energy, c_loc, c_tclk, c_slot, c_out, d_level_ptr, d_vdd, d_p1, d_p2, d_p1t, d_p2t, d_act, d_latest, d_ovf,
-        d_err, d_list[2], d_count, d_swround, d_swindex, g_loc, g_init, g_count, g_times, g_bad;
+        d_err, d_list[2], d_prev[2], d_pois[2], d_spill_top, d_count, d_swround, d_swindex, g_loc, g_init, g_count,
+        g_times, g_bad;
     std::vector<DevBuf> arena;        // per round: [buffer][slot group][region]
+    std::vector<DevBuf> spill;        // per round: spill heap (kept: readback may point into it)
     int32_t* h_pinned = nullptr;      // small pinned host buffer (count, err)
     cudaEvent_t ev0 = nullptr, ev1 = nullptr;
 
@@ -804,8 +809,8 @@ avfs_status avfs_sync(avfs_ctx* ctx) {
     return AVFS_OK;
 }
 
-static avfs_status run_round(avfs_ctx* ctx, Round& R, int round_idx, const int32_t* d_sw_list, int32_t prev_W,
-                             bool timed) {
+static avfs_status run_round(avfs_ctx* ctx, Round& R, int round_idx, const int32_t* d_sw_list,
+                             const int32_t* d_prev_idx, bool timed) {
     const bool persistent = (round_idx == 0);
     // launch bounds: sweep_kernel up to 1024 threads, level_kernel 512 threads
     const int wmax = persistent ? AVFS_SWEEP_THREADS / 32 : 16;
@@ -826,6 +831,27 @@ static avfs_status run_round(avfs_ctx* ctx, Round& R, int round_idx, const int32
     CK(ctx->arena[round_idx].ensure((size_t)std::max<int64_t>(n_buf, 1) * R.n_sw * R.region_bytes));
     CK(ctx->d_ovf.ensure(std::max<int64_t>(R.n_sw, 1) * sizeof(int32_t)));
     CK(cudaMemsetAsync(ctx->d_ovf.p, 0, R.n_sw * sizeof(int32_t), ctx->stream));
+    // spill heap: the requested size, within free device memory (keep 1 GiB)
+    if ((int)ctx->spill.size() <= round_idx) ctx->spill.resize(round_idx + 1);
+    R.spill_words = 0;
+    if (R.spill_want > 0) {
+        size_t fr = 0, tot = 0;
+        CK(cudaMemGetInfo(&fr, &tot));
+        const size_t have = ctx->spill[round_idx].n;
+        const size_t avail = fr + have > (1ull << 30) ? fr + have - (1ull << 30) : 0;
+        size_t bytes = std::min<size_t>((size_t)R.spill_want * 4, avail) & ~(size_t)15;
+        while (bytes >= 16 && ctx->spill[round_idx].ensure(bytes) != cudaSuccess) {
+            cudaGetLastError();
+            bytes = (bytes / 2) & ~(size_t)15;
+        }
+        if (bytes >= 16) R.spill_words = (int64_t)(bytes / 4);
+    }
+    CK(ctx->d_spill_top.ensure(8 * 8));
+    CK(cudaMemsetAsync(ctx->d_spill_top.as<unsigned long long>() + round_idx, 0, 8, ctx->stream));
+    const size_t pois_words = ((size_t)std::max<int64_t>(R.n_sw, 1) * std::max(ctx->n_gates, 1) + 31) / 32;
+    DevBuf& pois = ctx->d_pois[round_idx & 1];
+    CK(pois.ensure(pois_words * 4));
+    CK(cudaMemsetAsync(pois.p, 0, pois_words * 4, ctx->stream));
     SweepParams p{};
     p.gates = ctx->d_gates.as<GateDesc>();
     p.level_ptr = ctx->d_level_ptr.as<int32_t>();
@@ -847,7 +873,13 @@ static avfs_status run_round(avfs_ctx* ctx, Round& R, int round_idx, const int32
     p.arena = ctx->arena[round_idx].as<uint8_t>();
     p.region_bytes = R.region_bytes;
     p.W = R.W;
-    p.prev_W = prev_W;
+    p.n_pi = ctx->n_pi;
+    p.spill = ctx->spill[round_idx].as<float>();
+    p.spill_top = ctx->d_spill_top.as<unsigned long long>() + round_idx;
+    p.spill_words = (uint64_t)R.spill_words;
+    p.pois = pois.as<uint32_t>();
+    p.pois_prev = round_idx == 0 ? nullptr : ctx->d_pois[(round_idx - 1) & 1].as<uint32_t>();
+    p.prev_idx = d_prev_idx;
     p.act = ctx->d_act.as<unsigned long long>();
     p.latest = ctx->d_latest.as<unsigned int>();
     p.ovf = ctx->d_ovf.as<int32_t>();
@@ -940,21 +972,37 @@ avfs_status avfs_simulate(avfs_ctx* ctx, void* cuda_stream) {
     R0.capacity = ctx->opt.capacity;
     R0.W = 32 * R0.capacity;
     R0.region_bytes = 128 + 4 * (int64_t)R0.W;
-    st = run_round(ctx, R0, 0, nullptr, 0, ctx->opt.profile != 0);
+    {
+        const int64_t arena_words = ((int64_t)ctx->n_pi + ctx->n_pinned + ctx->n_scratch) * R0.n_sw * R0.region_bytes / 4;
+        R0.spill_want = ctx->opt.spill_bytes > 0 ? ctx->opt.spill_bytes / 4
+                      : ctx->opt.spill_bytes < 0 ? 0 : std::max<int64_t>(arena_words / 4, (256ll << 20) / 4);
+    }
+    st = run_round(ctx, R0, 0, nullptr, nullptr, ctx->opt.profile != 0);
     if (st != AVFS_OK) return st;
     ctx->rounds.push_back(R0);
     int cur = 0;
     for (int r = 0;; ++r) {
-        const Round& prev = ctx->rounds.back();
+        Round& prev = ctx->rounds.back();
         CK(ctx->d_list[cur].ensure(std::max<int64_t>(prev.n_sw, 1) * sizeof(int32_t)));
+        CK(ctx->d_prev[cur].ensure(std::max<int64_t>(prev.n_sw, 1) * sizeof(int32_t)));
         CK(cudaMemsetAsync(ctx->d_count.p, 0, 16, ctx->stream));
         CK(launch_compact_overflow(ctx->d_ovf.as<int32_t>(), prev.n_sw,
                                    r == 0 ? nullptr : ctx->d_list[cur ^ 1].as<int32_t>(), prev.sw_first,
-                                   ctx->d_list[cur].as<int32_t>(), ctx->d_count.as<int32_t>(), ctx->stream));
+                                   ctx->d_list[cur].as<int32_t>(), ctx->d_prev[cur].as<int32_t>(),
+                                   ctx->d_count.as<int32_t>(), ctx->stream));
         ctx->stats.launches++;
         CK(cudaMemcpyAsync(ctx->h_pinned, ctx->d_count.p, 4, cudaMemcpyDeviceToHost, ctx->stream));
         CK(cudaMemcpyAsync(ctx->h_pinned + 1, ctx->d_err.p, 4, cudaMemcpyDeviceToHost, ctx->stream));
+        CK(cudaMemcpyAsync(ctx->h_pinned + 2, ctx->d_spill_top.as<unsigned long long>() + r, 8,
+                           cudaMemcpyDeviceToHost, ctx->stream));
         CK(cudaStreamSynchronize(ctx->stream));
+        {
+            unsigned long long req = 0;
+            std::memcpy(&req, ctx->h_pinned + 2, 8);
+            prev.spill_req = (int64_t)req;
+            ctx->stats.spill_bytes += 4 * std::min<int64_t>(prev.spill_req, prev.spill_words);
+            ctx->stats.spill_heap_bytes += 4 * prev.spill_words;
+        }
         if (ctx->h_pinned[1] & 1)
             return fail(ctx, AVFS_ERR_DELAY_NONPOS, "a delay d' = d_nom (1 + f(P)) evaluated to <= 0");
         const int32_t n_ovf = ctx->h_pinned[0];
@@ -966,12 +1014,20 @@ avfs_status avfs_simulate(avfs_ctx* ctx, void* cuda_stream) {
         Rn.n_sw = n_ovf;
         Rn.sws.resize(n_ovf);
         CK(cudaMemcpy(Rn.sws.data(), ctx->d_list[cur].p, n_ovf * sizeof(int32_t), cudaMemcpyDeviceToHost));
-        Rn.capacity = std::min(prev.capacity * 4, 1024);
+        // with a spill heap the overflow was heap exhaustion: same capacity, a
+        // heap 4x what was asked for (poisoned cones asked for nothing), at
+        // least 64 MiB; without one, 4x capacity
+        if (prev.spill_want > 0) {
+            Rn.capacity = prev.capacity;
+            Rn.spill_want = std::max<int64_t>(4 * std::max<int64_t>(prev.spill_req, prev.spill_words), (64ll << 20) / 4);
+        } else {
+            Rn.capacity = std::min(prev.capacity * 4, 1024);
+        }
         Rn.W = 32 * Rn.capacity;
         Rn.region_bytes = 128 + 4 * (int64_t)Rn.W;
         ctx->stats.overflow_slot_warps += n_ovf;
         ctx->stats.rerun_rounds++;
-        st = run_round(ctx, Rn, r + 1, ctx->d_list[cur].as<int32_t>(), prev.W, false);
+        st = run_round(ctx, Rn, r + 1, ctx->d_list[cur].as<int32_t>(), ctx->d_prev[cur].as<int32_t>(), false);
         if (st != AVFS_OK) return st;
         ctx->rounds.push_back(std::move(Rn));
         cur ^= 1;

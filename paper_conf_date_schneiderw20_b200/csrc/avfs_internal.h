@@ -31,7 +31,8 @@ constexpr uint32_t HDR_OFF = 0xFFFFu;        //   region (exclusive prefix of th
 constexpr int HDR_INIT_SHIFT = 28;
 constexpr uint32_t HDR_INIT = 1u << 28;      // value before t = 0
 constexpr uint32_t HDR_POISON = 1u << 29;    // events not stored here or upstream
-constexpr uint32_t HDR_PREV = 1u << 30;      // would have been poisoned at the previous round's capacity
+constexpr uint32_t HDR_SPILL = 1u << 30;     // the region's events live in the round's spill heap; the
+                                             //   region's first event word pair holds their address
 
 // Gate descriptor, 32 B, read warp-uniformly (P:L154 step 1).
 struct alignas(16) GateDesc {
@@ -91,7 +92,17 @@ struct SweepParams {
     uint8_t* arena;
     int64_t region_bytes;
     int32_t W;                              // event capacity per region (32*C)
-    int32_t prev_W;                         // previous round's W (0: first pass)
+    int32_t n_pi;                           // gate index = output signal - n_pi
+    // spill heap of the round: regions whose inputs carry more than W events
+    // store their events here (bump allocation in words, 16-B granules)
+    float* spill;
+    unsigned long long* spill_top;          // words handed out (counts failed requests too)
+    uint64_t spill_words;                   // heap capacity
+    // poison bitmaps [group index in round][n_gates] bits: this round's, and
+    // the previous round's (null on pass 0) for exact activity accounting
+    uint32_t* pois;
+    const uint32_t* pois_prev;
+    const int32_t* prev_idx;                // [n_sw] group's index in the previous round
     // outputs
     unsigned long long* act;                // [n_signals][n_vdd]
     unsigned int* latest;                   // [n_vdd] float bits (non-negative)
@@ -113,8 +124,8 @@ cudaError_t launch_pi_activity(const uint32_t* p1t, const uint32_t* p2t, int32_t
                                int64_t n_pairs, int32_t n_vdd, int64_t slot_first, int64_t slot_end,
                                unsigned long long* act, cudaStream_t st);
 cudaError_t launch_compact_overflow(const int32_t* ovf, int64_t n_sw, const int32_t* sw_list,
-                                    int64_t sw_first, int32_t* out_list, int32_t* out_count,
-                                    cudaStream_t st);
+                                    int64_t sw_first, int32_t* out_list, int32_t* out_prev,
+                                    int32_t* out_count, cudaStream_t st);
 
 struct GatherRound {       // one simulated round for readback
     const uint8_t* pinned;

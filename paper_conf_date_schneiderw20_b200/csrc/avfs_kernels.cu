@@ -97,6 +97,15 @@ __device__ __forceinline__ uint8_t* region(uint32_t buf, const Env& E) {
     return E.row + (uint64_t)buf * (uint64_t)E.stride;
 }
 
+// First event word of a region: in place, or in the spill heap (HDR_SPILL in
+// any of the region's header words; the address is the region's first
+// event word pair).
+__device__ __forceinline__ const uint8_t* ev_base(const uint8_t* reg, uint32_t hw) {
+    const uint8_t* b = reg + 128;
+    if (hw & HDR_SPILL) b = reinterpret_cast<const uint8_t*>(__ldcg(reinterpret_cast<const unsigned long long*>(b)));
+    return b;
+}
+
 __device__ __forceinline__ uint32_t smem_u32(const void* p) {
     return static_cast<uint32_t>(__cvta_generic_to_shared(p));
 }
@@ -125,6 +134,7 @@ struct Staged {
     uint32_t hdr_s;       // shared address of header row 0 (row q at + 128 q)
     uint32_t ev_s[1];     // shared address of the staged events (input q at + 4 EV_STAGE q / K')
     uint32_t dly_s;       // shared address of the gate's 8 delays [pin][pol]
+    uint32_t grp_s;       // shared address of the slot group's index in the round (u32; read when poisoning)
 };
 __device__ __forceinline__ float4 lds_f32x4(uint32_t a) {
     float4 v;
@@ -245,7 +255,7 @@ __device__ __forceinline__ uint32_t merge_slot(const MergeIn& M, float* out, uin
     return (uint32_t)(op - out);
 }
 
-template <int K>
+template <int K, bool RERUN>
 __device__ __forceinline__ void eval_gate(const SweepParams& p, const Env& E, const uint4 ins, const uint4 hd,
                                           const Staged& S) {
     const int lane = E.lane;
@@ -270,31 +280,51 @@ __device__ __forceinline__ void eval_gate(const SweepParams& p, const Env& E, co
     const uint32_t y0 = (tt >> bits) & 1u;
     uint8_t* ro = region(out_loc, E);
     uint32_t* ro_hdr = reinterpret_cast<uint32_t*>(ro);
-    const bool first_pass = (p.prev_W == 0);
-    // one warp reduction: upstream poison / previous-capacity flags, any input event
-    const uint32_t R = __reduce_or_sync(FULL, (orh & (HDR_POISON | HDR_PREV)) | (m != 0 ? 1u : 0u));
+    auto poison = [&](bool own) {
+        __stcg(ro_hdr + lane, HDR_POISON | (y0 << HDR_INIT_SHIFT));
+        if (lane == 0) {            // poison bitmap bit of this (slot group, gate) in this round
+            const uint32_t gi = lds_u32(S.grp_s);
+            const uint64_t gbit = (uint64_t)gi * (uint32_t)p.n_gates + (sig - (uint32_t)p.n_pi);
+            atomicOr(p.pois + (gbit >> 5), 1u << (gbit & 31u));
+            if (own) p.ovf[gi] = 1;
+        }
+    };
+    // one warp reduction: upstream poison, any input event
+    const uint32_t R = __reduce_or_sync(FULL, (orh & HDR_POISON) | (m != 0 ? 1u : 0u));
     if (R & HDR_POISON) {                               // upstream overflow: nothing valid here
-        __stcg(ro_hdr + lane, HDR_POISON | HDR_PREV | (y0 << HDR_INIT_SHIFT));
+        poison(false);
         return;
     }
-    const bool any_prev = first_pass || (R & HDR_PREV);
     if (!(R & 1u)) {                                    // no input event in any slot: constant output
-        __stcg(ro_hdr + lane, (y0 << HDR_INIT_SHIFT) | (any_prev ? HDR_PREV : 0u));
+        __stcg(ro_hdr + lane, y0 << HDR_INIT_SHIFT);
         return;
     }
     const uint32_t incl = warp_incl_scan((uint32_t)m, lane);
     const uint32_t total_in = __shfl_sync(FULL, incl, 31);
     const uint32_t base = incl - (uint32_t)m;
     const uint32_t maxm = __reduce_max_sync(FULL, (uint32_t)m);
-    // capacity (reading C17): the inputs' events bound the outputs
-    const bool ovf = total_in > (uint32_t)p.W || maxm > HDR_N;
-    const bool prev = any_prev || total_in > (uint32_t)p.prev_W;
-    if (ovf) {
-        __stcg(ro_hdr + lane, HDR_POISON | (prev ? HDR_PREV : 0u) | (y0 << HDR_INIT_SHIFT));
-        if (lane == 0) p.ovf[p.i_base + E.i] = 1;
+    // the inputs' events bound the outputs (reading C17): header fields must
+    // hold them; more than W go to the spill heap, and if the heap is
+    // exhausted the slot group is rerun
+    if (total_in > HDR_OFF || maxm > HDR_N) {
+        poison(true);
         return;
     }
     float* out = reinterpret_cast<float*>(ro + 128) + base;
+    uint32_t hdr_part = (base << HDR_OFF_SHIFT) | (y0 << HDR_INIT_SHIFT);
+    if (total_in > (uint32_t)p.W) {
+        const uint32_t need = (total_in + 3u) & ~3u;
+        unsigned long long wb = 0;
+        if (lane == 0) wb = atomicAdd(p.spill_top, (unsigned long long)need);
+        wb = __shfl_sync(FULL, wb, 0);
+        if (wb + need > p.spill_words) {
+            poison(true);
+            return;
+        }
+        if (lane == 0) __stcg(reinterpret_cast<unsigned long long*>(ro + 128), reinterpret_cast<unsigned long long>(p.spill + wb));
+        out = p.spill + wb + base;
+        hdr_part |= HDR_SPILL;
+    }
     MergeIn M;
     M.bits = bits;
     M.proj = y0;
@@ -312,12 +342,18 @@ __device__ __forceinline__ void eval_gate(const SweepParams& p, const Env& E, co
     } else {
 #pragma unroll
         for (int q = 0; q < K; ++q)
-            M.ev[q] = reinterpret_cast<uint64_t>(region(in_loc[q], E) + 128) + 4 * ((hw[q] >> HDR_OFF_SHIFT) & HDR_OFF);
+            M.ev[q] = reinterpret_cast<uint64_t>(ev_base(region(in_loc[q], E), hw[q])) + 4 * ((hw[q] >> HDR_OFF_SHIFT) & HDR_OFF);
         my_n = merge_slot<K, false>(M, out, maxm);
     }
-    __stcg(ro_hdr + lane, my_n | (base << HDR_OFF_SHIFT) | (y0 << HDR_INIT_SHIFT) | (prev ? HDR_PREV : 0u));
+    __stcg(reinterpret_cast<uint32_t*>(region(out_loc, E)) + lane, my_n | hdr_part);
     // activity (reading C15) and latest PO arrival: counted once per
-    // slot across overflow rounds (where prev && !ovf)
+    // slot across rerun rounds -- only where the previous round poisoned this
+    // gate of this slot group (pass 0: everywhere)
+    bool prev = true;
+    if (RERUN) {
+        const uint64_t b = (uint64_t)__ldg(p.prev_idx + p.i_base + E.i) * (uint32_t)p.n_gates + (sig - (uint32_t)p.n_pi);
+        prev = (__ldg(p.pois_prev + (b >> 5)) >> (b & 31u)) & 1u;
+    }
     if (prev) {
         const uint32_t total = __reduce_add_sync(FULL, my_n);
         if (lane == 0 && total) atomicAdd(E.act_kv + (size_t)sig * (uint32_t)p.n_vdd, (unsigned long long)total);
@@ -329,13 +365,14 @@ __device__ __forceinline__ void eval_gate(const SweepParams& p, const Env& E, co
     }
 }
 
+template <bool RERUN>
 __device__ __forceinline__ void eval_dispatch(const SweepParams& p, const Env& E, const uint4 ins, const uint4 hd,
                                               const Staged& S) {
     switch ((hd.z >> 16) & 0xffu) {
-        case 1: eval_gate<1>(p, E, ins, hd, S); break;
-        case 2: eval_gate<2>(p, E, ins, hd, S); break;
-        case 3: eval_gate<3>(p, E, ins, hd, S); break;
-        default: eval_gate<4>(p, E, ins, hd, S); break;
+        case 1: eval_gate<1, RERUN>(p, E, ins, hd, S); break;
+        case 2: eval_gate<2, RERUN>(p, E, ins, hd, S); break;
+        case 3: eval_gate<3, RERUN>(p, E, ins, hd, S); break;
+        default: eval_gate<4, RERUN>(p, E, ins, hd, S); break;
     }
 }
 
@@ -357,7 +394,7 @@ constexpr int DW = 16;                                // gates per descriptor wi
 constexpr int OFF_DESC = 0, OFF_HDR = OFF_DESC + 2 * 16 * DW, OFF_EV = OFF_HDR + 4 * 128,
               OFF_META = OFF_EV + 2 * EV_STAGE;
 constexpr int WARP_SMEM_WORDS = OFF_META + 4;
-constexpr int LEVEL_SMEM_WORDS = 8;                   // delays of the current gate
+constexpr int LEVEL_SMEM_WORDS = 12;                  // delays of the current gate, group index
 
 __device__ __forceinline__ float* warp_smem(int warp, int words) {
     extern __shared__ __align__(16) float smem[];
@@ -384,6 +421,8 @@ __global__ void __launch_bounds__(AVFS_SWEEP_THREADS, AVFS_SWEEP_MINB) sweep_ker
     const uint4* gd = reinterpret_cast<const uint4*>(p.gates);
     for (int64_t i = blockIdx.x; i < p.n_sw; i += gridDim.x) {
         slot_group(p, i, lane, E);
+        __syncwarp();
+        if (lane == 0) meta[2] = (uint32_t)(p.i_base + i);
         const float4* dt = p.dtab + (int64_t)E.kv * p.n_gates * 2;
         for (int L = 0; L < p.depth; ++L) {
             const int ls = __ldg(p.level_ptr + L), le = __ldg(p.level_ptr + L + 1);
@@ -416,16 +455,16 @@ __global__ void __launch_bounds__(AVFS_SWEEP_THREADS, AVFS_SWEEP_MINB) sweep_ker
                 const uint32_t k = (lds_u32(d + 24) >> 16) & 0xffu;
                 const uint32_t sh = k > 2 ? 2u : (k > 1 ? 1u : 0u);      // log2 K'
                 const uint32_t q = (uint32_t)lane >> (5 - sh), sub = (uint32_t)lane & (31u >> sh);
-                uint32_t c = 0;
+                uint32_t c = 0, w = 0;
                 if (q < k) {
-                    const uint32_t w = lds_u32(s_hdr + 512 * (j & 3) + 128 * q + 124);
+                    w = lds_u32(s_hdr + 512 * (j & 3) + 128 * q + 124);
                     c = (((w >> HDR_OFF_SHIFT) & HDR_OFF) + (w & HDR_N) + 3) >> 2;
                 }
                 const uint32_t cap = (uint32_t)(EV_STAGE / 4) >> sh;   // chunks per input
                 const bool staged = __all_sync(FULL, c <= cap);
                 if (lane == 0) meta[j & 1] = staged ? 1u : 0u;
                 if (staged && sub < c) {
-                    const uint8_t* src = region(lds_u32(d + 4 * q), E) + 128 + 16 * sub;
+                    const uint8_t* src = ev_base(region(lds_u32(d + 4 * q), E), w) + 16 * sub;
                     const uint32_t dst = s_evr + 4 * EV_STAGE * (j & 1) + (4 * EV_STAGE >> sh) * q + 16 * sub;
                     cp_async16(dst, src);
                     const uint32_t st = 512u >> sh;                     // bytes covered by one pass of the lanes
@@ -461,8 +500,9 @@ __global__ void __launch_bounds__(AVFS_SWEEP_THREADS, AVFS_SWEEP_MINB) sweep_ker
                     S.hdr_s = s_hdr + 512 * (j & 3);
                     S.ev = meta[j & 1] != 0;
                     S.dly_s = d + 4 * 8 * DW;
+                    S.grp_s = smem_u32(meta + 2);
                     S.ev_s[0] = s_evr + 4 * EV_STAGE * (j & 1);
-                    eval_dispatch(p, E, dv[0], dv[1], S);
+                    eval_dispatch<false>(p, E, dv[0], dv[1], S);
                 }
             }
             __syncthreads();   // this level's stores -> the next levels' loads
@@ -483,6 +523,7 @@ __global__ void __launch_bounds__(512, 2) level_kernel(const SweepParams p, int 
     S.hdr = false;
     S.ev = false;
     S.dly_s = smem_u32(ws);
+    S.grp_s = smem_u32(ws + 8);
     const int g0 = __ldg(p.level_ptr + L);
     const int64_t items = (int64_t)(__ldg(p.level_ptr + L + 1) - g0) * p.n_sw;
     const int64_t gw = (int64_t)blockIdx.x * (blockDim.x >> 5) + warp;
@@ -494,8 +535,9 @@ __global__ void __launch_bounds__(512, 2) level_kernel(const SweepParams p, int 
         const float* dt = reinterpret_cast<const float*>(p.dtab) + ((int64_t)E.kv * p.n_gates + gi) * 8;
         __syncwarp();
         if (lane < 8) ws[lane] = __ldg(dt + lane);
+        if (lane == 8) reinterpret_cast<uint32_t*>(ws)[8] = (uint32_t)(p.i_base + i);
         __syncwarp();
-        eval_dispatch(p, E, __ldg(gd + 2 * gi), __ldg(gd + 2 * gi + 1), S);
+        eval_dispatch<true>(p, E, __ldg(gd + 2 * gi), __ldg(gd + 2 * gi + 1), S);
     }
 }
 
@@ -684,19 +726,20 @@ cudaError_t launch_pi_activity(const uint32_t* p1t, const uint32_t* p2t, int32_t
 // H7: list the slot groups whose pass overflowed (order is irrelevant: every
 // group's results are independent of where it is processed).
 __global__ void compact_kernel(const int32_t* __restrict__ ovf, int64_t n_sw, const int32_t* __restrict__ sw_list,
-                               int64_t sw_first, int32_t* out_list, int32_t* out_count) {
+                               int64_t sw_first, int32_t* out_list, int32_t* out_prev, int32_t* out_count) {
     const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (i >= n_sw || !ovf[i]) return;
     const int32_t pos = atomicAdd(out_count, 1);
     out_list[pos] = sw_list ? sw_list[i] : (int32_t)(sw_first + i);
+    out_prev[pos] = (int32_t)i;
 }
 
 cudaError_t launch_compact_overflow(const int32_t* ovf, int64_t n_sw, const int32_t* sw_list,
-                                    int64_t sw_first, int32_t* out_list, int32_t* out_count,
-                                    cudaStream_t st) {
+                                    int64_t sw_first, int32_t* out_list, int32_t* out_prev,
+                                    int32_t* out_count, cudaStream_t st) {
     if (n_sw == 0) return cudaSuccess;
     compact_kernel<<<(unsigned)((n_sw + 255) / 256), 256, 0, st>>>(ovf, n_sw, sw_list, sw_first, out_list,
-                                                                   out_count);
+                                                                   out_prev, out_count);
     return cudaGetLastError();
 }
 
@@ -733,7 +776,7 @@ __global__ void gather_kernel(const GatherParams p) {
         init = (h >> HDR_INIT_SHIFT) & 1u;
         n = (int)(h & HDR_N);
         const int off = (int)((h >> HDR_OFF_SHIFT) & HDR_OFF);
-        const float* ev = reinterpret_cast<const float*>(base + 128) + off;
+        const float* ev = reinterpret_cast<const float*>(ev_base(base, h)) + off;
         if (tout) for (int i = 0; i < p.cap; ++i) tout[i] = i < n ? ev[i] : 0.0f;
     }
     p.init[t] = (uint8_t)init;
@@ -781,7 +824,7 @@ __global__ void capture_kernel(const CaptureParams p) {
         const uint32_t h = reinterpret_cast<const uint32_t*>(base)[lane];
         init = (h >> HDR_INIT_SHIFT) & 1u;
         n = h & HDR_N;
-        const float* ev = reinterpret_cast<const float*>(base + 128) + ((h >> HDR_OFF_SHIFT) & HDR_OFF);
+        const float* ev = reinterpret_cast<const float*>(ev_base(base, h)) + ((h >> HDR_OFF_SHIFT) & HDR_OFF);
         if (valid)
             for (uint32_t e = 0; e < n; ++e) {
                 const float t = ev[e];

@@ -80,19 +80,28 @@ def test_deg_c_folded_polynomial_q_mode():
 
 @pytest.mark.parametrize("quantum", [Q, 0.0])
 def test_overflow_reruns_equal_large_capacity(quantum):
-    """Capacity 1 forces reruns (1 -> 4 -> 16 -> 64); results equal capacity 64 and the oracle."""
+    """Reading C17: the result is independent of capacity and of how overflow is handled.
+    No spill heap: capacity 1 forces reruns 1 -> 4 -> 16 -> 64.  A 4 KiB heap: it runs
+    out, the affected slot groups are rerun with larger heaps.  Default heap: every
+    oversize region spills, no rerun.  All equal capacity 64 and the oracle."""
     w = make_config(2, n_pairs=64, n_vdd=2)
-    st = full_compare(w, quantum, capacity=1, label="cap1")
+    st = full_compare(w, quantum, capacity=1, label="cap1-nospill", spill_bytes=-1)
     assert st["stats"]["rerun_rounds"] >= 2 and st["stats"]["overflow_slot_warps"] > 0
+    assert st["stats"]["spill_bytes"] == 0
+    st = full_compare(w, quantum, capacity=1, label="cap1-smallheap", spill_bytes=4096)
+    assert st["stats"]["rerun_rounds"] >= 1 and st["stats"]["spill_bytes"] > 0
+    st = full_compare(w, quantum, capacity=1, label="cap1-spill")
+    assert st["stats"]["rerun_rounds"] == 0 and st["stats"]["spill_bytes"] > 0
     full_compare(w, quantum, capacity=64, label="cap64")
 
 
-def test_overflow_exact_across_runs():
+@pytest.mark.parametrize("spill_bytes", [-1, 0, 8192])
+def test_overflow_exact_across_runs(spill_bytes):
     w = make_config(2, n_pairs=96, n_vdd=2)
     sig = np.arange(w.netlist.n_signals, dtype=np.int32)
     out = []
     for cap in (2, 64):
-        ctx = gpu_run(w, quantum=0.0, capacity=cap)
+        ctx = gpu_run(w, quantum=0.0, capacity=cap, spill_bytes=spill_bytes if cap == 2 else 0)
         out.append((ctx.activity(), ctx.latest_arrival(), *ctx.waveforms(sig, 0, 192, cap=48)))
         ctx.close()
     for a, b in zip(out[0], out[1]):
@@ -103,7 +112,10 @@ def test_capacity_exhausted_reports_error():
     from paper_conf_date_schneiderw20_b200 import AvfsError
     w = make_config(2, n_pairs=32, n_vdd=1)
     with pytest.raises(AvfsError) as e:
-        gpu_run(w, capacity=1, max_rerun_rounds=0)
+        gpu_run(w, capacity=1, max_rerun_rounds=0, spill_bytes=-1)
+    assert e.value.status == 7
+    with pytest.raises(AvfsError) as e:
+        gpu_run(w, capacity=1, max_rerun_rounds=0, spill_bytes=64)
     assert e.value.status == 7
 
 
