@@ -834,7 +834,9 @@ static avfs_status run_round(avfs_ctx* ctx, Round& R, int round_idx, const int32
     // spill heap: the requested size, within free device memory (keep 1 GiB)
     if ((int)ctx->spill.size() <= round_idx) ctx->spill.resize(round_idx + 1);
     R.spill_words = 0;
-    if (R.spill_want > 0) {
+    if (R.spill_want > 0 && ctx->spill[round_idx].n >= (size_t)R.spill_want * 4) {
+        R.spill_words = R.spill_want;                  // reuse the heap of a previous simulate
+    } else if (R.spill_want > 0) {
         size_t fr = 0, tot = 0;
         CK(cudaMemGetInfo(&fr, &tot));
         const size_t have = ctx->spill[round_idx].n;

@@ -170,15 +170,15 @@ __device__ __forceinline__ uint32_t merge_slot(const MergeIn& M, float* out, uin
     typedef typename EvAddr<STAGED>::T A;
     uint32_t bits = M.bits, proj = M.proj;
     const uint32_t tt = M.tt;
-    float* op = out;                             // next output slot (only the last output can be cancelled)
+    uint32_t cnt = 0;                            // outputs kept so far (only the last can be cancelled)
     float tl = -AVFS_INF;
     auto step = [&](float t, bool live, uint32_t y, float d) {
         const float co = t + d;
         const bool change = live && y != proj;
         const bool cancel = change && tl > t;
         const bool push = change && !cancel;
-        if (push) __stcg(op, co);
-        op += push ? 1 : (cancel ? -1 : 0);
+        if (push) __stcg(out + cnt, co);
+        cnt = cnt + (push ? 1u : 0u) - (cancel ? 1u : 0u);
         tl = push ? co : (cancel ? -AVFS_INF : tl);
         proj = y;
     };
@@ -206,7 +206,7 @@ __device__ __forceinline__ uint32_t merge_slot(const MergeIn& M, float* out, uin
 #pragma unroll 1
         for (uint32_t it = 0; it < steps; ++it) {
             const bool p = h1 < h0;             // ties: pin 0 first
-            const float t = p ? h1 : h0;
+            const float t = fminf(h0, h1);
             const A a = p ? a1 : a0;
             const float nx = a < (p ? e1 : e0) ? ld_ev<STAGED>(a) : AVFS_INF;
             h1 = p ? nx : h1;
@@ -252,7 +252,7 @@ __device__ __forceinline__ uint32_t merge_slot(const MergeIn& M, float* out, uin
             step(t, live, y, lds_f32(M.dly_s + 8 * pm + 4 * y));
         }
     }
-    return (uint32_t)(op - out);
+    return cnt;
 }
 
 template <int K, bool RERUN>
@@ -450,6 +450,7 @@ __global__ void __launch_bounds__(AVFS_SWEEP_THREADS, AVFS_SWEEP_MINB) sweep_ker
             // input q's events (extent = lane 31's offset + count) -> slot q of
             // the stage (EV_STAGE / K' words, 32 / K' lanes per input, <= 2
             // chunks of 16 B per lane); staged only if every input fits
+            bool staged_next = false, staged_cur = false;
             auto issue_ev = [&](int j) {
                 const uint32_t d = desc_at(j);
                 const uint32_t k = (lds_u32(d + 24) >> 16) & 0xffu;
@@ -462,7 +463,7 @@ __global__ void __launch_bounds__(AVFS_SWEEP_THREADS, AVFS_SWEEP_MINB) sweep_ker
                 }
                 const uint32_t cap = (uint32_t)(EV_STAGE / 4) >> sh;   // chunks per input
                 const bool staged = __all_sync(FULL, c <= cap);
-                if (lane == 0) meta[j & 1] = staged ? 1u : 0u;
+                staged_next = staged;
                 if (staged && sub < c) {
                     const uint8_t* src = ev_base(region(lds_u32(d + 4 * q), E), w) + 16 * sub;
                     const uint32_t dst = s_evr + 4 * EV_STAGE * (j & 1) + (4 * EV_STAGE >> sh) * q + 16 * sub;
@@ -484,6 +485,7 @@ __global__ void __launch_bounds__(AVFS_SWEEP_THREADS, AVFS_SWEEP_MINB) sweep_ker
                 cp_async_wait_all();
                 __syncwarp();
                 issue_ev(0);
+                staged_cur = staged_next;
                 cp_async_commit();
 #pragma unroll 1
                 for (int j = 0; j < nj; ++j) {
@@ -491,14 +493,16 @@ __global__ void __launch_bounds__(AVFS_SWEEP_THREADS, AVFS_SWEEP_MINB) sweep_ker
                     __syncwarp();
                     if (j % DW == 0 && j > 0 && j + DW < nj) issue_win(j / DW + 1);
                     if (j + 2 < nj) issue_hdr(j + 2);
+                    const bool st_j = staged_cur;
                     if (j + 1 < nj) issue_ev(j + 1);
+                    staged_cur = staged_next;
                     cp_async_commit();
                     const uint32_t d = desc_at(j);
                     const uint4* dv = reinterpret_cast<const uint4*>(ws + OFF_DESC + 16 * DW * ((j / DW) & 1) + 8 * (j % DW));
                     Staged S;
                     S.hdr = true;
                     S.hdr_s = s_hdr + 512 * (j & 3);
-                    S.ev = meta[j & 1] != 0;
+                    S.ev = st_j;
                     S.dly_s = d + 4 * 8 * DW;
                     S.grp_s = smem_u32(meta + 2);
                     S.ev_s[0] = s_evr + 4 * EV_STAGE * (j & 1);
