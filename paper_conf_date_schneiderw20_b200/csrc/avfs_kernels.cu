@@ -417,6 +417,7 @@ __global__ void __launch_bounds__(AVFS_SWEEP_THREADS, AVFS_SWEEP_MINB) sweep_ker
     float* ws = warp_smem(warp, WARP_SMEM_WORDS);
     const uint32_t s_desc = smem_u32(ws + OFF_DESC), s_hdr = smem_u32(ws + OFF_HDR), s_evr = smem_u32(ws + OFF_EV);
     uint32_t* meta = reinterpret_cast<uint32_t*>(ws + OFF_META);
+    const uint32_t s_grp = smem_u32(meta + 2);
     E.stride = (uint32_t)(p.pin_n_sw * p.region_bytes);
     const uint4* gd = reinterpret_cast<const uint4*>(p.gates);
     for (int64_t i = blockIdx.x; i < p.n_sw; i += gridDim.x) {
@@ -439,8 +440,8 @@ __global__ void __launch_bounds__(AVFS_SWEEP_THREADS, AVFS_SWEEP_MINB) sweep_ker
                     cp_async16(w + 4 * 8 * DW, dt + 2 * g + (lane & 1));
                 }
             };
-            auto desc_at = [&](int j) { return s_desc + 4 * 16 * DW * ((j / DW) & 1) + 32 * (j % DW); };
-            auto issue_hdr = [&](int j) {
+            auto desc_at = [&](uint32_t j) { return s_desc + 4 * 16 * DW * ((j / DW) & 1) + 32 * (j % DW); };
+            auto issue_hdr = [&](uint32_t j) {
                 const uint32_t d = desc_at(j);
                 const uint32_t q = (uint32_t)lane >> 3;
                 if (q < ((lds_u32(d + 24) >> 16) & 0xffu))
@@ -451,7 +452,7 @@ __global__ void __launch_bounds__(AVFS_SWEEP_THREADS, AVFS_SWEEP_MINB) sweep_ker
             // the stage (EV_STAGE / K' words, 32 / K' lanes per input, <= 2
             // chunks of 16 B per lane); staged only if every input fits
             bool staged_next = false, staged_cur = false;
-            auto issue_ev = [&](int j) {
+            auto issue_ev = [&](uint32_t j) {
                 const uint32_t d = desc_at(j);
                 const uint32_t k = (lds_u32(d + 24) >> 16) & 0xffu;
                 const uint32_t sh = k > 2 ? 2u : (k > 1 ? 1u : 0u);      // log2 K'
@@ -487,14 +488,15 @@ __global__ void __launch_bounds__(AVFS_SWEEP_THREADS, AVFS_SWEEP_MINB) sweep_ker
                 issue_ev(0);
                 staged_cur = staged_next;
                 cp_async_commit();
+                const uint32_t nju = (uint32_t)nj;
 #pragma unroll 1
-                for (int j = 0; j < nj; ++j) {
+                for (uint32_t j = 0; j < nju; ++j) {
                     cp_async_wait_all();
                     __syncwarp();
-                    if (j % DW == 0 && j > 0 && j + DW < nj) issue_win(j / DW + 1);
-                    if (j + 2 < nj) issue_hdr(j + 2);
+                    if (j % DW == 0 && j > 0 && j + DW < nju) issue_win((int)(j / DW) + 1);
+                    if (j + 2 < nju) issue_hdr(j + 2);
                     const bool st_j = staged_cur;
-                    if (j + 1 < nj) issue_ev(j + 1);
+                    if (j + 1 < nju) issue_ev(j + 1);
                     staged_cur = staged_next;
                     cp_async_commit();
                     const uint32_t d = desc_at(j);
@@ -504,7 +506,7 @@ __global__ void __launch_bounds__(AVFS_SWEEP_THREADS, AVFS_SWEEP_MINB) sweep_ker
                     S.hdr_s = s_hdr + 512 * (j & 3);
                     S.ev = st_j;
                     S.dly_s = d + 4 * 8 * DW;
-                    S.grp_s = smem_u32(meta + 2);
+                    S.grp_s = s_grp;
                     S.ev_s[0] = s_evr + 4 * EV_STAGE * (j & 1);
                     eval_dispatch<false>(p, E, dv[0], dv[1], S);
                 }
