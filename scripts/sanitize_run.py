@@ -1,4 +1,4 @@
-"""Small end-to-end runs for compute-sanitizer (c17 keep-all, multiplier with reruns, random DAG)."""
+"""Small end-to-end runs for compute-sanitizer (c17 keep-all, multiplier with spills and reruns, random DAG)."""
 import os, sys
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import numpy as np
@@ -7,14 +7,15 @@ from workloads import make_config
 
 for cfg, kw in ((1, dict(n_pairs=64)), (2, dict(n_pairs=64, n_vdd=2)), (3, dict(n_pairs=64, n_vdd=2, scale=0.02))):
     w = make_config(cfg, **kw)
-    for cap in (1, 8):
+    for cap, spill in ((1, 0), (1, -1), (1, 4096), (8, 0)):
         ctx = Context(0)
         load_workload(ctx, w.netlist, w.library, w.stimuli, w.vdd)
-        ctx.set_options(capacity=cap, keep_all=(cfg == 1), max_rerun_rounds=4)
+        ctx.set_options(capacity=cap, keep_all=(cfg == 1), max_rerun_rounds=4, spill_bytes=spill)
         ctx.simulate()
         a = ctx.activity()
         ctx.waveforms(w.netlist.po_sig, 0, w.n_slots, cap=8)
         ctx.capture(np.full(len(w.vdd), 50.0, np.float32))
         ctx.switching_energy()
-        print(cfg, cap, int(a.sum()), ctx.stats()["rerun_rounds"], flush=True)
+        st = ctx.stats()
+        print(cfg, cap, spill, int(a.sum()), st["rerun_rounds"], st["spill_bytes"], flush=True)
         ctx.close()
