@@ -316,6 +316,7 @@ def main():
         p2h = torch.from_numpy(w.stimuli.p2.view(np.int32)).pin_memory().numpy().view(np.uint32)
         h2d = int(p1h.nbytes + p2h.nbytes)
         d2h = int(n_sig * V * 8 + V * 4)
+        act_h = torch.empty((n_sig, V), dtype=torch.int64).pin_memory().numpy().view(np.uint64)
         e2e_ms = []
         for i in range(args.steps + 1):
             with torch.cuda.stream(stream):
@@ -324,7 +325,7 @@ def main():
             t0 = time.perf_counter()
             ctx.set_stimuli(p1h, p2h)
             ctx.simulate(stream)
-            a = ctx.activity()
+            a = ctx.activity(act_h)
             lat = ctx.latest_arrival()
             if world > 1:
                 import torch.distributed as dist

@@ -266,9 +266,15 @@ class Context:
 
     # ------------------------------------------------------------ (4)
     def activity(self, out=None) -> np.ndarray:
-        """[n_signals][n_vdd] uint64; `out` may be a torch CUDA int64/uint64 tensor."""
+        """[n_signals][n_vdd] uint64; `out` may be a torch CUDA int64/uint64 tensor
+        (device copy) or a C-contiguous uint64 numpy array (e.g. pinned host memory)."""
         if out is not None and hasattr(out, "data_ptr"):
             self._ck(self.lib.avfs_get_activity(self.h, C.c_void_p(out.data_ptr()), 1))
+            return out
+        if out is not None:
+            if out.dtype != np.uint64 or out.shape != (self.n_signals, self.n_vdd) or not out.flags.c_contiguous:
+                raise ValueError("activity out must be C-contiguous uint64 [n_signals][n_vdd]")
+            self._ck(self.lib.avfs_get_activity(self.h, _p(out), 0))
             return out
         a = np.zeros((self.n_signals, self.n_vdd), np.uint64)
         self._ck(self.lib.avfs_get_activity(self.h, _p(a), 0))

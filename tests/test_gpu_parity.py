@@ -253,3 +253,7 @@ def test_device_stimuli_and_torch_stream():
     out = torch.zeros((w.netlist.n_signals, 2), dtype=torch.int64, device="cuda")
     ctx.activity(out)
     assert np.array_equal(out.cpu().numpy().astype(np.uint64), a.activity())
+    # host readback into a caller-owned pinned buffer (bench.py's e2e path)
+    pinned = torch.empty((w.netlist.n_signals, 2), dtype=torch.int64).pin_memory().numpy().view(np.uint64)
+    assert ctx.activity(pinned) is pinned
+    assert np.array_equal(pinned, a.activity())
