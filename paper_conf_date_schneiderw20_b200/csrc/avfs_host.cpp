@@ -65,6 +65,7 @@ struct Round {
     int64_t spill_want = 0;          // requested heap words (0: no spill heap)
     int64_t spill_words = 0;         // heap words allocated for this round
     int64_t spill_req = 0;           // words requested by the round's gate-warps (incl. failed)
+    int32_t grp = 1;                 // slot groups per sweep CTA
 };
 
 }  // namespace
@@ -822,7 +823,17 @@ static avfs_status run_round(avfs_ctx* ctx, Round& R, int round_idx, const int32
     else CK(level_occupancy(wpc, smem, &bps));
     if (bps < 1) return fail(ctx, AVFS_ERR_CAPACITY, "sweep kernel does not fit on an SM (smem %d)", smem);
     const int64_t resident = (int64_t)ctx->n_sm * bps;
-    R.grid = (int32_t)(persistent ? std::min<int64_t>(R.n_sw, resident) : resident);
+    // narrow netlists (few gates per level): one sweep CTA walks G slot groups
+    // at once so that every warp has >= 2 gates of a level (power of 2, <= wpc)
+    int grp = 1;
+    if (persistent) {
+        const double per_level = ctx->depth > 0 ? (double)ctx->n_gates / ctx->depth : 1.0;
+        while (grp < wpc && per_level / (double)(wpc / grp) < 2.0) grp *= 2;
+        if (const char* e = getenv("AVFS_GROUPS_PER_CTA")) grp = std::max(1, std::min(wpc, atoi(e)));
+        while (wpc % grp) grp /= 2;
+    }
+    R.grp = grp;
+    R.grid = (int32_t)(persistent ? std::min<int64_t>((R.n_sw + grp - 1) / grp, resident) : resident);
     if (R.grid < 1) R.grid = 1;
     if ((int)ctx->arena.size() <= round_idx) ctx->arena.resize(round_idx + 1);
     const int64_t n_buf = (int64_t)ctx->n_pi + ctx->n_pinned + ctx->n_scratch;
@@ -875,6 +886,7 @@ static avfs_status run_round(avfs_ctx* ctx, Round& R, int round_idx, const int32
     p.arena = ctx->arena[round_idx].as<uint8_t>();
     p.region_bytes = R.region_bytes;
     p.W = R.W;
+    p.grp_per_cta = R.grp;
     p.n_pi = ctx->n_pi;
     p.spill = ctx->spill[round_idx].as<float>();
     p.spill_top = ctx->d_spill_top.as<unsigned long long>() + round_idx;

@@ -420,16 +420,21 @@ __global__ void __launch_bounds__(AVFS_SWEEP_THREADS, AVFS_SWEEP_MINB) sweep_ker
     const uint32_t s_grp = smem_u32(meta + 2);
     E.stride = (uint32_t)(p.pin_n_sw * p.region_bytes);
     const uint4* gd = reinterpret_cast<const uint4*>(p.gates);
-    for (int64_t i = blockIdx.x; i < p.n_sw; i += gridDim.x) {
-        slot_group(p, i, lane, E);
+    // narrow netlists: the CTA walks G slot groups at once, nw / G warps each
+    const int G = p.grp_per_cta, wpg = nw / G;
+    const int sg = warp / wpg, wl = warp % wpg;
+    for (int64_t i0 = (int64_t)blockIdx.x * G; i0 < p.n_sw; i0 += (int64_t)gridDim.x * G) {
+        const int64_t i = i0 + sg;
+        const bool valid = i < p.n_sw;                 // idle warps still meet every level barrier
+        slot_group(p, valid ? i : i0, lane, E);
         __syncwarp();
-        if (lane == 0) meta[2] = (uint32_t)(p.i_base + i);
+        if (lane == 0) meta[2] = (uint32_t)(p.i_base + (valid ? i : i0));
         const float4* dt = p.dtab + (int64_t)E.kv * p.n_gates * 2;
         for (int L = 0; L < p.depth; ++L) {
             const int ls = __ldg(p.level_ptr + L), le = __ldg(p.level_ptr + L + 1);
-            const int B = (le - ls + nw - 1) / nw;
-            const int g0 = ls + warp * B;
-            const int nj = max(0, min(B, le - g0));
+            const int B = (le - ls + wpg - 1) / wpg;
+            const int g0 = ls + wl * B;
+            const int nj = valid ? max(0, min(B, le - g0)) : 0;
             // descriptor window k (gates g0 + 16k ..): lane copies 16 B of the
             // descriptors (lanes 0..31 = 16 gates x 2) and 16 B of the delays
             auto issue_win = [&](int k) {

@@ -257,3 +257,19 @@ def test_device_stimuli_and_torch_stream():
     pinned = torch.empty((w.netlist.n_signals, 2), dtype=torch.int64).pin_memory().numpy().view(np.uint64)
     assert ctx.activity(pinned) is pinned
     assert np.array_equal(pinned, a.activity())
+
+
+def test_groups_per_cta_invariance(monkeypatch):
+    """Narrow netlists sweep several slot groups per CTA (warps split between
+    them); the result must not depend on the split (incl. idle tail warps)."""
+    w = make_config(2, n_pairs=200, n_vdd=3)
+    sig = np.arange(w.netlist.n_signals, dtype=np.int32)
+    out = []
+    for g in ("1", "2", "8", "32"):
+        monkeypatch.setenv("AVFS_GROUPS_PER_CTA", g)
+        ctx = gpu_run(w, quantum=0.0, capacity=8)
+        out.append((ctx.activity(), ctx.latest_arrival(), *ctx.waveforms(sig, 0, w.n_slots, cap=32)))
+        ctx.close()
+    for o in out[1:]:
+        for a, b in zip(out[0], o):
+            assert np.array_equal(a, b)
