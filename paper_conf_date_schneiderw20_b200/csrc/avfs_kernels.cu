@@ -30,6 +30,10 @@
 
 #include "avfs_internal.h"
 
+#ifndef AVFS_PTX_MERGE
+#define AVFS_PTX_MERGE 1      // 2-input staged merge as one PTX loop (0: the C++ loop)
+#endif
+
 namespace avfs {
 
 // Waveforms are produced and consumed inside one launch: read them at L2
@@ -165,6 +169,69 @@ __device__ __forceinline__ float ld_ev(uint64_t a) {
 template <bool STAGED> struct EvAddr { typedef uint64_t T; };
 template <> struct EvAddr<true> { typedef uint32_t T; };
 
+// The 2-input merge + inertial filter over shared-memory lists, as one PTX
+// loop with in-place predicated updates (the compiled C++ loop spends ~10 of
+// its ~41 instructions per step on register copies and constants).  Same
+// semantics as the generic step: ties pick pin 0, a change whose time
+// precedes the pending output cancels it (equality kept), outputs are stored
+// as they are pushed.  steps >= 1.
+__device__ __forceinline__ uint32_t merge2_smem(uint32_t a0, uint32_t e0, uint32_t a1, uint32_t e1, uint32_t bits,
+                                                uint32_t proj, uint32_t tt, float4 dl, float* out, uint32_t steps) {
+    float h0 = a0 < e0 ? lds_f32(a0) : AVFS_INF;
+    float h1 = a1 < e1 ? lds_f32(a1) : AVFS_INF;
+    a0 += 4;
+    a1 += 4;
+    float tl = -AVFS_INF;
+    uint32_t cnt = 0, it = 0;
+    asm volatile(
+        "{\n"
+        ".reg .pred p, ok, live, y1, chg, canc, push, more;\n"
+        ".reg .f32 t, nx, dA, dB, d, co;\n"
+        ".reg .b32 a, e, y, sh;\n"
+        ".reg .b64 ad;\n"
+        "MERGE2_%=:\n"
+        "setp.lt.f32 p, %1, %0;\n"
+        "min.f32 t, %0, %1;\n"
+        "selp.b32 a, %3, %2, p;\n"
+        "selp.b32 e, %10, %9, p;\n"
+        "setp.lt.u32 ok, a, e;\n"
+        "mov.f32 nx, 0f7F800000;\n"
+        "@ok ld.shared.f32 nx, [a];\n"
+        "@p add.u32 %3, %3, 4;\n"
+        "@!p add.u32 %2, %2, 4;\n"
+        "@p mov.f32 %1, nx;\n"
+        "@!p mov.f32 %0, nx;\n"
+        "setp.lt.f32 live, t, 0f7F800000;\n"
+        "selp.b32 sh, 2, 1, p;\n"
+        "@live xor.b32 %4, %4, sh;\n"
+        "shr.u32 y, %11, %4;\n"
+        "and.b32 y, y, 1;\n"
+        "setp.ne.u32 y1, y, 0;\n"
+        "selp.f32 dA, %15, %14, y1;\n"
+        "selp.f32 dB, %13, %12, y1;\n"
+        "selp.f32 d, dA, dB, p;\n"
+        "add.rn.f32 co, t, d;\n"
+        "setp.ne.and.u32 chg, y, %5, live;\n"
+        "setp.gt.and.f32 canc, %6, t, chg;\n"
+        "setp.le.and.f32 push, %6, t, chg;\n"
+        "mul.wide.u32 ad, %7, 4;\n"
+        "add.u64 ad, ad, %16;\n"
+        "@push st.global.cg.f32 [ad], co;\n"
+        "@push add.u32 %7, %7, 1;\n"
+        "@canc sub.u32 %7, %7, 1;\n"
+        "@push mov.f32 %6, co;\n"
+        "@canc mov.f32 %6, 0fFF800000;\n"
+        "mov.b32 %5, y;\n"
+        "add.u32 %8, %8, 1;\n"
+        "setp.lt.u32 more, %8, %17;\n"
+        "@more bra MERGE2_%=;\n"
+        "}\n"
+        : "+f"(h0), "+f"(h1), "+r"(a0), "+r"(a1), "+r"(bits), "+r"(proj), "+f"(tl), "+r"(cnt), "+r"(it)
+        : "r"(e0), "r"(e1), "r"(tt), "f"(dl.x), "f"(dl.y), "f"(dl.z), "f"(dl.w), "l"(out), "r"(steps)
+        : "memory");
+    return cnt;
+}
+
 template <int K, bool STAGED>
 __device__ __forceinline__ uint32_t merge_slot(const MergeIn& M, float* out, uint32_t steps) {
     typedef typename EvAddr<STAGED>::T A;
@@ -196,6 +263,10 @@ __device__ __forceinline__ uint32_t merge_slot(const MergeIn& M, float* out, uin
             const uint32_t y = (tt >> bits) & 1u;
             step(t, live, y, y ? M.d01.y : M.d01.x);
         }
+    } else if (K == 2 && STAGED && AVFS_PTX_MERGE) {
+        return steps ? merge2_smem((uint32_t)M.ev[0], (uint32_t)M.ev[0] + 4 * (uint32_t)M.n[0], (uint32_t)M.ev[1],
+                                   (uint32_t)M.ev[1] + 4 * (uint32_t)M.n[1], bits, proj, tt, M.d01, out, steps)
+                     : 0u;
     } else if (K == 2) {
         A a0 = (A)M.ev[0], a1 = (A)M.ev[1];
         const A e0 = a0 + 4 * (uint32_t)M.n[0], e1 = a1 + 4 * (uint32_t)M.n[1];
