@@ -587,7 +587,10 @@ __global__ void __launch_bounds__(AVFS_SWEEP_THREADS, AVFS_SWEEP_MINB) sweep_ker
                     eval_dispatch<false>(p, E, dv[0], dv[1], S);
                 }
             }
-            __syncthreads();   // this level's stores -> the next levels' loads
+            // this level's stores -> the next levels' loads; with several slot
+            // groups per CTA each group syncs only its own warps (named barrier)
+            if (G == 1 || G > 15) __syncthreads();
+            else asm volatile("bar.sync %0, %1;" ::"r"(1 + sg), "r"(32 * wpg) : "memory");
         }
     }
 }
