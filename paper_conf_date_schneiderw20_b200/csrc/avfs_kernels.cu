@@ -267,6 +267,34 @@ __device__ __forceinline__ uint32_t merge_slot(const MergeIn& M, float* out, uin
         return steps ? merge2_smem((uint32_t)M.ev[0], (uint32_t)M.ev[0] + 4 * (uint32_t)M.n[0], (uint32_t)M.ev[1],
                                    (uint32_t)M.ev[1] + 4 * (uint32_t)M.n[1], bits, proj, tt, M.d01, out, steps)
                      : 0u;
+    } else if (K == 2 && !STAGED) {
+        // lists in L2: each list keeps its head and the next two elements in
+        // registers, so the load feeding a comparison was issued >= 2 advances
+        // of that list earlier
+        A a0 = (A)M.ev[0], a1 = (A)M.ev[1];
+        const A e0 = a0 + 4 * (uint32_t)M.n[0], e1 = a1 + 4 * (uint32_t)M.n[1];
+        float h0 = a0 < e0 ? ld_ev<false>(a0) : AVFS_INF, g0 = a0 + 4 < e0 ? ld_ev<false>(a0 + 4) : AVFS_INF,
+              f0 = a0 + 8 < e0 ? ld_ev<false>(a0 + 8) : AVFS_INF;
+        float h1 = a1 < e1 ? ld_ev<false>(a1) : AVFS_INF, g1 = a1 + 4 < e1 ? ld_ev<false>(a1 + 4) : AVFS_INF,
+              f1 = a1 + 8 < e1 ? ld_ev<false>(a1 + 8) : AVFS_INF;
+        a0 += 12;
+        a1 += 12;
+#pragma unroll 1
+        for (uint32_t it = 0; it < steps; ++it) {
+            const bool p = h1 < h0;             // ties: pin 0 first
+            const float t = fminf(h0, h1);
+            const A a = p ? a1 : a0;
+            const float nx = a < (p ? e1 : e0) ? ld_ev<false>(a) : AVFS_INF;
+            if (p) {
+                h1 = g1; g1 = f1; f1 = nx; a1 += 4;
+            } else {
+                h0 = g0; g0 = f0; f0 = nx; a0 += 4;
+            }
+            const bool live = t < AVFS_INF;
+            bits ^= live ? (p ? 2u : 1u) : 0u;
+            const uint32_t y = (tt >> bits) & 1u;
+            step(t, live, y, p ? (y ? M.d01.w : M.d01.z) : (y ? M.d01.y : M.d01.x));
+        }
     } else if (K == 2) {
         A a0 = (A)M.ev[0], a1 = (A)M.ev[1];
         const A e0 = a0 + 4 * (uint32_t)M.n[0], e1 = a1 + 4 * (uint32_t)M.n[1];
