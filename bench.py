@@ -209,10 +209,12 @@ def run_reference(args, w, world, rank):
 
 def config_dict(w, args):
     d = w.describe()
-    d.update({"slots": w.n_slots, "evals_per_step": w.evals,
+    n = getattr(args, "shard_slots", None) or w.n_slots
+    d.update({"slots": n, "evals_per_step": w.netlist.n_gates * n,
               "mode": "F (FP64 delay polynomials, FP32 times)" if args.quantum == 0 else f"Q (quantum {args.quantum} ps)",
               "l2": "flushed by a 256 MiB write between timed steps; waveform arena >> L2",
-              "parallelism": f"slot-shard x{args.gpus} ({args.scaling})"})
+              "parallelism": (f"one slot shard of {args.shard_of} (rank 0), 1 GPU" if args.shard_of > 1 else
+                              f"slot-shard x{args.gpus} ({args.scaling})")})
     return d
 
 
@@ -229,6 +231,9 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--scaling", default="weak", choices=["weak", "strong"])
+    ap.add_argument("--shard-of", type=int, default=0,
+                    help="N=1 only: simulate rank 0's shard of an N-GPU run (e.g. config 5, "
+                         "specified on 8 x B200, does not fit one GPU whole)")
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3) if args.impl == "avfs" else args.warmup
 
@@ -255,6 +260,10 @@ def main():
     ctx.set_options(capacity=cap, quantum_ps=args.quantum, warps_per_cta=args.warps_per_cta, profile=True)
     total_slots = w.n_slots
     first, n_local = shard_range(total_slots, rank, world)
+    if args.shard_of > 1 and world == 1:
+        first, n_local = shard_range(total_slots, 0, args.shard_of)
+        total_slots = n_local
+        args.shard_slots = n_local
     ctx.set_slot_range(first, n_local)
     n_sig, V = w.netlist.n_signals, len(w.vdd)
     act_dev = torch.zeros((n_sig, V), dtype=torch.int64, device=dev)

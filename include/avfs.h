@@ -171,9 +171,11 @@ typedef struct {
                                   more than 32*C events (rerun at 4C)       */
     int32_t warps_per_cta;     /* 0: default (8)                              */
     int32_t profile;           /* 1: time the sweep kernel with CUDA events  */
-    int64_t spill_bytes;       /* pass-0 spill heap: 0 = auto (arena/4, at
-                                  least 256 MiB, within free memory); > 0 =
-                                  this many bytes; < 0 = no spill heap     */
+    int64_t spill_bytes;       /* pass-0 spill heap: 0 = auto (the larger of
+                                  arena/4, 256 MiB and 1.25x what the
+                                  previous simulate on this context asked
+                                  for, within free memory); > 0 = this many
+                                  bytes; < 0 = no spill heap               */
 } avfs_options;
 avfs_status avfs_set_options(avfs_ctx *ctx, const avfs_options *opt);
 avfs_status avfs_default_options(avfs_options *opt);

@@ -131,6 +131,7 @@ struct avfs_ctx {
         g_times, g_bad;
     std::vector<DevBuf> arena;        // per round: [buffer][slot group][region]
     std::vector<DevBuf> spill;        // per round: spill heap (kept: readback may point into it)
+    int64_t spill_hint = 0;           // heap words the last simulate asked for (all rounds)
     int32_t* h_pinned = nullptr;      // small pinned host buffer (count, err)
     cudaEvent_t ev0 = nullptr, ev1 = nullptr;
 
@@ -980,6 +981,10 @@ avfs_status avfs_simulate(avfs_ctx* ctx, void* cuda_stream) {
     ctx->stats.launches += 2;
 
     ctx->rounds.clear();
+    // rerun rounds' arenas and heaps of the previous simulate are stale: give
+    // their memory back so that pass 0 can size its heap from the hint
+    for (size_t r = 1; r < ctx->arena.size(); ++r) ctx->arena[r].release();
+    for (size_t r = 1; r < ctx->spill.size(); ++r) ctx->spill[r].release();
     Round R0;
     R0.n_sw = sw_hi - sw_lo;
     R0.sw_first = sw_lo;
@@ -988,8 +993,11 @@ avfs_status avfs_simulate(avfs_ctx* ctx, void* cuda_stream) {
     R0.region_bytes = 128 + 4 * (int64_t)R0.W;
     {
         const int64_t arena_words = ((int64_t)ctx->n_pi + ctx->n_pinned + ctx->n_scratch) * R0.n_sw * R0.region_bytes / 4;
+        // auto: arena/4 (>= 256 MiB), or 1.25x what the previous simulate asked
+        // for in all its rounds, so that repeated runs do not rerun
         R0.spill_want = ctx->opt.spill_bytes > 0 ? ctx->opt.spill_bytes / 4
-                      : ctx->opt.spill_bytes < 0 ? 0 : std::max<int64_t>(arena_words / 4, (256ll << 20) / 4);
+                      : ctx->opt.spill_bytes < 0 ? 0
+                      : std::max<int64_t>({arena_words / 4, (256ll << 20) / 4, ctx->spill_hint + ctx->spill_hint / 4});
     }
     st = run_round(ctx, R0, 0, nullptr, nullptr, ctx->opt.profile != 0);
     if (st != AVFS_OK) return st;
@@ -1045,6 +1053,11 @@ avfs_status avfs_simulate(avfs_ctx* ctx, void* cuda_stream) {
         if (st != AVFS_OK) return st;
         ctx->rounds.push_back(std::move(Rn));
         cur ^= 1;
+    }
+    {
+        int64_t req = 0;
+        for (const Round& R : ctx->rounds) req += R.spill_req;
+        ctx->spill_hint = req;
     }
     if (ctx->opt.profile) {
         float ms = 0;
