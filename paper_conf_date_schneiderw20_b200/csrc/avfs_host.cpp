@@ -66,6 +66,7 @@ struct Round {
     int64_t spill_words = 0;         // heap words allocated for this round
     int64_t spill_req = 0;           // words requested by the round's gate-warps (incl. failed)
     int32_t grp = 1;                 // slot groups per sweep CTA
+    int32_t split = 1;               // sweep CTAs per slot group
 };
 
 }  // namespace
@@ -127,7 +128,7 @@ struct avfs_ctx {
     // device state
     bool dev_net_valid = false, dev_vdd_valid = false;
     DevBuf d_gates, d_ddesc, d_dtab, d_coef, d_cload, d_island, d_energy, c_loc, c_tclk, c_slot, c_out, d_level_ptr, d_vdd, d_p1, d_p2, d_p1t, d_p2t, d_act, d_latest, d_ovf,
-        d_err, d_list[2], d_prev[2], d_pois[2], d_spill_top, d_count, d_swround, d_swindex, g_loc, g_init, g_count,
+        d_err, d_list[2], d_prev[2], d_pois[2], d_spill_top, d_lvlsync, d_count, d_swround, d_swindex, g_loc, g_init, g_count,
         g_times, g_bad;
     std::vector<DevBuf> arena;        // per round: [buffer][slot group][region]
     std::vector<DevBuf> spill;        // per round: spill heap (kept: readback may point into it)
@@ -834,7 +835,28 @@ static avfs_status run_round(avfs_ctx* ctx, Round& R, int round_idx, const int32
         while (wpc % grp) grp /= 2;
     }
     R.grp = grp;
-    R.grid = (int32_t)(persistent ? std::min<int64_t>((R.n_sw + grp - 1) / grp, resident) : resident);
+    // few slot groups for the SMs (last wave mostly empty): S co-resident CTAs
+    // share a group; S minimises waves / S, ties to the smaller S, and every
+    // warp keeps >= 2 gates of a level
+    int split = 1;
+    if (persistent && grp == 1) {
+        const double per_level = ctx->depth > 0 ? (double)ctx->n_gates / ctx->depth : 1.0;
+        double best = 1e300;
+        for (int S = 1; S <= 4; S *= 2) {
+            if (S > 1 && per_level / S / wpc < 2.0) break;
+            const int64_t g = std::max<int64_t>(resident / S * S, S);
+            const double cost = (double)((R.n_sw * S + g - 1) / g) / S;
+            if (cost < best - 1e-9) { best = cost; split = S; }
+        }
+        if (const char* e = getenv("AVFS_SPLIT")) split = std::max(1, std::min(4, atoi(e)));
+    }
+    R.split = split;
+    if (persistent && split > 1) {
+        const int64_t items = R.n_sw * split;
+        R.grid = (int32_t)std::min<int64_t>(items, std::max<int64_t>(resident / split * split, split));
+    } else {
+        R.grid = (int32_t)(persistent ? std::min<int64_t>((R.n_sw + grp - 1) / grp, resident) : resident);
+    }
     if (R.grid < 1) R.grid = 1;
     if ((int)ctx->arena.size() <= round_idx) ctx->arena.resize(round_idx + 1);
     const int64_t n_buf = (int64_t)ctx->n_pi + ctx->n_pinned + ctx->n_scratch;
@@ -888,6 +910,12 @@ static avfs_status run_round(avfs_ctx* ctx, Round& R, int round_idx, const int32
     p.region_bytes = R.region_bytes;
     p.W = R.W;
     p.grp_per_cta = R.grp;
+    p.split = R.split;
+    if (R.split > 1) {
+        CK(ctx->d_lvlsync.ensure((size_t)R.n_sw * 4));
+        CK(cudaMemsetAsync(ctx->d_lvlsync.p, 0, (size_t)R.n_sw * 4, ctx->stream));
+        p.lvl_sync = ctx->d_lvlsync.as<unsigned int>();
+    }
     p.n_pi = ctx->n_pi;
     p.spill = ctx->spill[round_idx].as<float>();
     p.spill_top = ctx->d_spill_top.as<unsigned long long>() + round_idx;

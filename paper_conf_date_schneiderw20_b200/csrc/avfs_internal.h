@@ -93,6 +93,8 @@ struct SweepParams {
     int64_t region_bytes;
     int32_t W;                              // event capacity per region (32*C)
     int32_t grp_per_cta;                    // slot groups a sweep CTA walks at once (power of 2)
+    int32_t split;                          // sweep CTAs sharing one slot group (grp_per_cta == 1)
+    unsigned int* lvl_sync;                 // [n_sw] level counters of split groups (zeroed per round)
     int32_t n_pi;                           // gate index = output signal - n_pi
     // spill heap of the round: regions whose inputs carry more than W events
     // store their events here (bump allocation in words, 16-B granules)

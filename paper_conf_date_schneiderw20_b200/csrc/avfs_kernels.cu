@@ -623,6 +623,154 @@ __global__ void __launch_bounds__(AVFS_SWEEP_THREADS, AVFS_SWEEP_MINB) sweep_ker
     }
 }
 
+// The same sweep with each slot group shared by S = p.split co-resident CTAs
+// (consecutive blocks; the grid is a multiple of S): CTA part s takes the
+// s-th 1/S slice of every level, and the S parts meet at a level barrier
+// made of an L2 counter per group.  Chosen when few slot groups would leave
+// the last wave of CTAs mostly empty.  (A separate kernel: folding it into
+// the one above changed that kernel's scheduling enough to cost 7 % on
+// config 2.)
+template <bool SPLIT>
+__global__ void __launch_bounds__(AVFS_SWEEP_THREADS, AVFS_SWEEP_MINB) sweep_split_kernel(const SweepParams p) {
+    const int lane = threadIdx.x & 31;
+    const int warp = threadIdx.x >> 5;
+    const int nw = blockDim.x >> 5;
+    Env E;
+    float* ws = warp_smem(warp, WARP_SMEM_WORDS);
+    const uint32_t s_desc = smem_u32(ws + OFF_DESC), s_hdr = smem_u32(ws + OFF_HDR), s_evr = smem_u32(ws + OFF_EV);
+    uint32_t* meta = reinterpret_cast<uint32_t*>(ws + OFF_META);
+    const uint32_t s_grp = smem_u32(meta + 2);
+    E.stride = (uint32_t)(p.pin_n_sw * p.region_bytes);
+    const uint4* gd = reinterpret_cast<const uint4*>(p.gates);
+    // narrow netlists: the CTA walks G slot groups at once, nw / G warps each;
+    // few slot groups: S co-resident CTAs (consecutive blocks, grid a multiple
+    // of S) share one group, each taking 1/S of every level (G == 1 then)
+    const int G = SPLIT ? 1 : p.grp_per_cta, wpg = nw / G, S = SPLIT ? p.split : 1;
+    const int sg = warp / wpg, wl = warp % wpg;
+    const int64_t u_end = SPLIT ? p.n_sw * S : p.n_sw;
+    const int64_t u_step = SPLIT ? (int64_t)gridDim.x : (int64_t)gridDim.x * G;
+    for (int64_t u = SPLIT ? (int64_t)blockIdx.x : (int64_t)blockIdx.x * G; u < u_end; u += u_step) {
+        const int64_t i0 = SPLIT ? u / S : u;
+        const int part = SPLIT ? (int)(u % S) : 0;
+        const int64_t i = i0 + sg;
+        const bool valid = i < p.n_sw;                 // idle warps still meet every level barrier
+        slot_group(p, valid ? i : i0, lane, E);
+        __syncwarp();
+        if (lane == 0) meta[2] = (uint32_t)(p.i_base + (valid ? i : i0));
+        const float4* dt = p.dtab + (int64_t)E.kv * p.n_gates * 2;
+        for (int L = 0; L < p.depth; ++L) {
+            const int ls0 = __ldg(p.level_ptr + L), le0 = __ldg(p.level_ptr + L + 1);
+            const int P = SPLIT ? (le0 - ls0 + S - 1) / S : 0;
+            const int ls = SPLIT ? min(le0, ls0 + part * P) : ls0;
+            const int le = SPLIT ? min(le0, ls + P) : le0;
+            const int B = (le - ls + wpg - 1) / wpg;
+            const int g0 = ls + wl * B;
+            const int nj = valid ? max(0, min(B, le - g0)) : 0;
+            // descriptor window k (gates g0 + 16k ..): lane copies 16 B of the
+            // descriptors (lanes 0..31 = 16 gates x 2) and 16 B of the delays
+            auto issue_win = [&](int k) {
+                const int g = g0 + DW * k + (lane >> 1);
+                const uint32_t w = s_desc + 4 * 16 * DW * (k & 1) + 16 * lane;
+                if (g < le) {
+                    cp_async16(w, gd + 2 * g + (lane & 1));
+                    cp_async16(w + 4 * 8 * DW, dt + 2 * g + (lane & 1));
+                }
+            };
+            auto desc_at = [&](uint32_t j) { return s_desc + 4 * 16 * DW * ((j / DW) & 1) + 32 * (j % DW); };
+            auto issue_hdr = [&](uint32_t j) {
+                const uint32_t d = desc_at(j);
+                const uint32_t q = (uint32_t)lane >> 3;
+                if (q < ((lds_u32(d + 24) >> 16) & 0xffu))
+                    cp_async16(s_hdr + 512 * (j & 3) + 128 * q + 16 * (lane & 7),
+                               region(lds_u32(d + 4 * q), E) + 16 * (lane & 7));
+            };
+            // input q's events (extent = lane 31's offset + count) -> slot q of
+            // the stage (EV_STAGE / K' words, 32 / K' lanes per input, <= 2
+            // chunks of 16 B per lane); staged only if every input fits
+            bool staged_next = false, staged_cur = false;
+            auto issue_ev = [&](uint32_t j) {
+                const uint32_t d = desc_at(j);
+                const uint32_t k = (lds_u32(d + 24) >> 16) & 0xffu;
+                const uint32_t sh = k > 2 ? 2u : (k > 1 ? 1u : 0u);      // log2 K'
+                const uint32_t q = (uint32_t)lane >> (5 - sh), sub = (uint32_t)lane & (31u >> sh);
+                uint32_t c = 0, w = 0;
+                if (q < k) {
+                    w = lds_u32(s_hdr + 512 * (j & 3) + 128 * q + 124);
+                    c = (((w >> HDR_OFF_SHIFT) & HDR_OFF) + (w & HDR_N) + 3) >> 2;
+                }
+                const uint32_t cap = (uint32_t)(EV_STAGE / 4) >> sh;   // chunks per input
+                const bool staged = __all_sync(FULL, c <= cap);
+                staged_next = staged;
+                if (staged && sub < c) {
+                    const uint8_t* src = ev_base(region(lds_u32(d + 4 * q), E), w) + 16 * sub;
+                    const uint32_t dst = s_evr + 4 * EV_STAGE * (j & 1) + (4 * EV_STAGE >> sh) * q + 16 * sub;
+                    cp_async16(dst, src);
+                    const uint32_t st = 512u >> sh;                     // bytes covered by one pass of the lanes
+                    if (sub + (32u >> sh) < c) cp_async16(dst + st, src + st);
+                }
+            };
+            if (nj > 0) {
+                // prologue: descriptor windows 0, 1; header rows 0, 1; events of gate 0
+                issue_win(0);
+                if (nj > DW) issue_win(1);
+                cp_async_commit();
+                cp_async_wait_all();
+                __syncwarp();
+                issue_hdr(0);
+                if (nj > 1) issue_hdr(1);
+                cp_async_commit();
+                cp_async_wait_all();
+                __syncwarp();
+                issue_ev(0);
+                staged_cur = staged_next;
+                cp_async_commit();
+                const uint32_t nju = (uint32_t)nj;
+#pragma unroll 1
+                for (uint32_t j = 0; j < nju; ++j) {
+                    cp_async_wait_all();
+                    __syncwarp();
+                    if (j % DW == 0 && j > 0 && j + DW < nju) issue_win((int)(j / DW) + 1);
+                    if (j + 2 < nju) issue_hdr(j + 2);
+                    const bool st_j = staged_cur;
+                    if (j + 1 < nju) issue_ev(j + 1);
+                    staged_cur = staged_next;
+                    cp_async_commit();
+                    const uint32_t d = desc_at(j);
+                    const uint4* dv = reinterpret_cast<const uint4*>(ws + OFF_DESC + 16 * DW * ((j / DW) & 1) + 8 * (j % DW));
+                    Staged S;
+                    S.hdr = true;
+                    S.hdr_s = s_hdr + 512 * (j & 3);
+                    S.ev = st_j;
+                    S.dly_s = d + 4 * 8 * DW;
+                    S.grp_s = s_grp;
+                    S.ev_s[0] = s_evr + 4 * EV_STAGE * (j & 1);
+                    eval_dispatch<false>(p, E, dv[0], dv[1], S);
+                }
+            }
+            // this level's stores -> the next levels' loads; with several slot
+            // groups per CTA each group syncs only its own warps (named barrier)
+            if (G == 1 || G > 15) __syncthreads();
+            else asm volatile("bar.sync %0, %1;" ::"r"(1 + sg), "r"(32 * wpg) : "memory");
+            if (SPLIT) {                                // the other parts of this level (L2 counter)
+                if (threadIdx.x == 0) {
+                    unsigned int* ctr = p.lvl_sync + i;
+                    __threadfence();
+                    atomicAdd(ctr, 1u);
+                    const unsigned int target = (unsigned int)S * (unsigned int)(L + 1);
+                    unsigned int v;
+                    while (true) {
+                        asm volatile("ld.acquire.gpu.u32 %0, [%1];" : "=r"(v) : "l"(ctr) : "memory");
+                        if (v >= target) break;
+                        __nanosleep(64);
+                    }
+                    __threadfence();
+                }
+                __syncthreads();
+            }
+        }
+    }
+}
+
 // Level-parallel variant for overflow reruns (few slot groups): one launch per
 // level, warps take (gate, slot group) items of the level grid-wide.
 __global__ void __launch_bounds__(512, 2) level_kernel(const SweepParams p, int L) {
@@ -689,16 +837,19 @@ int sweep_smem_bytes(int warps_per_cta) { return 16 + warps_per_cta * WARP_SMEM_
 int level_smem_bytes(int warps_per_cta) { return 16 + warps_per_cta * LEVEL_SMEM_WORDS * 4; }
 
 cudaError_t sweep_occupancy(int warps_per_cta, int smem, int* blocks_per_sm) {
+    int b1 = 0, b2 = 0;
     cudaError_t e = cudaFuncSetAttribute(sweep_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
-    if (e != cudaSuccess) return e;
-    return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, sweep_kernel, warps_per_cta * 32, smem);
+    if (e == cudaSuccess) e = cudaFuncSetAttribute(sweep_split_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+    if (e == cudaSuccess) e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b1, sweep_kernel, warps_per_cta * 32, smem);
+    if (e == cudaSuccess) e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b2, sweep_split_kernel<true>, warps_per_cta * 32, smem);
+    *blocks_per_sm = b1 < b2 ? b1 : b2;      // split groups need every CTA resident
+    return e;
 }
 
 cudaError_t launch_sweep(const SweepParams& p, int grid, int warps_per_cta, cudaStream_t st) {
     const int smem = sweep_smem_bytes(warps_per_cta);
-    cudaError_t e = cudaFuncSetAttribute(sweep_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
-    if (e != cudaSuccess) return e;
-    sweep_kernel<<<grid, warps_per_cta * 32, smem, st>>>(p);
+    if (p.split > 1) sweep_split_kernel<true><<<grid, warps_per_cta * 32, smem, st>>>(p);
+    else sweep_kernel<<<grid, warps_per_cta * 32, smem, st>>>(p);
     return cudaGetLastError();
 }
 

@@ -273,3 +273,19 @@ def test_groups_per_cta_invariance(monkeypatch):
     for o in out[1:]:
         for a, b in zip(out[0], o):
             assert np.array_equal(a, b)
+
+
+def test_split_groups_invariance(monkeypatch):
+    """Few slot groups: S co-resident CTAs share one group (each a 1/S slice of
+    every level, cross-CTA level barrier); results must equal S = 1."""
+    w = make_config(3, n_pairs=64, n_vdd=2, scale=0.1)
+    sig = np.arange(w.netlist.n_signals, dtype=np.int32)
+    out = []
+    for sp in ("1", "2", "4"):
+        monkeypatch.setenv("AVFS_SPLIT", sp)
+        ctx = gpu_run(w, quantum=0.0, capacity=4)
+        out.append((ctx.activity(), ctx.latest_arrival(), *ctx.waveforms(sig, 0, w.n_slots, cap=16)))
+        ctx.close()
+    for o in out[1:]:
+        for a, b in zip(out[0], o):
+            assert np.array_equal(a, b)
