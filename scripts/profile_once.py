@@ -14,11 +14,15 @@ ap.add_argument("--config", type=int, default=4)
 ap.add_argument("--capacity", type=int, default=0)
 ap.add_argument("--warps-per-cta", type=int, default=0)
 ap.add_argument("--runs", type=int, default=2)
+ap.add_argument("--shard-of", type=int, default=0)
 a = ap.parse_args()
 w = make_config(a.config)
 ctx = Context(0)
 load_workload(ctx, w.netlist, w.library, w.stimuli, w.vdd)
 ctx.set_options(capacity=a.capacity or w.capacity, warps_per_cta=a.warps_per_cta, profile=True)
+if a.shard_of > 1:
+    from paper_conf_date_schneiderw20_b200 import shard_range
+    ctx.set_slot_range(*shard_range(w.n_slots, 0, a.shard_of))
 s = torch.cuda.Stream()
 for _ in range(a.runs):
     ctx.simulate(s)
