@@ -370,7 +370,7 @@ def main():
             "e2e": e2e,
             "gpu_launches": int(stats["launches"] * args.steps),
             "clocks": ck,
-            "stats": {k: stats[k] for k in ("evals", "slot_warps", "overflow_slot_warps", "rerun_rounds", "spill_bytes",
+            "stats": {k: stats[k] for k in ("evals", "slot_warps", "overflow_slot_warps", "rerun_rounds", "spill_bytes", "batches",
                                             "grid", "warps_per_cta", "n_scratch_buffers", "n_pinned",
                                             "arena_bytes", "launches")},
             "paper_context": "P100 (CUDA 10): 1186 MEPS average at one Vdd, 310-1785x over a serial "

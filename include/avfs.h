@@ -176,6 +176,15 @@ typedef struct {
                                   previous simulate on this context asked
                                   for, within free memory); > 0 = this many
                                   bytes; < 0 = no spill heap               */
+    int64_t max_batch_slots;   /* slot batching (arena reused per batch):
+                                  0 = auto (batch only if all slot groups'
+                                  arena does not fit in device memory);
+                                  > 0 = at most this many slots (rounded
+                                  down to 32-slot groups) per batch.  With
+                                  more than one batch, activity, latest
+                                  arrival and energy cover every slot;
+                                  waveforms / final values only the last
+                                  batch's slots, and capture is refused.   */
 } avfs_options;
 avfs_status avfs_set_options(avfs_ctx *ctx, const avfs_options *opt);
 avfs_status avfs_default_options(avfs_options *opt);
@@ -263,6 +272,7 @@ typedef struct {
     double sweep_ms;             /* CUDA-event time of pass-0 sweep (profile=1) */
     int64_t spill_bytes;         /* spill-heap bytes used by the kept rounds  */
     int64_t spill_heap_bytes;    /* spill-heap bytes allocated (all rounds)   */
+    int64_t batches;             /* slot batches of the last simulate         */
 } avfs_stats;
 avfs_status avfs_get_stats(avfs_ctx *ctx, avfs_stats *st);
 

@@ -133,6 +133,8 @@ struct avfs_ctx {
     std::vector<DevBuf> arena;        // per round: [buffer][slot group][region]
     std::vector<DevBuf> spill;        // per round: spill heap (kept: readback may point into it)
     int64_t spill_hint = 0;           // heap words the last simulate asked for (all rounds)
+    int64_t spill_per_group = 0;      // largest heap words per slot group asked for so far (sizing hint)
+    int32_t n_batches = 1;            // slot batches of the last simulate (readback keeps the last)
     int32_t* h_pinned = nullptr;      // small pinned host buffer (count, err)
     cudaEvent_t ev0 = nullptr, ev1 = nullptr;
 
@@ -1013,9 +1015,57 @@ avfs_status avfs_simulate(avfs_ctx* ctx, void* cuda_stream) {
     // their memory back so that pass 0 can size its heap from the hint
     for (size_t r = 1; r < ctx->arena.size(); ++r) ctx->arena[r].release();
     for (size_t r = 1; r < ctx->spill.size(); ++r) ctx->spill[r].release();
+    // slot batching: when the arena for every slot group would not
+    // fit, the groups run in batches on the same arena and heap; activity,
+    // latest arrival and energy accumulate over all batches, waveform readback
+    // keeps the last batch
+    const int64_t n_sw_all = sw_hi - sw_lo;
+    const int64_t region0 = 128 + 4 * (int64_t)(32 * ctx->opt.capacity);
+    const int64_t per_group = ((int64_t)ctx->n_pi + ctx->n_pinned + ctx->n_scratch) * region0;
+    // device bytes one group needs: its arena share plus its expected spill
+    // (learned from earlier batches / simulates, words per group)
+    auto group_bytes = [&]() { return (double)per_group + 1.25 * 4.0 * (double)ctx->spill_per_group; };
+    auto avail_bytes = [&]() -> double {
+        size_t fr = 0, tot = 0;
+        if (cudaMemGetInfo(&fr, &tot) != cudaSuccess) return 0.0;
+        double own = 0;
+        for (auto& a : ctx->arena) own += (double)a.n;
+        for (auto& h : ctx->spill) own += (double)h.n;
+        return (double)fr + own - (double)(2ll << 30);
+    };
+    int64_t nb = n_sw_all;
+    bool learn = false;                                 // first batch only one wave: learn the spill per group
+    if (ctx->opt.max_batch_slots > 0) {
+        nb = std::max<int64_t>(1, ctx->opt.max_batch_slots / 32);
+    } else if (!ctx->arena.empty() && ctx->arena[0].n >= (size_t)(n_sw_all * per_group) &&
+               ctx->spill_per_group * n_sw_all * 5 / 4 <= (int64_t)(ctx->spill.empty() ? 0 : ctx->spill[0].n / 4)) {
+        nb = n_sw_all;                                  // fits the arena and heap of a previous simulate
+    } else {
+        const int64_t fit = (int64_t)(0.8 * avail_bytes() / std::max(group_bytes(), 1.0));
+        if (fit < n_sw_all) {
+            nb = std::max<int64_t>(1, fit);
+            if (ctx->spill_per_group == 0) { nb = std::min<int64_t>(nb, (int64_t)ctx->n_sm); learn = true; }
+        }
+    }
+    nb = std::min(nb, n_sw_all);
+    ctx->n_batches = 0;
+    double sweep_ms_sum = 0;
+    int64_t hint = 0;
+    for (int64_t b0 = sw_lo; b0 < sw_hi; b0 += nb) {
+    if (b0 > sw_lo) {                                   // earlier batches' rerun memory is not kept
+        for (size_t r = 1; r < ctx->arena.size(); ++r) ctx->arena[r].release();
+        for (size_t r = 1; r < ctx->spill.size(); ++r) ctx->spill[r].release();
+        if (learn && ctx->opt.max_batch_slots <= 0) {   // resize the remaining batches
+            const int64_t fit = (int64_t)(0.8 * avail_bytes() / std::max(group_bytes(), 1.0));
+            nb = std::max<int64_t>(1, std::min(fit, sw_hi - b0));
+            learn = false;
+        }
+    }
+    ctx->n_batches++;
+    ctx->rounds.clear();
     Round R0;
-    R0.n_sw = sw_hi - sw_lo;
-    R0.sw_first = sw_lo;
+    R0.n_sw = std::min(nb, sw_hi - b0);
+    R0.sw_first = b0;
     R0.capacity = ctx->opt.capacity;
     R0.W = 32 * R0.capacity;
     R0.region_bytes = 128 + 4 * (int64_t)R0.W;
@@ -1025,10 +1075,12 @@ avfs_status avfs_simulate(avfs_ctx* ctx, void* cuda_stream) {
         // for in all its rounds, so that repeated runs do not rerun
         R0.spill_want = ctx->opt.spill_bytes > 0 ? ctx->opt.spill_bytes / 4
                       : ctx->opt.spill_bytes < 0 ? 0
-                      : std::max<int64_t>({arena_words / 4, (256ll << 20) / 4, ctx->spill_hint + ctx->spill_hint / 4});
+                      : std::max<int64_t>({arena_words / 4, (256ll << 20) / 4,
+                                           ctx->spill_per_group * R0.n_sw + ctx->spill_per_group * R0.n_sw / 4});
     }
     st = run_round(ctx, R0, 0, nullptr, nullptr, ctx->opt.profile != 0);
     if (st != AVFS_OK) return st;
+    const int64_t R0n = std::max<int64_t>(R0.n_sw, 1);
     ctx->rounds.push_back(R0);
     int cur = 0;
     for (int r = 0;; ++r) {
@@ -1085,18 +1137,23 @@ avfs_status avfs_simulate(avfs_ctx* ctx, void* cuda_stream) {
     {
         int64_t req = 0;
         for (const Round& R : ctx->rounds) req += R.spill_req;
-        ctx->spill_hint = req;
+        hint = std::max(hint, req);
+        ctx->spill_per_group = std::max<int64_t>(ctx->spill_per_group, (req + R0n - 1) / R0n);
     }
     if (ctx->opt.profile) {
         float ms = 0;
         CK(cudaEventElapsedTime(&ms, ctx->ev0, ctx->ev1));
-        ctx->stats.sweep_ms = ms;
+        sweep_ms_sum += ms;
     }
+    }  // batches
+    ctx->spill_hint = hint;
+    if (ctx->opt.profile) ctx->stats.sweep_ms = sweep_ms_sum;
     ctx->sim_done = true;
     ctx->stats.slots = end - first;
     ctx->stats.evals = (int64_t)ctx->n_gates * (end - first);
     ctx->stats.slot_warps = sw_hi - sw_lo;
     ctx->stats.grid = ctx->rounds[0].grid;
+    ctx->stats.batches = ctx->n_batches;
     ctx->stats.n_scratch_buffers = ctx->n_scratch;
     ctx->stats.n_pinned = ctx->n_pinned;
     int64_t ab = 0;
@@ -1205,6 +1262,9 @@ static avfs_status gather(avfs_ctx* ctx, int32_t n_sig, const int32_t* sig, int6
     if (count) CK(cudaMemcpyAsync(count, ctx->g_count.p, n * 4, cudaMemcpyDeviceToHost, ctx->stream));
     if (times && cap > 0) CK(cudaMemcpyAsync(times, ctx->g_times.p, n * cap * 4, cudaMemcpyDeviceToHost, ctx->stream));
     CK(cudaStreamSynchronize(ctx->stream));
+    if (bad && ctx->n_batches > 1)
+        return fail(ctx, AVFS_ERR_STATE, "waveforms of slots outside the last of %d batches are not retained "
+                    "(raise max_batch_slots or restrict the slot range)", ctx->n_batches);
     if (bad) return fail(ctx, AVFS_ERR_STATE, "readback hit slots without valid data (code %d)", bad);
     return AVFS_OK;
 }
@@ -1236,6 +1296,9 @@ avfs_status avfs_capture(avfs_ctx* ctx, const float* t_clk, int32_t n_bins, floa
     if (!t_clk || !fail_pairs) return fail(ctx, AVFS_ERR_ARG, "null t_clk / fail_pairs");
     if (slack_hist && (n_bins < 1 || !(width_ps > 0))) return fail(ctx, AVFS_ERR_ARG, "bad histogram bins");
     if (ctx->rounds.size() > 8) return fail(ctx, AVFS_ERR_STATE, "too many rounds");
+    if (ctx->n_batches > 1)
+        return fail(ctx, AVFS_ERR_STATE, "capture needs every slot's PO waveforms; the last simulate ran in %d batches "
+                    "(raise max_batch_slots or restrict the slot range)", ctx->n_batches);
     avfs_status ms = ensure_round_map(ctx);
     if (ms != AVFS_OK) return ms;
     const int32_t V = (int32_t)ctx->vdd.size();

@@ -16,14 +16,14 @@ REL, ABS = 1e-5, 1e-3
 
 
 def gpu_run(w_or_parts, quantum=0.0, capacity=None, keep_all=True, probes=None, slot_range=None,
-            stream=None, warps_per_cta=0, max_rerun_rounds=3, netlist=None, spill_bytes=0):
+            stream=None, warps_per_cta=0, max_rerun_rounds=3, netlist=None, spill_bytes=0, max_batch_slots=0):
     from paper_conf_date_schneiderw20_b200 import Context, load_workload
     nl = netlist if netlist is not None else w_or_parts.netlist
     ctx = Context(0)
     load_workload(ctx, nl, w_or_parts.library, w_or_parts.stimuli, w_or_parts.vdd)
     ctx.set_options(capacity=capacity or w_or_parts.capacity, quantum_ps=quantum, keep_all=keep_all,
                     probes=probes, warps_per_cta=warps_per_cta, max_rerun_rounds=max_rerun_rounds,
-                    spill_bytes=spill_bytes,
+                    spill_bytes=spill_bytes, max_batch_slots=max_batch_slots,
                     profile=True)
     if slot_range is not None:
         ctx.set_slot_range(*slot_range)

@@ -289,3 +289,32 @@ def test_split_groups_invariance(monkeypatch):
     for o in out[1:]:
         for a, b in zip(out[0], o):
             assert np.array_equal(a, b)
+
+
+@pytest.mark.parametrize("quantum", [Q, 0.0])
+def test_slot_batching(quantum):
+    """SURVEY H5 batching: slot groups run in batches on one reused arena.
+    Activity and latest arrival equal the unbatched run (and the oracle);
+    the last batch's waveforms are kept, earlier ones are refused, as is capture."""
+    from paper_conf_date_schneiderw20_b200 import AvfsError
+    w = make_config(3, n_pairs=96, n_vdd=3, scale=0.05)
+    sig = np.arange(w.netlist.n_signals, dtype=np.int32)
+    a = gpu_run(w, quantum=quantum, capacity=4)
+    b = gpu_run(w, quantum=quantum, capacity=4, max_batch_slots=64)      # 2 groups per batch
+    assert b.stats()["batches"] == 5 and a.stats()["batches"] == 1
+    assert np.array_equal(a.activity(), b.activity())
+    assert np.array_equal(a.latest_arrival(), b.latest_arrival())
+    last = w.n_slots - 32                                              # slots of the last group (pairs 64..95, Vdd 2)
+    wa, wb = a.waveforms(sig, last, 32, cap=16), b.waveforms(sig, last, 32, cap=16)
+    for x, y in zip(wa, wb):
+        assert np.array_equal(x, y)
+    with pytest.raises(AvfsError):
+        b.waveforms(sig, 0, 32, cap=16)
+    with pytest.raises(AvfsError):
+        b.capture(np.full(3, 100.0, np.float32))
+    j, k = oracle.all_slots(w.stimuli.n_pairs, len(w.vdd))
+    ref = oracle.simulate(w.netlist, w.library, w.stimuli, w.vdd, j, k, quantum=quantum, cap=0)
+    ra, ok = activity_ref(ref, len(w.vdd), w.netlist.n_signals)
+    assert np.array_equal(b.activity().astype(np.int64)[ok], ra[ok])
+    a.close()
+    b.close()
