@@ -30,6 +30,9 @@
 
 #include "avfs_internal.h"
 
+#ifndef AVFS_PRUNE
+#define AVFS_PRUNE 1          // drop input events the gate cannot observe in that slot
+#endif
 #ifndef AVFS_PTX_MERGE
 #define AVFS_PTX_MERGE 1      // 2-input staged merge as one PTX loop (0: the C++ loop)
 #endif
@@ -368,14 +371,31 @@ __device__ __forceinline__ void eval_gate(const SweepParams& p, const Env& E, co
                       : __ldcg(reinterpret_cast<const uint32_t*>(region(in_loc[q], E)) + lane);
     int n[KMAX] = {0, 0, 0, 0};
     uint32_t bits = 0, orh = 0;
-    int m = 0;
 #pragma unroll
     for (int q = 0; q < K; ++q) {
         n[q] = (int)(hw[q] & HDR_N);
         bits |= ((hw[q] >> HDR_INIT_SHIFT) & 1u) << q;
         orh |= hw[q];
-        m += n[q];
     }
+    if (K >= 2 && AVFS_PRUNE) {
+        // Events this slot's output cannot observe: with the stable inputs
+        // (no event) at their values, the truth table restricted to the
+        // remaining minterms does not depend on input q (e.g. AND with another
+        // input stable at 0).  Such events never change the evaluated output
+        // (reading C4), so they are dropped from the merge -- fewer merge
+        // steps and tighter output offsets, identical waveforms.
+        constexpr uint32_t POS[4] = {0xAAAAu, 0xCCCCu, 0xF0F0u, 0xFF00u};
+        uint32_t mt = 0xFFFFu >> (16 - (1 << K));       // minterms consistent with the stable inputs
+#pragma unroll
+        for (int q = 0; q < K; ++q)
+            if (n[q] == 0) mt &= ((bits >> q) & 1u) ? POS[q] : ~POS[q];
+#pragma unroll
+        for (int q = 0; q < K; ++q)
+            if ((((tt >> (1 << q)) ^ tt) & mt & ~POS[q]) == 0) n[q] = 0;
+    }
+    int m = 0;
+#pragma unroll
+    for (int q = 0; q < K; ++q) m += n[q];
     const uint32_t y0 = (tt >> bits) & 1u;
     uint8_t* ro = region(out_loc, E);
     uint32_t* ro_hdr = reinterpret_cast<uint32_t*>(ro);
