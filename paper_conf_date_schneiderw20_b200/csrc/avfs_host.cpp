@@ -347,6 +347,24 @@ avfs_status upload_netlist(avfs_ctx* ctx) {
         d.sig = (uint32_t)(ctx->n_pi + g);
         d.ttk = (uint32_t)ctx->cell_tt[ctx->gate_cell[g]] | ((uint32_t)k << 16) |
                 ((ctx->is_po[ctx->n_pi + g] ? 1u : 0u) << 24);
+        // 2-input gates: observability table for the event pruning of the
+        // sweep -- entry (stable-input mask s | their values << 2) holds, per
+        // input with events, whether the truth table restricted to the stable
+        // inputs' values depends on it
+        if (k == 2) {
+            const uint32_t tt = ctx->cell_tt[ctx->gate_cell[g]];
+            for (uint32_t idx = 0; idx < 16; ++idx) {
+                const uint32_t st = idx & 3u, val = (idx >> 2) & st;
+                uint32_t obs = 0;
+                for (uint32_t q = 0; q < 2; ++q) {
+                    if (st & (1u << q)) continue;
+                    for (uint32_t b = 0; b < 4; ++b)
+                        if (!(b & (1u << q)) && (b & st) == val && ((tt >> b) & 1u) != ((tt >> (b | (1u << q))) & 1u))
+                            obs |= 1u << q;
+                }
+                d.obs |= obs << (2 * idx);
+            }
+        }
         e.coef_off = ctx->coef_off[g];
         e.k = (uint32_t)k;
         e.island = (uint32_t)ctx->island[g];

@@ -40,7 +40,7 @@ struct alignas(16) GateDesc {
     uint32_t out_loc;
     uint32_t sig;        // output signal id (activity row)
     uint32_t ttk;        // bits 0..15 truth table, 16..23 #inputs, 24..31 flags (bit 24: PO)
-    uint32_t pad;
+    uint32_t obs;        // 2-input gates: observability table (2 bits per stable-input pattern)
 };
 static_assert(sizeof(GateDesc) == 32, "GateDesc layout");
 

@@ -377,7 +377,12 @@ __device__ __forceinline__ void eval_gate(const SweepParams& p, const Env& E, co
         bits |= ((hw[q] >> HDR_INIT_SHIFT) & 1u) << q;
         orh |= hw[q];
     }
-    if (K >= 2 && AVFS_PRUNE) {
+    if (K == 2 && AVFS_PRUNE) {                          // table lookup (host-built, GateDesc.obs)
+        const uint32_t st = (n[0] == 0 ? 1u : 0u) | (n[1] == 0 ? 2u : 0u);
+        const uint32_t ob = hd.w >> (2 * (st | ((bits & st) << 2)));
+        n[0] = (ob & 1u) ? n[0] : 0;
+        n[1] = (ob & 2u) ? n[1] : 0;
+    } else if (K >= 3 && AVFS_PRUNE) {
         // Events this slot's output cannot observe: with the stable inputs
         // (no event) at their values, the truth table restricted to the
         // remaining minterms does not depend on input q (e.g. AND with another
