@@ -561,15 +561,16 @@ __global__ void __launch_bounds__(AVFS_SWEEP_THREADS, AVFS_SWEEP_MINB) sweep_ker
             const int nj = valid ? max(0, min(B, le - g0)) : 0;
             // descriptor window k (gates g0 + 16k ..): lane copies 16 B of the
             // descriptors (lanes 0..31 = 16 gates x 2) and 16 B of the delays
+            // descriptor ring of 2 DW gates (32 B each), delay ring behind it
             auto issue_win = [&](int k) {
                 const int g = g0 + DW * k + (lane >> 1);
-                const uint32_t w = s_desc + 4 * 16 * DW * (k & 1) + 16 * lane;
+                const uint32_t w = s_desc + 32 * ((uint32_t)(DW * k + (lane >> 1)) & (2 * DW - 1)) + 16 * (lane & 1);
                 if (g < le) {
                     cp_async16(w, gd + 2 * g + (lane & 1));
-                    cp_async16(w + 4 * 8 * DW, dt + 2 * g + (lane & 1));
+                    cp_async16(w + 32 * 2 * DW, dt + 2 * g + (lane & 1));
                 }
             };
-            auto desc_at = [&](uint32_t j) { return s_desc + 4 * 16 * DW * ((j / DW) & 1) + 32 * (j % DW); };
+            auto desc_at = [&](uint32_t j) { return s_desc + 32 * (j & (2 * DW - 1)); };
             auto issue_hdr = [&](uint32_t j) {
                 const uint32_t d = desc_at(j);
                 const uint32_t q = (uint32_t)lane >> 3;
@@ -629,12 +630,12 @@ __global__ void __launch_bounds__(AVFS_SWEEP_THREADS, AVFS_SWEEP_MINB) sweep_ker
                     staged_cur = staged_next;
                     cp_async_commit();
                     const uint32_t d = desc_at(j);
-                    const uint4* dv = reinterpret_cast<const uint4*>(ws + OFF_DESC + 16 * DW * ((j / DW) & 1) + 8 * (j % DW));
+                    const uint4* dv = reinterpret_cast<const uint4*>(ws + OFF_DESC + 8 * (j & (2 * DW - 1)));
                     Staged S;
                     S.hdr = true;
                     S.hdr_s = s_hdr + 512 * (j & 3);
                     S.ev = st_j;
-                    S.dly_s = d + 4 * 8 * DW;
+                    S.dly_s = d + 32 * 2 * DW;
                     S.grp_s = s_grp;
                     S.ev_s[0] = s_evr + 4 * EV_STAGE * (j & 1);
                     eval_dispatch<false>(p, E, dv[0], dv[1], S);
@@ -693,15 +694,16 @@ __global__ void __launch_bounds__(AVFS_SWEEP_THREADS, AVFS_SWEEP_MINB) sweep_spl
             const int nj = valid ? max(0, min(B, le - g0)) : 0;
             // descriptor window k (gates g0 + 16k ..): lane copies 16 B of the
             // descriptors (lanes 0..31 = 16 gates x 2) and 16 B of the delays
+            // descriptor ring of 2 DW gates (32 B each), delay ring behind it
             auto issue_win = [&](int k) {
                 const int g = g0 + DW * k + (lane >> 1);
-                const uint32_t w = s_desc + 4 * 16 * DW * (k & 1) + 16 * lane;
+                const uint32_t w = s_desc + 32 * ((uint32_t)(DW * k + (lane >> 1)) & (2 * DW - 1)) + 16 * (lane & 1);
                 if (g < le) {
                     cp_async16(w, gd + 2 * g + (lane & 1));
-                    cp_async16(w + 4 * 8 * DW, dt + 2 * g + (lane & 1));
+                    cp_async16(w + 32 * 2 * DW, dt + 2 * g + (lane & 1));
                 }
             };
-            auto desc_at = [&](uint32_t j) { return s_desc + 4 * 16 * DW * ((j / DW) & 1) + 32 * (j % DW); };
+            auto desc_at = [&](uint32_t j) { return s_desc + 32 * (j & (2 * DW - 1)); };
             auto issue_hdr = [&](uint32_t j) {
                 const uint32_t d = desc_at(j);
                 const uint32_t q = (uint32_t)lane >> 3;
@@ -761,12 +763,12 @@ __global__ void __launch_bounds__(AVFS_SWEEP_THREADS, AVFS_SWEEP_MINB) sweep_spl
                     staged_cur = staged_next;
                     cp_async_commit();
                     const uint32_t d = desc_at(j);
-                    const uint4* dv = reinterpret_cast<const uint4*>(ws + OFF_DESC + 16 * DW * ((j / DW) & 1) + 8 * (j % DW));
+                    const uint4* dv = reinterpret_cast<const uint4*>(ws + OFF_DESC + 8 * (j & (2 * DW - 1)));
                     Staged S;
                     S.hdr = true;
                     S.hdr_s = s_hdr + 512 * (j & 3);
                     S.ev = st_j;
-                    S.dly_s = d + 4 * 8 * DW;
+                    S.dly_s = d + 32 * 2 * DW;
                     S.grp_s = s_grp;
                     S.ev_s[0] = s_evr + 4 * EV_STAGE * (j & 1);
                     eval_dispatch<false>(p, E, dv[0], dv[1], S);
