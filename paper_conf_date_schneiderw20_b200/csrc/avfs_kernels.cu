@@ -143,6 +143,14 @@ struct Staged {
     uint32_t dly_s;       // shared address of the gate's 8 delays [pin][pol]
     uint32_t grp_s;       // shared address of the slot group's index in the round (u32; read when poisoning)
 };
+__device__ __forceinline__ uint4 lds_u32x4(uint32_t a) {
+    uint4 v;
+    asm volatile("ld.shared.v4.u32 {%0, %1, %2, %3}, [%4];" : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "r"(a));
+    return v;
+}
+__device__ __forceinline__ void sts_u32(uint32_t a, uint32_t v) {
+    asm volatile("st.shared.u32 [%0], %1;" ::"r"(a), "r"(v) : "memory");
+}
 __device__ __forceinline__ float4 lds_f32x4(uint32_t a) {
     float4 v;
     asm volatile("ld.shared.v4.f32 {%0, %1, %2, %3}, [%4];" : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w) : "r"(a));
@@ -538,10 +546,10 @@ __global__ void __launch_bounds__(AVFS_SWEEP_THREADS, AVFS_SWEEP_MINB) sweep_ker
     const int warp = threadIdx.x >> 5;
     const int nw = blockDim.x >> 5;
     Env E;
-    float* ws = warp_smem(warp, WARP_SMEM_WORDS);
-    const uint32_t s_desc = smem_u32(ws + OFF_DESC), s_hdr = smem_u32(ws + OFF_HDR), s_evr = smem_u32(ws + OFF_EV);
-    uint32_t* meta = reinterpret_cast<uint32_t*>(ws + OFF_META);
-    const uint32_t s_grp = smem_u32(meta + 2);
+    // shared addresses only (no generic pointers into the warp's area)
+    const uint32_t ws_s = smem_u32(warp_smem(0, 0)) + 4u * (uint32_t)(warp * WARP_SMEM_WORDS);
+    const uint32_t s_desc = ws_s + 4 * OFF_DESC, s_hdr = ws_s + 4 * OFF_HDR, s_evr = ws_s + 4 * OFF_EV;
+    const uint32_t s_grp = ws_s + 4 * (OFF_META + 2);
     E.stride = (uint32_t)(p.pin_n_sw * p.region_bytes);
     const uint4* gd = reinterpret_cast<const uint4*>(p.gates);
     // narrow netlists: the CTA walks G slot groups at once, nw / G warps each
@@ -552,7 +560,7 @@ __global__ void __launch_bounds__(AVFS_SWEEP_THREADS, AVFS_SWEEP_MINB) sweep_ker
         const bool valid = i < p.n_sw;                 // idle warps still meet every level barrier
         slot_group(p, valid ? i : i0, lane, E);
         __syncwarp();
-        if (lane == 0) meta[2] = (uint32_t)(p.i_base + (valid ? i : i0));
+        if (lane == 0) sts_u32(s_grp, (uint32_t)(p.i_base + (valid ? i : i0)));
         const float4* dt = p.dtab + (int64_t)E.kv * p.n_gates * 2;
         for (int L = 0; L < p.depth; ++L) {
             const int ls = __ldg(p.level_ptr + L), le = __ldg(p.level_ptr + L + 1);
@@ -630,7 +638,7 @@ __global__ void __launch_bounds__(AVFS_SWEEP_THREADS, AVFS_SWEEP_MINB) sweep_ker
                     staged_cur = staged_next;
                     cp_async_commit();
                     const uint32_t d = desc_at(j);
-                    const uint4* dv = reinterpret_cast<const uint4*>(ws + OFF_DESC + 8 * (j & (2 * DW - 1)));
+                    const uint4 dv0 = lds_u32x4(d), dv1 = lds_u32x4(d + 16);
                     Staged S;
                     S.hdr = true;
                     S.hdr_s = s_hdr + 512 * (j & 3);
@@ -638,7 +646,7 @@ __global__ void __launch_bounds__(AVFS_SWEEP_THREADS, AVFS_SWEEP_MINB) sweep_ker
                     S.dly_s = d + 32 * 2 * DW;
                     S.grp_s = s_grp;
                     S.ev_s[0] = s_evr + 4 * EV_STAGE * (j & 1);
-                    eval_dispatch<false>(p, E, dv[0], dv[1], S);
+                    eval_dispatch<false>(p, E, dv0, dv1, S);
                 }
             }
             // this level's stores -> the next levels' loads; with several slot
@@ -662,10 +670,10 @@ __global__ void __launch_bounds__(AVFS_SWEEP_THREADS, AVFS_SWEEP_MINB) sweep_spl
     const int warp = threadIdx.x >> 5;
     const int nw = blockDim.x >> 5;
     Env E;
-    float* ws = warp_smem(warp, WARP_SMEM_WORDS);
-    const uint32_t s_desc = smem_u32(ws + OFF_DESC), s_hdr = smem_u32(ws + OFF_HDR), s_evr = smem_u32(ws + OFF_EV);
-    uint32_t* meta = reinterpret_cast<uint32_t*>(ws + OFF_META);
-    const uint32_t s_grp = smem_u32(meta + 2);
+    // shared addresses only (no generic pointers into the warp's area)
+    const uint32_t ws_s = smem_u32(warp_smem(0, 0)) + 4u * (uint32_t)(warp * WARP_SMEM_WORDS);
+    const uint32_t s_desc = ws_s + 4 * OFF_DESC, s_hdr = ws_s + 4 * OFF_HDR, s_evr = ws_s + 4 * OFF_EV;
+    const uint32_t s_grp = ws_s + 4 * (OFF_META + 2);
     E.stride = (uint32_t)(p.pin_n_sw * p.region_bytes);
     const uint4* gd = reinterpret_cast<const uint4*>(p.gates);
     // narrow netlists: the CTA walks G slot groups at once, nw / G warps each;
@@ -682,7 +690,7 @@ __global__ void __launch_bounds__(AVFS_SWEEP_THREADS, AVFS_SWEEP_MINB) sweep_spl
         const bool valid = i < p.n_sw;                 // idle warps still meet every level barrier
         slot_group(p, valid ? i : i0, lane, E);
         __syncwarp();
-        if (lane == 0) meta[2] = (uint32_t)(p.i_base + (valid ? i : i0));
+        if (lane == 0) sts_u32(s_grp, (uint32_t)(p.i_base + (valid ? i : i0)));
         const float4* dt = p.dtab + (int64_t)E.kv * p.n_gates * 2;
         for (int L = 0; L < p.depth; ++L) {
             const int ls0 = __ldg(p.level_ptr + L), le0 = __ldg(p.level_ptr + L + 1);
@@ -763,7 +771,7 @@ __global__ void __launch_bounds__(AVFS_SWEEP_THREADS, AVFS_SWEEP_MINB) sweep_spl
                     staged_cur = staged_next;
                     cp_async_commit();
                     const uint32_t d = desc_at(j);
-                    const uint4* dv = reinterpret_cast<const uint4*>(ws + OFF_DESC + 8 * (j & (2 * DW - 1)));
+                    const uint4 dv0 = lds_u32x4(d), dv1 = lds_u32x4(d + 16);
                     Staged S;
                     S.hdr = true;
                     S.hdr_s = s_hdr + 512 * (j & 3);
@@ -771,7 +779,7 @@ __global__ void __launch_bounds__(AVFS_SWEEP_THREADS, AVFS_SWEEP_MINB) sweep_spl
                     S.dly_s = d + 32 * 2 * DW;
                     S.grp_s = s_grp;
                     S.ev_s[0] = s_evr + 4 * EV_STAGE * (j & 1);
-                    eval_dispatch<false>(p, E, dv[0], dv[1], S);
+                    eval_dispatch<false>(p, E, dv0, dv1, S);
                 }
             }
             // this level's stores -> the next levels' loads; with several slot
