@@ -883,8 +883,15 @@ cudaError_t sweep_occupancy(int warps_per_cta, int smem, int* blocks_per_sm) {
 
 cudaError_t launch_sweep(const SweepParams& p, int grid, int warps_per_cta, cudaStream_t st) {
     const int smem = sweep_smem_bytes(warps_per_cta);
-    if (p.split > 1) sweep_split_kernel<true><<<grid, warps_per_cta * 32, smem, st>>>(p);
-    else sweep_kernel<<<grid, warps_per_cta * 32, smem, st>>>(p);
+    if (p.split > 1) {
+        // the parts of a slot group wait for each other: a cooperative launch
+        // guarantees that every CTA of the grid is resident (or fails)
+        SweepParams q = p;
+        void* args[] = {&q};
+        return cudaLaunchCooperativeKernel(reinterpret_cast<const void*>(sweep_split_kernel<true>), dim3(grid),
+                                           dim3(warps_per_cta * 32), args, (size_t)smem, st);
+    }
+    sweep_kernel<<<grid, warps_per_cta * 32, smem, st>>>(p);
     return cudaGetLastError();
 }
 
