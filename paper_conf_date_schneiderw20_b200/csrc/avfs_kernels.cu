@@ -500,12 +500,13 @@ __device__ __forceinline__ void eval_gate(const SweepParams& p, const Env& E, co
 template <bool RERUN>
 __device__ __forceinline__ void eval_dispatch(const SweepParams& p, const Env& E, const uint4 ins, const uint4 hd,
                                               const Staged& S) {
-    switch ((hd.z >> 16) & 0xffu) {
-        case 1: eval_gate<1, RERUN>(p, E, ins, hd, S); break;
-        case 2: eval_gate<2, RERUN>(p, E, ins, hd, S); break;
-        case 3: eval_gate<3, RERUN>(p, E, ins, hd, S); break;
-        default: eval_gate<4, RERUN>(p, E, ins, hd, S); break;
-    }
+    // compare chain in order of frequency (2-input cells first) instead of a
+    // jump table
+    const uint32_t k = (hd.z >> 16) & 0xffu;
+    if (k == 2) eval_gate<2, RERUN>(p, E, ins, hd, S);
+    else if (k == 1) eval_gate<1, RERUN>(p, E, ins, hd, S);
+    else if (k == 3) eval_gate<3, RERUN>(p, E, ins, hd, S);
+    else eval_gate<4, RERUN>(p, E, ins, hd, S);
 }
 
 __device__ __forceinline__ void slot_group(const SweepParams& p, int64_t i, int lane, Env& E) {
