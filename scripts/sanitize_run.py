@@ -19,3 +19,18 @@ for cfg, kw in ((1, dict(n_pairs=64)), (2, dict(n_pairs=64, n_vdd=2)), (3, dict(
         st = ctx.stats()
         print(cfg, cap, spill, int(a.sum()), st["rerun_rounds"], st["spill_bytes"], flush=True)
         ctx.close()
+
+# work-distribution variants: G slot groups per CTA (named barriers), S CTAs per group
+w = make_config(3, n_pairs=96, n_vdd=2, scale=0.05)
+for env in ({"AVFS_GROUPS_PER_CTA": "4"}, {"AVFS_SPLIT": "2"}):
+    os.environ.pop("AVFS_GROUPS_PER_CTA", None)
+    os.environ.pop("AVFS_SPLIT", None)
+    os.environ.update(env)
+    ctx = Context(0)
+    load_workload(ctx, w.netlist, w.library, w.stimuli, w.vdd)
+    ctx.set_options(capacity=4)
+    ctx.simulate()
+    print(env, int(ctx.activity().sum()), flush=True)
+    ctx.close()
+os.environ.pop("AVFS_GROUPS_PER_CTA", None)
+os.environ.pop("AVFS_SPLIT", None)
