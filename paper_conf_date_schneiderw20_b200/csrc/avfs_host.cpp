@@ -895,7 +895,8 @@ static avfs_status run_round(avfs_ctx* ctx, Round& R, int round_idx, const int32
         CK(cudaMemGetInfo(&fr, &tot));
         const size_t have = ctx->spill[round_idx].n;
         const size_t avail = fr + have > (1ull << 30) ? fr + have - (1ull << 30) : 0;
-        size_t bytes = std::min<size_t>((size_t)R.spill_want * 4, avail) & ~(size_t)15;
+        // 25 % headroom so that slowly growing requests do not reallocate every run
+        size_t bytes = std::min<size_t>((size_t)R.spill_want * 5, avail) & ~(size_t)15;
         while (bytes >= 16 && ctx->spill[round_idx].ensure(bytes) != cudaSuccess) {
             cudaGetLastError();
             bytes = (bytes / 2) & ~(size_t)15;
