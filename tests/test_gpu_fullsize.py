@@ -34,7 +34,8 @@ def sample_slots(w, n):
 
 
 @pytest.mark.parametrize("cfg,quantum", [(2, 0.0), (3, 0.0), (4, 0.0), pytest.param(5, 0.0, marks=pytest.mark.slow),
-                                         (2, 2.0 ** -8), (4, 2.0 ** -8)])
+                                         (2, 2.0 ** -8), (3, 2.0 ** -8), (4, 2.0 ** -8),
+                                         pytest.param(5, 2.0 ** -8, marks=pytest.mark.slow)])
 def test_fullsize_sampled_po_parity(cfg, quantum):
     w = make_config(cfg)
     nl = w.netlist
