@@ -568,6 +568,8 @@ avfs_status avfs_load_netlist(avfs_ctx* ctx, int32_t n_pi, int32_t n_gates, cons
     if (st != AVFS_OK) return st;
     build_coef(ctx);
     ctx->net_loaded = true;
+    ctx->spill_per_group = 0;          // the heap sizing hint belongs to the previous netlist
+    ctx->spill_hint = 0;
     ctx->plan_valid = false;
     ctx->dev_net_valid = false;
     ctx->names.clear();
