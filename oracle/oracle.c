@@ -25,7 +25,10 @@
  *                       Pinned by T2-T10 (closed forms, brute force, a second
  *                       independent formulation in tests/).
  *
- * No function here is "parity unpinned".
+ * No function here is "parity unpinned": O6 (flags, taint) is pinned by
+ * tests/test_oracle_o6.py (windows at 0.5x / 1.5x the C13 bound for both
+ * decision kinds, the truth-table exemption, soundness against a binary32
+ * emulation of the method).
  *
  * Build: gcc -O2 -fopenmp -ffp-contract=off -shared -fPIC (see oracle/__init__.py).
  */

@@ -270,6 +270,10 @@ class Context:
         """[n_signals][n_vdd] uint64; `out` may be a torch CUDA int64/uint64 tensor
         (device copy) or a C-contiguous uint64 numpy array (e.g. pinned host memory)."""
         if out is not None and hasattr(out, "data_ptr"):
+            import torch
+            if (not out.is_cuda or out.dtype not in (torch.int64, torch.uint64)
+                    or tuple(out.shape) != (self.n_signals, self.n_vdd) or not out.is_contiguous()):
+                raise ValueError("activity out tensor must be a contiguous CUDA int64/uint64 [n_signals][n_vdd]")
             self._ck(self.lib.avfs_get_activity(self.h, C.c_void_p(out.data_ptr()), 1))
             return out
         if out is not None:

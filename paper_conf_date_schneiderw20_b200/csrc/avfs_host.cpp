@@ -510,6 +510,7 @@ avfs_status avfs_load_library(avfs_ctx* ctx, int32_t n_cells, const avfs_cell* c
     ctx->c_max = c_max_fF;
     ctx->lib_loaded = true;
     ctx->net_loaded = false;
+    ctx->stim_set = false;             // stimuli are sized by the netlist's PIs
     ctx->plan_valid = false;
     ctx->dev_net_valid = false;
     invalidate_sim(ctx);
@@ -568,6 +569,7 @@ avfs_status avfs_load_netlist(avfs_ctx* ctx, int32_t n_pi, int32_t n_gates, cons
     if (st != AVFS_OK) return st;
     build_coef(ctx);
     ctx->net_loaded = true;
+    ctx->stim_set = false;             // stimuli were packed for the previous netlist's PIs
     ctx->spill_per_group = 0;          // the heap sizing hint belongs to the previous netlist
     ctx->spill_hint = 0;
     ctx->plan_valid = false;

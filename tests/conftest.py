@@ -18,3 +18,20 @@ def oracle_mod():
     import oracle
     oracle.build()
     return oracle
+
+
+def pytest_terminal_summary(terminalreporter):
+    """Every parity comparison's taint counts (reading C13) in the log: tainted
+    pairs are compared and reported, never silently excluded."""
+    try:
+        from tests.parity import REPORT
+    except Exception:
+        return
+    if not REPORT:
+        return
+    terminalreporter.write_sep("-", "parity taint report (F mode: tainted pairs compared, not asserted)")
+    for label, r in REPORT:
+        terminalreporter.write_line(
+            f"{label}: pairs={r['pairs']} tainted={r['tainted']} ({100 * r['tainted_frac']:.2f}%) "
+            f"tainted_differ={r['tainted_differ']} flags={r['flags']} events={r['events']} "
+            f"max_err={r['max_time_err']:.3g}")
