@@ -273,6 +273,8 @@ typedef struct {
     int64_t spill_bytes;         /* spill-heap bytes used by the kept rounds  */
     int64_t spill_heap_bytes;    /* spill-heap bytes allocated (all rounds)   */
     int64_t batches;             /* slot batches of the last simulate         */
+    int64_t enc_bytes;           /* algorithmic bytes of the stored encoding
+                                    (records, entries, times)  */
 } avfs_stats;
 avfs_status avfs_get_stats(avfs_ctx *ctx, avfs_stats *st);
 

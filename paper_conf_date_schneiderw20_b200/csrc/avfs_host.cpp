@@ -131,6 +131,8 @@ struct avfs_ctx {
         d_err, d_list[2], d_prev[2], d_pois[2], d_spill_top, d_lvlsync, d_count, d_swround, d_swindex, g_loc, g_init, g_count,
         g_times, g_bad;
     std::vector<DevBuf> arena;        // per round: [buffer][slot group][region]
+    std::vector<DevBuf> recs;         // per round: [buffer][slot group] records
+    DevBuf d_zero, d_enc;
     std::vector<DevBuf> spill;        // per round: spill heap (kept: readback may point into it)
     int64_t spill_hint = 0;           // heap words the last simulate asked for (all rounds)
     int64_t spill_per_group = 0;      // largest heap words per slot group asked for so far (sizing hint)
@@ -322,12 +324,18 @@ avfs_status build_plan(avfs_ctx* ctx) {
     return AVFS_OK;
 }
 
-// arena buffer of a location: PIs 0..n_pi-1, kept signals next, scratch last
+// arena buffer of a gate output: kept signals first, scratch after (PIs have
+// no buffer: their waveforms are the stimulus words, reading C2)
 uint32_t buffer_id(const avfs_ctx* ctx, uint32_t loc) {
     const uint32_t kind = loc & LOC_KIND, id = loc & LOC_ID;
-    if (kind == LOC_PI) return id;
-    if (kind == LOC_PINNED) return (uint32_t)ctx->n_pi + id;
-    return (uint32_t)(ctx->n_pi + ctx->n_pinned) + id;
+    if (kind == LOC_PINNED) return id;
+    return (uint32_t)ctx->n_pinned + id;
+}
+
+// location code of a gate input as the sweep reads it
+uint32_t input_code(const avfs_ctx* ctx, uint32_t loc) {
+    if ((loc & LOC_KIND) == LOC_PI) return loc;
+    return (loc & LOC_KIND) | buffer_id(ctx, loc);
 }
 
 avfs_status upload_netlist(avfs_ctx* ctx) {
@@ -342,29 +350,12 @@ avfs_status upload_netlist(avfs_ctx* ctx) {
         std::memset(&d, 0, sizeof d);
         std::memset(&e, 0, sizeof e);
         const int k = (int)(ctx->fanin_ptr[g + 1] - ctx->fanin_ptr[g]);
-        for (int p = 0; p < KMAX; ++p) d.in_loc[p] = p < k ? buffer_id(ctx, ctx->loc[ctx->fanin_sig[ctx->fanin_ptr[g] + p]]) : 0u;
+        for (int p = 0; p < KMAX; ++p) d.in_loc[p] = p < k ? input_code(ctx, ctx->loc[ctx->fanin_sig[ctx->fanin_ptr[g] + p]]) : 0u;
         d.out_loc = buffer_id(ctx, ctx->loc[ctx->n_pi + g]);
         d.sig = (uint32_t)(ctx->n_pi + g);
-        d.ttk = (uint32_t)ctx->cell_tt[ctx->gate_cell[g]] | ((uint32_t)k << 16) |
-                ((ctx->is_po[ctx->n_pi + g] ? 1u : 0u) << 24);
-        // 2-input gates: observability table for the event pruning of the
-        // sweep -- entry (stable-input mask s | their values << 2) holds, per
-        // input with events, whether the truth table restricted to the stable
-        // inputs' values depends on it
-        if (k == 2) {
-            const uint32_t tt = ctx->cell_tt[ctx->gate_cell[g]];
-            for (uint32_t idx = 0; idx < 16; ++idx) {
-                const uint32_t st = idx & 3u, val = (idx >> 2) & st;
-                uint32_t obs = 0;
-                for (uint32_t q = 0; q < 2; ++q) {
-                    if (st & (1u << q)) continue;
-                    for (uint32_t b = 0; b < 4; ++b)
-                        if (!(b & (1u << q)) && (b & st) == val && ((tt >> b) & 1u) != ((tt >> (b | (1u << q))) & 1u))
-                            obs |= 1u << q;
-                }
-                d.obs |= obs << (2 * idx);
-            }
-        }
+        const uint32_t ttm = (uint32_t)ctx->cell_tt[ctx->gate_cell[g]] & (0xFFFFu >> (16 - (1 << k)));
+        d.ttk = ttm | ((uint32_t)k << 16) | ((ctx->is_po[ctx->n_pi + g] ? 1u : 0u) << 24);
+        d.fanout = (uint32_t)std::min<int64_t>(ctx->fanout[ctx->n_pi + g], 0xFFFFFF);
         e.coef_off = ctx->coef_off[g];
         e.k = (uint32_t)k;
         e.island = (uint32_t)ctx->island[g];
@@ -838,33 +829,27 @@ avfs_status avfs_sync(avfs_ctx* ctx) {
 
 static avfs_status run_round(avfs_ctx* ctx, Round& R, int round_idx, const int32_t* d_sw_list,
                              const int32_t* d_prev_idx, bool timed) {
-    const bool persistent = (round_idx == 0);
-    // launch bounds: sweep_kernel up to 1024 threads, level_kernel 512 threads
-    const int wmax = persistent ? AVFS_SWEEP_THREADS / 32 : 16;
+    const bool rerun = round_idx > 0;
+    const int wmax = AVFS_SWEEP_THREADS / 32;
     int wpc = ctx->opt.warps_per_cta > 0 ? ctx->opt.warps_per_cta : wmax;
     wpc = std::min(wpc, wmax);
-    const int smem = persistent ? sweep_smem_bytes(wpc) : level_smem_bytes(wpc);
-    int bps = 0;
-    if (persistent) CK(sweep_occupancy(wpc, smem, &bps));
-    else CK(level_occupancy(wpc, smem, &bps));
-    if (bps < 1) return fail(ctx, AVFS_ERR_CAPACITY, "sweep kernel does not fit on an SM (smem %d)", smem);
-    const int64_t resident = (int64_t)ctx->n_sm * bps;
+    const double per_level = ctx->depth > 0 ? (double)ctx->n_gates / ctx->depth : 1.0;
     // narrow netlists (few gates per level): one sweep CTA walks G slot groups
     // at once so that every warp has >= 2 gates of a level (power of 2, <= wpc)
     int grp = 1;
-    if (persistent) {
-        const double per_level = ctx->depth > 0 ? (double)ctx->n_gates / ctx->depth : 1.0;
-        while (grp < wpc && per_level / (double)(wpc / grp) < 2.0) grp *= 2;
-        if (const char* e = getenv("AVFS_GROUPS_PER_CTA")) grp = std::max(1, std::min(wpc, atoi(e)));
-        while (wpc % grp) grp /= 2;
-    }
-    R.grp = grp;
-    // few slot groups for the SMs (last wave mostly empty): S co-resident CTAs
-    // share a group; S minimises waves / S, ties to the smaller S, and every
-    // warp keeps >= 2 gates of a level
+    while (grp < wpc && per_level / (double)(wpc / grp) < 2.0) grp *= 2;
+    if (const char* e = getenv("AVFS_GROUPS_PER_CTA")) grp = std::max(1, std::min(wpc, atoi(e)));
+    while (wpc % grp) grp /= 2;
+    const int smem = sweep_smem_bytes(wpc, grp);
+    int bps = 0;
+    CK(sweep_occupancy(wpc, smem, &bps));
+    if (bps < 1) return fail(ctx, AVFS_ERR_CAPACITY, "sweep kernel does not fit on an SM (smem %d)", smem);
+    const int64_t resident = (int64_t)ctx->n_sm * bps;
+    // few slot groups for the SMs (last wave mostly empty, e.g. reruns): S
+    // co-resident CTAs share a group; S minimises waves / S, ties to the
+    // smaller S, and every warp keeps >= 2 gates of a level
     int split = 1;
-    if (persistent && grp == 1) {
-        const double per_level = ctx->depth > 0 ? (double)ctx->n_gates / ctx->depth : 1.0;
+    if (grp == 1) {
         double best = 1e300;
         for (int S = 1; S <= 4; S *= 2) {
             if (S > 1 && per_level / S / wpc < 2.0) break;
@@ -874,26 +859,29 @@ static avfs_status run_round(avfs_ctx* ctx, Round& R, int round_idx, const int32
         }
         if (const char* e = getenv("AVFS_SPLIT")) split = std::max(1, std::min(4, atoi(e)));
     }
+    R.grp = grp;
     R.split = split;
-    if (persistent && split > 1) {
+    if (split > 1) {
         const int64_t items = R.n_sw * split;
         R.grid = (int32_t)std::min<int64_t>(items, std::max<int64_t>(resident / split * split, split));
     } else {
-        R.grid = (int32_t)(persistent ? std::min<int64_t>((R.n_sw + grp - 1) / grp, resident) : resident);
+        R.grid = (int32_t)std::min<int64_t>((R.n_sw + grp - 1) / grp, resident);
     }
     if (R.grid < 1) R.grid = 1;
     if ((int)ctx->arena.size() <= round_idx) ctx->arena.resize(round_idx + 1);
-    const int64_t n_buf = (int64_t)ctx->n_pi + ctx->n_pinned + ctx->n_scratch;
+    if ((int)ctx->recs.size() <= round_idx) ctx->recs.resize(round_idx + 1);
+    const int64_t n_buf = (int64_t)ctx->n_pinned + ctx->n_scratch;
     if ((uint64_t)R.n_sw * R.region_bytes >= (1ull << 32))
         return fail(ctx, AVFS_ERR_NOMEM, "slot-group stride exceeds 4 GiB; restrict the slot range");
     CK(ctx->arena[round_idx].ensure((size_t)std::max<int64_t>(n_buf, 1) * R.n_sw * R.region_bytes));
+    CK(ctx->recs[round_idx].ensure((size_t)std::max<int64_t>(n_buf, 1) * R.n_sw * sizeof(uint4)));
     CK(ctx->d_ovf.ensure(std::max<int64_t>(R.n_sw, 1) * sizeof(int32_t)));
     CK(cudaMemsetAsync(ctx->d_ovf.p, 0, R.n_sw * sizeof(int32_t), ctx->stream));
     // spill heap: the requested size, within free device memory (keep 1 GiB)
     if ((int)ctx->spill.size() <= round_idx) ctx->spill.resize(round_idx + 1);
     R.spill_words = 0;
     if (R.spill_want > 0 && ctx->spill[round_idx].n >= (size_t)R.spill_want * 4) {
-        R.spill_words = R.spill_want;                  // reuse the heap of a previous simulate
+        R.spill_words = (int64_t)(ctx->spill[round_idx].n / 4);     // reuse the heap (with its headroom)
     } else if (R.spill_want > 0) {
         size_t fr = 0, tot = 0;
         CK(cudaMemGetInfo(&fr, &tot));
@@ -913,6 +901,8 @@ static avfs_status run_round(avfs_ctx* ctx, Round& R, int round_idx, const int32
     DevBuf& pois = ctx->d_pois[round_idx & 1];
     CK(pois.ensure(pois_words * 4));
     CK(cudaMemsetAsync(pois.p, 0, pois_words * 4, ctx->stream));
+    CK(ctx->d_zero.ensure(16));
+    CK(cudaMemsetAsync(ctx->d_zero.p, 0, 16, ctx->stream));
     SweepParams p{};
     p.gates = ctx->d_gates.as<GateDesc>();
     p.level_ptr = ctx->d_level_ptr.as<int32_t>();
@@ -933,6 +923,7 @@ static avfs_status run_round(avfs_ctx* ctx, Round& R, int round_idx, const int32
     p.pin_n_sw = R.n_sw;
     p.arena = ctx->arena[round_idx].as<uint8_t>();
     p.region_bytes = R.region_bytes;
+    p.recs = ctx->recs[round_idx].as<uint4>();
     p.W = R.W;
     p.grp_per_cta = R.grp;
     p.split = R.split;
@@ -948,19 +939,14 @@ static avfs_status run_round(avfs_ctx* ctx, Round& R, int round_idx, const int32
     p.pois = pois.as<uint32_t>();
     p.pois_prev = round_idx == 0 ? nullptr : ctx->d_pois[(round_idx - 1) & 1].as<uint32_t>();
     p.prev_idx = d_prev_idx;
+    p.zero = ctx->d_zero.as<float>();
     p.act = ctx->d_act.as<unsigned long long>();
     p.latest = ctx->d_latest.as<unsigned int>();
     p.ovf = ctx->d_ovf.as<int32_t>();
-    CK(launch_pi_regions(p, ctx->n_pi, ctx->stream));   // materialise the PI waveforms of this round
-    ctx->stats.launches++;
+    p.enc_units = ctx->d_enc.as<unsigned long long>();
     if (timed) CK(cudaEventRecord(ctx->ev0, ctx->stream));
-    if (persistent) {
-        CK(launch_sweep(p, R.grid, wpc, ctx->stream));
-        ctx->stats.launches++;
-    } else {
-        for (int L = 0; L < ctx->depth; ++L) CK(launch_level(p, L, R.grid, wpc, ctx->stream));
-        ctx->stats.launches += ctx->depth;
-    }
+    CK(launch_sweep(p, rerun, R.grid, wpc, ctx->stream));
+    ctx->stats.launches++;
     if (timed) CK(cudaEventRecord(ctx->ev1, ctx->stream));
     if (round_idx == 0) ctx->stats.warps_per_cta = wpc;
     return AVFS_OK;
@@ -1007,6 +993,8 @@ avfs_status avfs_simulate(avfs_ctx* ctx, void* cuda_stream) {
     CK(cudaMemsetAsync(ctx->d_act.p, 0, (size_t)S * V * sizeof(unsigned long long), ctx->stream));
     CK(cudaMemsetAsync(ctx->d_latest.p, 0, (size_t)V * 4, ctx->stream));
     CK(cudaMemsetAsync(ctx->d_err.p, 0, 16, ctx->stream));
+    CK(ctx->d_enc.ensure(8));
+    CK(cudaMemsetAsync(ctx->d_enc.p, 0, 8, ctx->stream));
     // delay computation kernel: d'(gate, pin, pol, Vdd) in FP64 -> binary32 table
     CK(ctx->d_dtab.ensure((size_t)V * std::max(ctx->n_gates, 1) * 8 * sizeof(float)));
     {
@@ -1037,14 +1025,15 @@ avfs_status avfs_simulate(avfs_ctx* ctx, void* cuda_stream) {
     // rerun rounds' arenas and heaps of the previous simulate are stale: give
     // their memory back so that pass 0 can size its heap from the hint
     for (size_t r = 1; r < ctx->arena.size(); ++r) ctx->arena[r].release();
+    for (size_t r = 1; r < ctx->recs.size(); ++r) ctx->recs[r].release();
     for (size_t r = 1; r < ctx->spill.size(); ++r) ctx->spill[r].release();
     // slot batching: when the arena for every slot group would not
     // fit, the groups run in batches on the same arena and heap; activity,
     // latest arrival and energy accumulate over all batches, waveform readback
     // keeps the last batch
     const int64_t n_sw_all = sw_hi - sw_lo;
-    const int64_t region0 = 128 + 4 * (int64_t)(32 * ctx->opt.capacity);
-    const int64_t per_group = ((int64_t)ctx->n_pi + ctx->n_pinned + ctx->n_scratch) * region0;
+    const int64_t region0 = REG_TIMES + 4 * (int64_t)(32 * ctx->opt.capacity);
+    const int64_t per_group = ((int64_t)ctx->n_pinned + ctx->n_scratch) * (region0 + (int64_t)sizeof(uint4));
     // device bytes one group needs: its arena share plus its expected spill
     // (learned from earlier batches / simulates, words per group)
     auto group_bytes = [&]() { return (double)per_group + 1.25 * 4.0 * (double)ctx->spill_per_group; };
@@ -1053,6 +1042,7 @@ avfs_status avfs_simulate(avfs_ctx* ctx, void* cuda_stream) {
         if (cudaMemGetInfo(&fr, &tot) != cudaSuccess) return 0.0;
         double own = 0;
         for (auto& a : ctx->arena) own += (double)a.n;
+        for (auto& a : ctx->recs) own += (double)a.n;
         for (auto& h : ctx->spill) own += (double)h.n;
         return (double)fr + own - (double)(2ll << 30);
     };
@@ -1077,6 +1067,7 @@ avfs_status avfs_simulate(avfs_ctx* ctx, void* cuda_stream) {
     for (int64_t b0 = sw_lo; b0 < sw_hi; b0 += nb) {
     if (b0 > sw_lo) {                                   // earlier batches' rerun memory is not kept
         for (size_t r = 1; r < ctx->arena.size(); ++r) ctx->arena[r].release();
+        for (size_t r = 1; r < ctx->recs.size(); ++r) ctx->recs[r].release();
         for (size_t r = 1; r < ctx->spill.size(); ++r) ctx->spill[r].release();
         if (learn && ctx->opt.max_batch_slots <= 0) {   // resize the remaining batches
             const int64_t fit = (int64_t)(0.8 * avail_bytes() / std::max(group_bytes(), 1.0));
@@ -1091,9 +1082,9 @@ avfs_status avfs_simulate(avfs_ctx* ctx, void* cuda_stream) {
     R0.sw_first = b0;
     R0.capacity = ctx->opt.capacity;
     R0.W = 32 * R0.capacity;
-    R0.region_bytes = 128 + 4 * (int64_t)R0.W;
+    R0.region_bytes = REG_TIMES + 4 * (int64_t)R0.W;
     {
-        const int64_t arena_words = ((int64_t)ctx->n_pi + ctx->n_pinned + ctx->n_scratch) * R0.n_sw * R0.region_bytes / 4;
+        const int64_t arena_words = ((int64_t)ctx->n_pinned + ctx->n_scratch) * R0.n_sw * R0.region_bytes / 4;
         // auto: arena/4 (>= 256 MiB), or 1.25x what the previous simulate asked
         // for in all its rounds, so that repeated runs do not rerun
         R0.spill_want = ctx->opt.spill_bytes > 0 ? ctx->opt.spill_bytes / 4
@@ -1149,7 +1140,7 @@ avfs_status avfs_simulate(avfs_ctx* ctx, void* cuda_stream) {
             Rn.capacity = std::min(prev.capacity * 4, 1024);
         }
         Rn.W = 32 * Rn.capacity;
-        Rn.region_bytes = 128 + 4 * (int64_t)Rn.W;
+        Rn.region_bytes = REG_TIMES + 4 * (int64_t)Rn.W;
         ctx->stats.overflow_slot_warps += n_ovf;
         ctx->stats.rerun_rounds++;
         st = run_round(ctx, Rn, r + 1, ctx->d_list[cur].as<int32_t>(), ctx->d_prev[cur].as<int32_t>(), false);
@@ -1272,7 +1263,8 @@ static avfs_status gather(avfs_ctx* ctx, int32_t n_sig, const int32_t* sig, int6
     g.sw_round = ctx->d_swround.as<int32_t>();
     g.sw_index = ctx->d_swindex.as<int32_t>();
     for (size_t r = 0; r < ctx->rounds.size(); ++r)
-        g.rounds[r] = GatherRound{ctx->arena[r].as<uint8_t>(), ctx->rounds[r].region_bytes, ctx->rounds[r].n_sw};
+        g.rounds[r] = GatherRound{ctx->arena[r].as<uint8_t>(), ctx->recs[r].as<uint4>(), ctx->rounds[r].region_bytes,
+                                  ctx->rounds[r].n_sw};
     g.cap = times ? cap : 0;
     g.init = ctx->g_init.as<uint8_t>();
     g.count = ctx->g_count.as<int32_t>();
@@ -1361,7 +1353,8 @@ avfs_status avfs_capture(avfs_ctx* ctx, const float* t_clk, int32_t n_bins, floa
     p.sw_round = ctx->d_swround.as<int32_t>();
     p.sw_index = ctx->d_swindex.as<int32_t>();
     for (size_t r = 0; r < ctx->rounds.size(); ++r)
-        p.rounds[r] = GatherRound{ctx->arena[r].as<uint8_t>(), ctx->rounds[r].region_bytes, ctx->rounds[r].n_sw};
+        p.rounds[r] = GatherRound{ctx->arena[r].as<uint8_t>(), ctx->recs[r].as<uint4>(), ctx->rounds[r].region_bytes,
+                                  ctx->rounds[r].n_sw};
     p.slot_fail = ctx->c_slot.as<uint32_t>();
     p.slot_last = ctx->c_slot.as<uint32_t>() + (size_t)n_sw * 32;
     p.fail_po = ctx->c_out.as<uint32_t>();
@@ -1414,6 +1407,21 @@ avfs_status avfs_get_stats(avfs_ctx* ctx, avfs_stats* st) {
         b += (1.0 + (double)ctx->fanout[s]) * (4.0 * slots + 4.0 * (double)a);
     }
     ctx->stats.alg_bytes = (int64_t)b;
+    // the same for the encoding the sweep moves: per (gate
+    // output, slot group) a 16-B record, per slot with events a 4-B entry,
+    // 4 B per transition, each written once and read once per reading pin;
+    // PI waveforms are the stimulus words (8 B per (PI, group) per reading pin)
+    unsigned long long units = 0;
+    CK(cudaMemcpy(&units, ctx->d_enc.p, 8, cudaMemcpyDeviceToHost));
+    const double groups = (double)ctx->stats.slot_warps;
+    double e = 4.0 * (double)units;
+    for (int32_t s = 0; s < S; ++s) {
+        uint64_t a = 0;
+        for (int32_t k = 0; k < V; ++k) a += act[(size_t)s * V + k];
+        if (s < ctx->n_pi) e += (double)ctx->fanout[s] * 8.0 * groups;
+        else e += (1.0 + (double)ctx->fanout[s]) * (16.0 * groups + 4.0 * (double)a);
+    }
+    ctx->stats.enc_bytes = (int64_t)e;
     *st = ctx->stats;
     return AVFS_OK;
 }

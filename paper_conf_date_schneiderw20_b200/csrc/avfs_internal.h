@@ -24,23 +24,36 @@ constexpr uint32_t LOC_PINNED = 2u << 30;    // low bits: pinned id (PO / probe 
 constexpr uint32_t LOC_KIND = 3u << 30;
 constexpr uint32_t LOC_ID = ~LOC_KIND;
 
-// Header word of one (signal, slot) waveform (reading C1):
-constexpr uint32_t HDR_N = 0x00000FFFu;      // transition count (< 4096; larger counts overflow)
-constexpr int HDR_OFF_SHIFT = 12;            // bits 12..27: offset of the slot's first event in the
-constexpr uint32_t HDR_OFF = 0xFFFFu;        //   region (exclusive prefix of the counts of lanes < l)
-constexpr int HDR_INIT_SHIFT = 28;
-constexpr uint32_t HDR_INIT = 1u << 28;      // value before t = 0
-constexpr uint32_t HDR_POISON = 1u << 29;    // events not stored here or upstream
-constexpr uint32_t HDR_SPILL = 1u << 30;     // the region's events live in the round's spill heap; the
-                                             //   region's first event word pair holds their address
+// Waveform of one (signal, 32-slot group) (reading C1), in two parts:
+//
+//  record  uint4 {init, E, A, meta} in the round's record array
+//          [buffer][group]: init = bit l is slot l's value before t = 0,
+//          E = slots with >= 1 transition, A = slots that own an entry
+//          (E is a subset of A), meta = total stored transitions (REC_NTOT)
+//          plus REC_POISON / REC_SPILL.  PIs have no record: it is the
+//          stimulus words (init = p1, E = A = p1 xor p2, one event at t = 0).
+//  region  in the round's arena [buffer][group]: 32 entry words, compact in
+//          the order of A's set bits (entry = n | off << ENT_OFF_SHIFT: the
+//          slot's count and the word offset of its first time), then at byte
+//          REG_TIMES the binary32 times (W words); when the record says
+//          REC_SPILL the times live in the spill heap at the 64-bit address
+//          stored at byte REG_SPILLPTR.
+constexpr uint32_t REC_NTOT = 0x0FFFFFFFu;
+constexpr uint32_t REC_POISON = 1u << 29;    // events not stored here or upstream (overflow)
+constexpr uint32_t REC_SPILL = 1u << 30;
+constexpr uint32_t ENT_N = 0xFFFu;           // per-slot count limit 4095
+constexpr int ENT_OFF_SHIFT = 12;            // 20-bit time offset: <= 2^20 - 1 times per (signal, group)
+constexpr uint32_t OFF_LIMIT = 1u << 20;
+constexpr int REG_SPILLPTR = 128;
+constexpr int REG_TIMES = 144;
 
-// Gate descriptor, 32 B, read warp-uniformly (P:L154 step 1).
+// Gate descriptor, 32 B, read by one lane per gate (P:L154 step 1).
 struct alignas(16) GateDesc {
-    uint32_t in_loc[KMAX];
-    uint32_t out_loc;
-    uint32_t sig;        // output signal id (activity row)
-    uint32_t ttk;        // bits 0..15 truth table, 16..23 #inputs, 24..31 flags (bit 24: PO)
-    uint32_t obs;        // 2-input gates: observability table (2 bits per stable-input pattern)
+    uint32_t in_loc[KMAX];   // location codes of the inputs (LOC_PI | pi, or kind | buffer id)
+    uint32_t out_loc;        // arena buffer id of the output
+    uint32_t sig;            // output signal id (activity row)
+    uint32_t ttk;            // bits 0..15 truth table, 16..23 #inputs, 24..31 flags (bit 24: PO)
+    uint32_t fanout;         // reading pins of the output (algorithmic-byte accounting)
 };
 static_assert(sizeof(GateDesc) == 32, "GateDesc layout");
 
@@ -68,8 +81,6 @@ struct DelayParams {
     int32_t* err;                            // bit 0: non-positive delay
 };
 
-// One slot-warp region: 32 header words followed by W = 32*C event times
-// (compact: lane l's events start at the exclusive prefix sum of the counts).
 struct SweepParams {
     const GateDesc* __restrict__ gates;     // sorted by level
     const int32_t* __restrict__ level_ptr;  // [depth+1] offsets into gates (level 1..depth)
@@ -82,45 +93,44 @@ struct SweepParams {
     int64_t n_pairs;
     int32_t n_vdd;
     int64_t slot_first, slot_end;           // public slot range simulated
-    // slot-warps of this run: sw = sw_list ? sw_list[i] : sw_first + i, i < n_sw
+    // slot groups of this run: sw = sw_list ? sw_list[i] : sw_first + i, i < n_sw
     const int32_t* __restrict__ sw_list;
     int64_t sw_first;
     int64_t n_sw;                           // slot groups in this launch
     int64_t i_base;                         // index of this launch's first group within the round
-    int64_t pin_n_sw;                       // slot groups in the round (pinned arena / ovf flags)
-    // arena of the round: [buffer][pin_n_sw][region]; buffers = PIs, kept signals, scratch
+    int64_t pin_n_sw;                       // slot groups in the round (arena / records / ovf flags)
+    // arena of the round: [buffer][pin_n_sw][region]; buffers = kept signals, then scratch
     uint8_t* arena;
     int64_t region_bytes;
-    int32_t W;                              // event capacity per region (32*C)
+    uint4* recs;                            // [buffer][pin_n_sw] records
+    int32_t W;                              // in-place time capacity per region (words)
     int32_t grp_per_cta;                    // slot groups a sweep CTA walks at once (power of 2)
     int32_t split;                          // sweep CTAs sharing one slot group (grp_per_cta == 1)
     unsigned int* lvl_sync;                 // [n_sw] level counters of split groups (zeroed per round)
     int32_t n_pi;                           // gate index = output signal - n_pi
-    // spill heap of the round: regions whose inputs carry more than W events
-    // store their events here (bump allocation in words, 16-B granules)
+    // spill heap of the round: gates whose inputs carry more than W events
+    // store their times here (bump allocation in words, 16-B granules)
     float* spill;
     unsigned long long* spill_top;          // words handed out (counts failed requests too)
     uint64_t spill_words;                   // heap capacity
     // poison bitmaps [group index in round][n_gates] bits: this round's, and
-    // the previous round's (null on pass 0) for exact activity accounting
+    // the previous round's (null on pass 0): set = poisoned and not counted yet
     uint32_t* pois;
     const uint32_t* pois_prev;
     const int32_t* prev_idx;                // [n_sw] group's index in the previous round
+    const float* zero;                      // 4 words of 0.0f: the time of every PI event (reading C2)
     // outputs
     unsigned long long* act;                // [n_signals][n_vdd]
     unsigned int* latest;                   // [n_vdd] float bits (non-negative)
-    int32_t* ovf;                           // [n_sw] overflow flag per slot-warp
+    int32_t* ovf;                           // [n_sw] overflow flag per slot group
+    unsigned long long* enc_units;          // sum over gates of (1 + fanout) * #slots with events
 };
 
 // launch wrappers (avfs_kernels.cu)
-int sweep_smem_bytes(int warps_per_cta);
-int level_smem_bytes(int warps_per_cta);
+int sweep_smem_bytes(int warps_per_cta, int grp_per_cta);
 cudaError_t sweep_occupancy(int warps_per_cta, int smem, int* blocks_per_sm);
 cudaError_t launch_delays(const DelayParams& p, cudaStream_t st);
-cudaError_t launch_sweep(const SweepParams& p, int grid, int warps_per_cta, cudaStream_t st);
-cudaError_t level_occupancy(int warps_per_cta, int smem, int* blocks_per_sm);
-cudaError_t launch_level(const SweepParams& p, int level, int grid, int warps_per_cta, cudaStream_t st);
-cudaError_t launch_pi_regions(const SweepParams& p, int32_t n_pi, cudaStream_t st);
+cudaError_t launch_sweep(const SweepParams& p, bool rerun, int grid, int warps_per_cta, cudaStream_t st);
 cudaError_t launch_expand(const uint32_t* p1, const uint32_t* p2, int64_t n_pairs, int32_t words,
                           int32_t n_pi, int32_t n_pw, uint32_t* p1t, uint32_t* p2t, cudaStream_t st);
 cudaError_t launch_pi_activity(const uint32_t* p1t, const uint32_t* p2t, int32_t n_pi, int32_t n_pw,
@@ -131,12 +141,13 @@ cudaError_t launch_compact_overflow(const int32_t* ovf, int64_t n_sw, const int3
                                     int32_t* out_count, cudaStream_t st);
 
 struct GatherRound {       // one simulated round for readback
-    const uint8_t* pinned;
+    const uint8_t* pinned;      // arena (kept buffers first)
+    const uint4* recs;          // records [buffer][n_sw]
     int64_t region_bytes;
     int64_t n_sw;
 };
 struct GatherParams {
-    const uint32_t* sig_loc;    // [n_sig] location codes (PI or pinned)
+    const uint32_t* sig_loc;    // [n_sig] location codes (LOC_PI | pi, or LOC_PINNED | arena buffer)
     int32_t n_sig;
     int64_t slot0, n_slots;
     int64_t n_pairs;

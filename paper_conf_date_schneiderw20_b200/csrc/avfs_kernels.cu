@@ -11,31 +11,27 @@
 //   sweep_kernel        H6+H7 persistent level sweep.  One CTA owns one
 //                           32-slot group (same Vdd, 32 stimulus pairs) at a
 //                           time and walks every level of the netlist with a
-//                           CTA barrier between levels (P:L166 level-wise
-//                           processing); warp w evaluates gates w, w+nw, ...
-//                           of the level for the 32 slots (the
-//                           horizontal plane = one gate, all slots).  Per
-//                           gate: delays from the FP64 delay table (P:L139,
-//                           Eq. 9), coalesced header loads, an
-//                           event-parallel merge + inertial filter (P:L148,
-//                           readings C3-C6) built from warp ballots, compact
-//                           stores, capacity check, activity and
-//                           latest-arrival reductions (P:L141 step 4).
-//   level_kernel        H7  the same evaluation, one launch per level, for
-//                           the overflow reruns.
+//                           barrier between levels (P:L166 level-wise
+//                           processing).  Warps grab batches of a level's
+//                           gates; per batch a bit-parallel phase (lane =
+//                           gate, 32 slots per word) evaluates the initial
+//                           values and finds the slots with observable input
+//                           events, and an item phase (lane = (gate, slot))
+//                           merges those slots' input lists with the
+//                           inertial filter (readings C3-C6).
+//                           Delays from the FP64 delay table (Eq. 9).
+//                           Reruns (H7) use the same kernel on the
+//                           overflowed slot groups.
+//   delay_kernel        H2/H3 Eq. (4)/(9) in FP64 per (Vdd, gate, arc).
 //   compact_kernel      H7  list of overflowed slot groups for the rerun.
 //   gather_kernel       H9  readback of kept waveforms.
+//   capture_kernel      NEXT-1 test-response analysis.
+//   energy_kernel       NEXT-4 switching energy.
 #include <cuda_runtime.h>
 #include <cstdint>
 
 #include "avfs_internal.h"
 
-#ifndef AVFS_PRUNE
-#define AVFS_PRUNE 1          // drop input events the gate cannot observe in that slot
-#endif
-#ifndef AVFS_PTX_MERGE
-#define AVFS_PTX_MERGE 1      // 2-input staged merge as one PTX loop (0: the C++ loop)
-#endif
 
 namespace avfs {
 
@@ -71,47 +67,43 @@ __device__ __forceinline__ uint32_t warp_incl_scan(uint32_t v, int) {
 #define FULL 0xffffffffu
 
 // ---------------------------------------------------------------------------
-// Gate evaluation for one gate x one 32-slot group.
+// Persistent level sweep (H6 + H7).
 //
-// Lane l = slot l.  The K input header words (staged rows in shared memory,
-// or one coalesced 128-B row each) give per slot the event counts n_q, the
-// offsets of the event lists, the initial input values and hence the
-// initial output y0 = TT(inputs) (reading C1).  m = sum_q n_q bounds the
-// slot's output events; its warp prefix sum places slot l's outputs at
-// offset base(l) of the output region (the header stores offset and count).
-// Each lane then merges its K sorted lists (ties: ascending pin, reading C5)
-// for exactly max_l m(l) steps, evaluating the truth table after every input
-// event and applying the inertial filter (reading C3: a change whose
-// time precedes the pending output cancels it, reading C4: no reschedule on
-// confirming events); surviving outputs t + d(pin, polarity) (Eq. 9 delays)
-// are stored as they are pushed -- only the last one can later be cancelled,
-// and the next push overwrites it.
+// One CTA owns one 32-slot group (one operating point, 32 stimulus pairs) at
+// a time and walks every level of the netlist with a barrier between levels
+// (P:L166 level-wise processing).  A warp repeatedly grabs a batch of QN
+// gates of the current level and evaluates it in two phases:
 //
-// Capacity: the region of a 32-slot group holds W = 32 C times; a gate-warp
-// whose inputs carry more than W events in total (an upper bound of its
-// outputs) is poisoned and the slot group rerun at 4C (reading C17).
+//  Phase A (lane = gate; bit-parallel over the 32 slots).  Each lane reads
+//  its gate's descriptor and the records of the gate's inputs (init, event
+//  and entry masks, counts), evaluates the truth table on the 32 initial
+//  values at once (Shannon expansion, y0 = TT(inputs), reading C1) and the
+//  mask A of slots where some input event is observable: the output is not
+//  constant over the input values the slot can take (an input without events
+//  is fixed at its value, one with events is free) -- an event the gate
+//  cannot observe never changes the evaluated output (reading C4) and is not
+//  merged.  Gates with A = 0 (no observable event in any slot) are finished
+//  here: their record {y0, no events} is written and nothing else is read.
+//  The others are queued with their masks, input time bases, and Eq. (9)
+//  delays.  Time storage: a gate whose inputs carry U events in total (an
+//  upper bound of its outputs, reading C17) stores its times in place if
+//  U <= W, else in the round's spill heap; heap exhausted -> poisoned and
+//  the slot group rerun (H7).
+//
+//  Phase B (lane = item = (queued gate, slot in A); items packed 32 per
+//  pass).  Per item: the observable inputs (the per-slot pruning rule
+//  above), their entries (count, offset), output offsets as a segmented
+//  prefix sum of the items' input event counts, then the lane-serial merge
+//  of the sorted input lists by (time, pin) (ties: ascending pin, reading
+//  C5) with the inertial filter (reading C3: a change whose time
+//  precedes the pending output cancels it, equality kept; C4: no reschedule
+//  on confirming events).  Surviving outputs t + d(pin, polarity) are
+//  stored as they are pushed -- only the last one can later be cancelled.
+//  Counts, event masks, activity (reading C15) and the latest PO arrival
+//   are accumulated per queued gate in shared memory; a final step
+//  (lane = queued gate) writes the output records and does one global
+//  atomic per gate and operating point.
 // ---------------------------------------------------------------------------
-
-struct Env {
-    uint8_t* row;                  // arena + i * region_bytes
-    uint32_t stride;               // bytes between buffers = n_sw * region_bytes (< 4 GiB, checked on host)
-    int64_t i;                     // index of the slot group in the round (overflow flag)
-    int kv, lane;
-    unsigned long long* act_kv;    // &act[0][kv]
-};
-
-__device__ __forceinline__ uint8_t* region(uint32_t buf, const Env& E) {
-    return E.row + (uint64_t)buf * (uint64_t)E.stride;
-}
-
-// First event word of a region: in place, or in the spill heap (HDR_SPILL in
-// any of the region's header words; the address is the region's first
-// event word pair).
-__device__ __forceinline__ const uint8_t* ev_base(const uint8_t* reg, uint32_t hw) {
-    const uint8_t* b = reg + 128;
-    if (hw & HDR_SPILL) b = reinterpret_cast<const uint8_t*>(__ldcg(reinterpret_cast<const unsigned long long*>(b)));
-    return b;
-}
 
 __device__ __forceinline__ uint32_t smem_u32(const void* p) {
     return static_cast<uint32_t>(__cvta_generic_to_shared(p));
@@ -126,131 +118,264 @@ __device__ __forceinline__ uint32_t lds_u32(uint32_t a) {
     asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v) : "r"(a));
     return v;
 }
-__device__ __forceinline__ void cp_async16(uint32_t dst, const void* src) {
-    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(dst), "l"(src) : "memory");
+__device__ __forceinline__ uint32_t lds_u16(uint32_t a) {
+    unsigned short v;
+    asm volatile("ld.shared.u16 %0, [%1];" : "=h"(v) : "r"(a));
+    return v;
 }
-__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
-__device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_all;" ::: "memory"); }
-
-constexpr int EV_STAGE = 256;   // staged event words per gate (EV_STAGE / K' per input)
-
-// Where a gate's inputs are: header rows (4 x 32 words) and, if they fit, the
-// inputs' compact event lists staged in shared memory by the sweep pipeline.
-struct Staged {
-    bool hdr, ev;
-    uint32_t hdr_s;       // shared address of header row 0 (row q at + 128 q)
-    uint32_t ev_s[1];     // shared address of the staged events (input q at + 4 EV_STAGE q / K')
-    uint32_t dly_s;       // shared address of the gate's 8 delays [pin][pol]
-    uint32_t grp_s;       // shared address of the slot group's index in the round (u32; read when poisoning)
-};
+__device__ __forceinline__ unsigned long long lds_u64(uint32_t a) {
+    unsigned long long v;
+    asm volatile("ld.shared.u64 %0, [%1];" : "=l"(v) : "r"(a));
+    return v;
+}
 __device__ __forceinline__ uint4 lds_u32x4(uint32_t a) {
     uint4 v;
     asm volatile("ld.shared.v4.u32 {%0, %1, %2, %3}, [%4];" : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "r"(a));
     return v;
-}
-__device__ __forceinline__ void sts_u32(uint32_t a, uint32_t v) {
-    asm volatile("st.shared.u32 [%0], %1;" ::"r"(a), "r"(v) : "memory");
 }
 __device__ __forceinline__ float4 lds_f32x4(uint32_t a) {
     float4 v;
     asm volatile("ld.shared.v4.f32 {%0, %1, %2, %3}, [%4];" : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w) : "r"(a));
     return v;
 }
+__device__ __forceinline__ void sts_u32(uint32_t a, uint32_t v) {
+    asm volatile("st.shared.u32 [%0], %1;" ::"r"(a), "r"(v) : "memory");
+}
+__device__ __forceinline__ void sts_u16(uint32_t a, uint32_t v) {
+    asm volatile("st.shared.u16 [%0], %1;" ::"r"(a), "h"((unsigned short)v) : "memory");
+}
+__device__ __forceinline__ void sts_u64(uint32_t a, unsigned long long v) {
+    asm volatile("st.shared.u64 [%0], %1;" ::"r"(a), "l"(v) : "memory");
+}
+__device__ __forceinline__ void sts_u32x4(uint32_t a, uint4 v) {
+    asm volatile("st.shared.v4.u32 [%0], {%1, %2, %3, %4};" ::"r"(a), "r"(v.x), "r"(v.y), "r"(v.z), "r"(v.w)
+                 : "memory");
+}
+__device__ __forceinline__ void sts_f32x4(uint32_t a, float4 v) {
+    asm volatile("st.shared.v4.f32 [%0], {%1, %2, %3, %4};" ::"r"(a), "f"(v.x), "f"(v.y), "f"(v.z), "f"(v.w)
+                 : "memory");
+}
+__device__ __forceinline__ uint32_t atoms_add(uint32_t a, uint32_t v) {
+    uint32_t r;
+    asm volatile("atom.shared.add.u32 %0, [%1], %2;" : "=r"(r) : "r"(a), "r"(v) : "memory");
+    return r;
+}
+__device__ __forceinline__ void atoms_or(uint32_t a, uint32_t v) {
+    asm volatile("red.shared.or.b32 [%0], %1;" ::"r"(a), "r"(v) : "memory");
+}
+__device__ __forceinline__ void atoms_max(uint32_t a, uint32_t v) {
+    asm volatile("red.shared.max.u32 [%0], %1;" ::"r"(a), "r"(v) : "memory");
+}
+__device__ __forceinline__ void atoms_add_u64(uint32_t a, unsigned long long v) {
+    asm volatile("red.shared.add.u64 [%0], %1;" ::"r"(a), "l"(v) : "memory");
+}
 
-// Lane-serial merge + inertial filter of one slot.  Input q's list: n[q]
-// events from ev[q] (shared-memory addresses if STAGED, else global
-// pointers); outputs go to out[0..).  Runs exactly `steps` (= the warp's max
-// m) steps; lanes with fewer events idle through the rest.  Returns the
-// output count.  One step: take the earliest head (ties: lower pin), flip
-// that pin, evaluate the truth table, and apply the filter.
-struct MergeIn {
-    uint64_t ev[KMAX];
-    int n[KMAX];
-    uint32_t bits, proj, tt, dly_s;
-    float4 d01;           // delays of pins 0, 1: {p0 fall, p0 rise, p1 fall, p1 rise}
+constexpr int QN = 16;                 // gates per batch (Phase A lanes, queue entries)
+constexpr int QW = 44;                 // words per queue entry
+enum : int {
+    Q_TTK = 0, Q_SIG = 1, Q_OUT = 2, Q_Y0 = 3,      // descriptor words, output initial values
+    Q_A = 4, Q_EOUT = 5, Q_ACT = 6, Q_CARRY = 7,    // entry mask, accumulated event mask / count, next time offset
+    Q_TB = 8,                                       // u64 time base of the output
+    Q_LAST = 10, Q_FLAG = 11,                       // latest PO time bits; flags | fanout << 8
+    Q_X = 12, Q_E = 16, Q_AQ = 20, Q_LOC = 24,      // per input: init, event, entry masks; location
+    Q_ITB = 28,                                     // 4 x u64 time bases of the inputs
+    Q_DLY = 36                                      // 8 delays [pin][pol], binary32 ps
+};
+constexpr uint32_t QF_POISON = 1u, QF_COUNT = 2u, QF_OWN = 4u, QF_SPILL = 8u;
+constexpr int ITEM_WORDS = QN * 32 / 2;             // u16 items: queue entry << 5 | slot
+constexpr int WARP_SMEM_WORDS = QN * QW + ITEM_WORDS;
+constexpr int CTA_HDR_WORDS = 2 * 32 + 4;           // level counters [group][2], pad
+
+struct Grp {
+    uint8_t* row;          // arena + gi * region_bytes
+    uint4* rec;            // recs + gi
+    uint32_t stride;       // bytes between arena buffers (pin_n_sw * region_bytes < 4 GiB, host-checked)
+    uint32_t rstride;      // records between buffers (pin_n_sw)
+    int64_t gi;            // group index in the round
+    int kv, pw;
+    uint32_t vmask;        // slots of the group inside the simulated range
 };
 
-template <bool STAGED>
-__device__ __forceinline__ float ld_ev(uint64_t a) {
-    return STAGED ? lds_f32((uint32_t)a) : ld_f32(reinterpret_cast<const void*>(a));
+__device__ __forceinline__ void group_setup(const SweepParams& p, int64_t i, int lane, Grp& G) {
+    const int64_t sw = p.sw_list ? (int64_t)p.sw_list[i] : p.sw_first + i;
+    G.kv = (int)(sw / p.n_pw);
+    G.pw = (int)(sw % p.n_pw);
+    G.gi = p.i_base + i;
+    G.row = p.arena + G.gi * p.region_bytes;
+    G.rec = p.recs + G.gi;
+    G.stride = (uint32_t)(p.pin_n_sw * p.region_bytes);
+    G.rstride = (uint32_t)p.pin_n_sw;
+    const int64_t j = (int64_t)G.pw * 32 + lane;
+    const int64_t pub = (int64_t)G.kv * p.n_pairs + j;
+    G.vmask = __ballot_sync(FULL, j < p.n_pairs && pub >= p.slot_first && pub < p.slot_end);
 }
 
-// Address arithmetic of the list walk: 32-bit shared-memory addresses when
-// STAGED, 64-bit global pointers otherwise.
-template <bool STAGED> struct EvAddr { typedef uint64_t T; };
-template <> struct EvAddr<true> { typedef uint32_t T; };
+// all-ones iff truth-table bit b is set
+__device__ __forceinline__ uint32_t tt_leaf(uint32_t tt, int b) {
+    return (uint32_t)((int32_t)(tt << (31 - b)) >> 31);
+}
+__device__ __forceinline__ uint32_t mux(uint32_t s, uint32_t one, uint32_t zero) { return (s & one) | (~s & zero); }
 
-// The 2-input merge + inertial filter over shared-memory lists, as one PTX
-// loop with in-place predicated updates (the compiled C++ loop spends ~10 of
-// its ~41 instructions per step on register copies and constants).  Same
-// semantics as the generic step: ties pick pin 0, a change whose time
-// precedes the pending output cancels it (equality kept), outputs are stored
-// as they are pushed.  steps >= 1.
-__device__ __forceinline__ uint32_t merge2_smem(uint32_t a0, uint32_t e0, uint32_t a1, uint32_t e1, uint32_t bits,
-                                                uint32_t proj, uint32_t tt, float4 dl, float* out, uint32_t steps) {
-    float h0 = a0 < e0 ? lds_f32(a0) : AVFS_INF;
-    float h1 = a1 < e1 ? lds_f32(a1) : AVFS_INF;
-    a0 += 4;
-    a1 += 4;
-    float tl = -AVFS_INF;
-    uint32_t cnt = 0, it = 0;
-    asm volatile(
-        "{\n"
-        ".reg .pred p, ok, live, y1, chg, canc, push, more;\n"
-        ".reg .f32 t, nx, dA, dB, d, co;\n"
-        ".reg .b32 a, e, y, sh;\n"
-        ".reg .b64 ad;\n"
-        "MERGE2_%=:\n"
-        "setp.lt.f32 p, %1, %0;\n"
-        "min.f32 t, %0, %1;\n"
-        "selp.b32 a, %3, %2, p;\n"
-        "selp.b32 e, %10, %9, p;\n"
-        "setp.lt.u32 ok, a, e;\n"
-        "mov.f32 nx, 0f7F800000;\n"
-        "@ok ld.shared.f32 nx, [a];\n"
-        "@p add.u32 %3, %3, 4;\n"
-        "@!p add.u32 %2, %2, 4;\n"
-        "@p mov.f32 %1, nx;\n"
-        "@!p mov.f32 %0, nx;\n"
-        "setp.lt.f32 live, t, 0f7F800000;\n"
-        "selp.b32 sh, 2, 1, p;\n"
-        "@live xor.b32 %4, %4, sh;\n"
-        "shr.u32 y, %11, %4;\n"
-        "and.b32 y, y, 1;\n"
-        "setp.ne.u32 y1, y, 0;\n"
-        "selp.f32 dA, %15, %14, y1;\n"
-        "selp.f32 dB, %13, %12, y1;\n"
-        "selp.f32 d, dA, dB, p;\n"
-        "add.rn.f32 co, t, d;\n"
-        "setp.ne.and.u32 chg, y, %5, live;\n"
-        "setp.gt.and.f32 canc, %6, t, chg;\n"
-        "setp.le.and.f32 push, %6, t, chg;\n"
-        "mul.wide.u32 ad, %7, 4;\n"
-        "add.u64 ad, ad, %16;\n"
-        "@push st.global.cg.f32 [ad], co;\n"
-        "@push add.u32 %7, %7, 1;\n"
-        "@canc sub.u32 %7, %7, 1;\n"
-        "@push mov.f32 %6, co;\n"
-        "@canc mov.f32 %6, 0fFF800000;\n"
-        "mov.b32 %5, y;\n"
-        "add.u32 %8, %8, 1;\n"
-        "setp.lt.u32 more, %8, %17;\n"
-        "@more bra MERGE2_%=;\n"
-        "}\n"
-        : "+f"(h0), "+f"(h1), "+r"(a0), "+r"(a1), "+r"(bits), "+r"(proj), "+f"(tl), "+r"(cnt), "+r"(it)
-        : "r"(e0), "r"(e1), "r"(tt), "f"(dl.x), "f"(dl.y), "f"(dl.z), "f"(dl.w), "l"(out), "r"(steps)
-        : "memory");
-    return cnt;
+// Bit-parallel gate evaluation over the 32 slots of a group.  KM = number of
+// input positions evaluated (2 or 4; missing inputs have X = E = 0).
+//   y0   = TT(X)                           (value before t = 0)
+//   A    = can0 & can1: slots whose output is not constant over the inputs'
+//          possible values (X fixed where E = 0, free where E = 1)
+template <int KM>
+__device__ __forceinline__ void eval_masks(uint32_t tt, const uint32_t (&X)[4], const uint32_t (&E)[4], uint32_t& y0,
+                                           uint32_t& A) {
+    uint32_t lf[1 << KM];
+#pragma unroll
+    for (int b = 0; b < (1 << KM); ++b) lf[b] = tt_leaf(tt, b);
+    uint32_t n[1 << KM];
+#pragma unroll
+    for (int b = 0; b < (1 << KM); ++b) n[b] = lf[b];
+#pragma unroll
+    for (int q = 0; q < KM; ++q)
+#pragma unroll
+        for (int b = 0; b < (1 << (KM - 1 - q)); ++b) n[b] = mux(X[q], n[2 * b + 1], n[2 * b]);
+    y0 = n[0];
+    uint32_t cons[1 << KM];
+    cons[0] = E[0] | ~X[0];
+    cons[1] = E[0] | X[0];
+#pragma unroll
+    for (int q = 1; q < KM; ++q) {
+        const uint32_t l0 = E[q] | ~X[q], l1 = E[q] | X[q];
+#pragma unroll
+        for (int b = (1 << q) - 1; b >= 0; --b) {
+            cons[b + (1 << q)] = cons[b] & l1;
+            cons[b] = cons[b] & l0;
+        }
+    }
+    uint32_t c0 = 0, c1 = 0;
+#pragma unroll
+    for (int b = 0; b < (1 << KM); ++b) {
+        c1 |= cons[b] & lf[b];
+        c0 |= cons[b] & ~lf[b];
+    }
+    A = c0 & c1;
 }
 
-template <int K, bool STAGED>
-__device__ __forceinline__ uint32_t merge_slot(const MergeIn& M, float* out, uint32_t steps) {
-    typedef typename EvAddr<STAGED>::T A;
-    uint32_t bits = M.bits, proj = M.proj;
-    const uint32_t tt = M.tt;
-    uint32_t cnt = 0;                            // outputs kept so far (only the last can be cancelled)
-    float tl = -AVFS_INF;
-    auto step = [&](float t, bool live, uint32_t y, float d) {
+__device__ __forceinline__ void poison_bit(const SweepParams& p, int64_t gi, uint32_t sig) {
+    const uint64_t gbit = (uint64_t)gi * (uint32_t)p.n_gates + (sig - (uint32_t)p.n_pi);
+    atomicOr(p.pois + (gbit >> 5), 1u << (gbit & 31u));
+}
+
+// Phase A for gates g0 .. g0 + nb - 1 (nb <= QN); returns the number queued.
+template <bool RERUN>
+__device__ __forceinline__ int phase_a(const SweepParams& p, const Grp& G, int g0, int nb, uint32_t q_s,
+                                       const float4* __restrict__ dt, int lane) {
+    const bool on = lane < nb;
+    const int g = g0 + (on ? lane : 0);
+    const uint4* gd = reinterpret_cast<const uint4*>(p.gates);
+    uint4 d0 = make_uint4(0, 0, 0, 0), d1 = make_uint4(0, 0, 0, 0);
+    float4 dl0 = make_float4(0, 0, 0, 0), dl1 = dl0;
+    if (on) {
+        d0 = __ldg(gd + 2 * g);
+        d1 = __ldg(gd + 2 * g + 1);
+        dl0 = __ldg(dt + 2 * g);
+        dl1 = __ldg(dt + 2 * g + 1);
+    }
+    const uint32_t tt = d1.z & 0xffffu, K = on ? (d1.z >> 16) & 0xffu : 0u;
+    const uint32_t loc[4] = {d0.x, d0.y, d0.z, d0.w};
+    uint32_t X[4], E[4], AQ[4], M[4];
+#pragma unroll
+    for (int q = 0; q < 4; ++q) {
+        X[q] = E[q] = AQ[q] = M[q] = 0;
+        if ((uint32_t)q < K) {
+            const uint32_t id = loc[q] & LOC_ID;
+            if ((loc[q] & LOC_KIND) == LOC_PI) {       // reading C2: one event at t = 0 iff p1 != p2
+                const int64_t ix = (int64_t)id * p.n_pw + G.pw;
+                const uint32_t w1 = __ldg(p.p1t + ix), w2 = __ldg(p.p2t + ix);
+                X[q] = w1;
+                E[q] = AQ[q] = (w1 ^ w2) & G.vmask;
+                M[q] = (uint32_t)__popc(E[q]);
+            } else {
+                const uint4 r = __ldcg(G.rec + (size_t)id * G.rstride);
+                X[q] = r.x;
+                E[q] = r.y;
+                AQ[q] = r.z;
+                M[q] = r.w;
+            }
+        }
+    }
+    uint32_t y0, A;
+    if (__any_sync(FULL, K > 2)) eval_masks<4>(tt, X, E, y0, A);
+    else eval_masks<2>(tt, X, E, y0, A);
+    const uint32_t U = (M[0] & REC_NTOT) + (M[1] & REC_NTOT) + (M[2] & REC_NTOT) + (M[3] & REC_NTOT);
+    bool pois = on && ((M[0] | M[1] | M[2] | M[3]) & REC_POISON);
+    bool own = false, spilled = false;
+    bool active = on && !pois && A != 0;
+    bool counted = true;                      // activity of this (group, gate) not yet counted
+    const uint32_t sig = d1.y;
+    if (RERUN && on) {
+        const uint64_t b = (uint64_t)__ldg(p.prev_idx + (G.gi - 0)) * (uint32_t)p.n_gates + (sig - (uint32_t)p.n_pi);
+        counted = (__ldg(p.pois_prev + (b >> 5)) >> (b & 31u)) & 1u;
+    }
+    uint8_t* oreg = G.row + (size_t)d1.x * G.stride;
+    unsigned long long tb = 0;
+    if (active) {
+        if (U >= OFF_LIMIT) {
+            own = true;
+        } else if (U <= (uint32_t)p.W) {
+            tb = reinterpret_cast<unsigned long long>(oreg + REG_TIMES);
+        } else {
+            const unsigned long long need = (U + 3u) & ~3u;
+            const unsigned long long wb = atomicAdd(p.spill_top, need);
+            if (wb + need > p.spill_words) {
+                own = true;
+            } else {
+                tb = reinterpret_cast<unsigned long long>(p.spill + wb);
+                __stcg(reinterpret_cast<unsigned long long*>(oreg + REG_SPILLPTR), tb);
+                spilled = true;
+            }
+        }
+        if (own) {
+            pois = true;
+            active = false;
+        }
+    }
+    if (on && !active) {                      // finished here: constant output, or poisoned
+        __stcg(G.rec + (size_t)d1.x * G.rstride, make_uint4(y0, 0u, 0u, pois ? REC_POISON : 0u));
+        if (pois) {
+            if (!RERUN || counted) poison_bit(p, G.gi, sig);
+            if (own) p.ovf[G.gi] = 1;
+        }
+    }
+    const uint32_t bal = __ballot_sync(FULL, active);
+    if (active) {
+        const uint32_t qe = q_s + 4u * QW * (uint32_t)__popc(bal & lanemask_lt());
+        sts_u32x4(qe + 4 * Q_TTK, make_uint4(d1.z, sig, d1.x, y0));
+        sts_u32x4(qe + 4 * Q_A, make_uint4(A, 0u, 0u, 0u));
+        sts_u32x4(qe + 4 * Q_TB, make_uint4((uint32_t)tb, (uint32_t)(tb >> 32), 0u,
+                                            (counted ? QF_COUNT : 0u) | (spilled ? QF_SPILL : 0u) | (d1.w << 8)));
+        sts_u32x4(qe + 4 * Q_X, make_uint4(X[0], X[1], X[2], X[3]));
+        sts_u32x4(qe + 4 * Q_E, make_uint4(E[0], E[1], E[2], E[3]));
+        sts_u32x4(qe + 4 * Q_AQ, make_uint4(AQ[0], AQ[1], AQ[2], AQ[3]));
+        sts_u32x4(qe + 4 * Q_LOC, make_uint4(loc[0], loc[1], loc[2], loc[3]));
+#pragma unroll
+        for (int q = 0; q < 4; ++q) {
+            unsigned long long itb = reinterpret_cast<unsigned long long>(p.zero);
+            if ((uint32_t)q < K && (loc[q] & LOC_KIND) != LOC_PI) {
+                const uint8_t* r = G.row + (size_t)(loc[q] & LOC_ID) * G.stride;
+                itb = (M[q] & REC_SPILL) ? __ldcg(reinterpret_cast<const unsigned long long*>(r + REG_SPILLPTR))
+                                         : reinterpret_cast<unsigned long long>(r + REG_TIMES);
+            }
+            sts_u64(qe + 4 * Q_ITB + 8 * q, itb);
+        }
+        sts_f32x4(qe + 4 * Q_DLY, dl0);
+        sts_f32x4(qe + 4 * Q_DLY + 16, dl1);
+    }
+    return __popc(bal);
+}
+
+// One filter step (readings C3, C4): y is the gate's value after the input
+// event at t; a change either cancels the pending last output (it lies after
+// t) or pushes t + d.
+struct Filt {
+    uint32_t proj, cnt;
+    float tl;
+    __device__ __forceinline__ void step(float t, bool live, uint32_t y, float d, float* out) {
         const float co = t + d;
         const bool change = live && y != proj;
         const bool cancel = change && tl > t;
@@ -259,533 +384,288 @@ __device__ __forceinline__ uint32_t merge_slot(const MergeIn& M, float* out, uin
         cnt = cnt + (push ? 1u : 0u) - (cancel ? 1u : 0u);
         tl = push ? co : (cancel ? -AVFS_INF : tl);
         proj = y;
-    };
-    if (K == 1) {
-        A a = (A)M.ev[0];
-        const A e = a + 4 * (uint32_t)M.n[0];
-        float h = a < e ? ld_ev<STAGED>(a) : AVFS_INF;
-#pragma unroll 1
-        for (uint32_t it = 0; it < steps; ++it) {
-            const float t = h;
-            a += 4;
-            h = a < e ? ld_ev<STAGED>(a) : AVFS_INF;
-            const bool live = t < AVFS_INF;
-            bits ^= live ? 1u : 0u;
-            const uint32_t y = (tt >> bits) & 1u;
-            step(t, live, y, y ? M.d01.y : M.d01.x);
-        }
-    } else if (K == 2 && STAGED && AVFS_PTX_MERGE) {
-        return steps ? merge2_smem((uint32_t)M.ev[0], (uint32_t)M.ev[0] + 4 * (uint32_t)M.n[0], (uint32_t)M.ev[1],
-                                   (uint32_t)M.ev[1] + 4 * (uint32_t)M.n[1], bits, proj, tt, M.d01, out, steps)
-                     : 0u;
-    } else if (K == 2 && !STAGED) {
-        // lists in L2: each list keeps its head and the next two elements in
-        // registers, so the load feeding a comparison was issued >= 2 advances
-        // of that list earlier
-        A a0 = (A)M.ev[0], a1 = (A)M.ev[1];
-        const A e0 = a0 + 4 * (uint32_t)M.n[0], e1 = a1 + 4 * (uint32_t)M.n[1];
-        float h0 = a0 < e0 ? ld_ev<false>(a0) : AVFS_INF, g0 = a0 + 4 < e0 ? ld_ev<false>(a0 + 4) : AVFS_INF,
-              f0 = a0 + 8 < e0 ? ld_ev<false>(a0 + 8) : AVFS_INF;
-        float h1 = a1 < e1 ? ld_ev<false>(a1) : AVFS_INF, g1 = a1 + 4 < e1 ? ld_ev<false>(a1 + 4) : AVFS_INF,
-              f1 = a1 + 8 < e1 ? ld_ev<false>(a1 + 8) : AVFS_INF;
-        a0 += 12;
-        a1 += 12;
-#pragma unroll 1
-        for (uint32_t it = 0; it < steps; ++it) {
-            const bool p = h1 < h0;             // ties: pin 0 first
-            const float t = fminf(h0, h1);
-            const A a = p ? a1 : a0;
-            const float nx = a < (p ? e1 : e0) ? ld_ev<false>(a) : AVFS_INF;
-            if (p) {
-                h1 = g1; g1 = f1; f1 = nx; a1 += 4;
-            } else {
-                h0 = g0; g0 = f0; f0 = nx; a0 += 4;
-            }
-            const bool live = t < AVFS_INF;
-            bits ^= live ? (p ? 2u : 1u) : 0u;
-            const uint32_t y = (tt >> bits) & 1u;
-            step(t, live, y, p ? (y ? M.d01.w : M.d01.z) : (y ? M.d01.y : M.d01.x));
-        }
-    } else if (K == 2) {
-        A a0 = (A)M.ev[0], a1 = (A)M.ev[1];
-        const A e0 = a0 + 4 * (uint32_t)M.n[0], e1 = a1 + 4 * (uint32_t)M.n[1];
-        float h0 = a0 < e0 ? ld_ev<STAGED>(a0) : AVFS_INF;
-        float h1 = a1 < e1 ? ld_ev<STAGED>(a1) : AVFS_INF;
-        a0 += 4;
-        a1 += 4;
-#pragma unroll 1
-        for (uint32_t it = 0; it < steps; ++it) {
-            const bool p = h1 < h0;             // ties: pin 0 first
-            const float t = fminf(h0, h1);
-            const A a = p ? a1 : a0;
-            const float nx = a < (p ? e1 : e0) ? ld_ev<STAGED>(a) : AVFS_INF;
-            h1 = p ? nx : h1;
-            h0 = p ? h0 : nx;
-            a1 = p ? a + 4 : a1;
-            a0 = p ? a0 : a + 4;
-            const bool live = t < AVFS_INF;
-            bits ^= live ? (p ? 2u : 1u) : 0u;
-            const uint32_t y = (tt >> bits) & 1u;
-            step(t, live, y, p ? (y ? M.d01.w : M.d01.z) : (y ? M.d01.y : M.d01.x));
-        }
-    } else {
-        float h[K];
-        A a[K], e[K];
-#pragma unroll
-        for (int q = 0; q < K; ++q) {
-            a[q] = (A)M.ev[q];
-            e[q] = a[q] + 4 * (uint32_t)M.n[q];
-            h[q] = a[q] < e[q] ? ld_ev<STAGED>(a[q]) : AVFS_INF;
-            a[q] += 4;
-        }
-#pragma unroll 1
-        for (uint32_t it = 0; it < steps; ++it) {
-            float t = h[0];
-            int pm = 0;
-#pragma unroll
-            for (int q = 1; q < K; ++q) {
-                const bool lt = h[q] < t;
-                t = lt ? h[q] : t;
-                pm = lt ? q : pm;
-            }
-            A ap = a[0], ep = e[0];
-#pragma unroll
-            for (int q = 1; q < K; ++q)
-                if (pm == q) { ap = a[q]; ep = e[q]; }
-            const float nx = ap < ep ? ld_ev<STAGED>(ap) : AVFS_INF;
-#pragma unroll
-            for (int q = 0; q < K; ++q)
-                if (pm == q) { h[q] = nx; a[q] = ap + 4; }
-            const bool live = t < AVFS_INF;
-            bits ^= live ? (1u << pm) : 0u;
-            const uint32_t y = (tt >> bits) & 1u;
-            step(t, live, y, lds_f32(M.dly_s + 8 * pm + 4 * y));
-        }
     }
-    return cnt;
+};
+
+// Merge of at most two sorted lists (pins p0 < p1; list 1 may be empty), the
+// next element of each list already loaded (one element of lookahead).
+__device__ __forceinline__ uint32_t merge_two(const float* a0, int n0, const float* a1, int n1, uint32_t bits,
+                                              uint32_t tm0, uint32_t tm1, uint32_t proj, uint32_t tt, float4 dl,
+                                              float* out, uint32_t steps) {
+    float h0 = n0 > 0 ? ld_f32(a0) : AVFS_INF, g0 = n0 > 1 ? ld_f32(a0 + 1) : AVFS_INF;
+    float h1 = n1 > 0 ? ld_f32(a1) : AVFS_INF, g1 = n1 > 1 ? ld_f32(a1 + 1) : AVFS_INF;
+    a0 += 2;
+    a1 += 2;
+    n0 -= 2;
+    n1 -= 2;
+    Filt F{proj, 0u, -AVFS_INF};
+#pragma unroll 1
+    for (uint32_t it = 0; it < steps; ++it) {
+        const bool p = h1 < h0;                       // ties: the lower pin first (reading C5)
+        const float t = fminf(h0, h1);
+        const float* a = p ? a1 : a0;
+        const float nx = (p ? n1 : n0) > 0 ? ld_f32(a) : AVFS_INF;
+        h1 = p ? g1 : h1;
+        g1 = p ? nx : g1;
+        h0 = p ? h0 : g0;
+        g0 = p ? g0 : nx;
+        a1 += p ? 1 : 0;
+        n1 -= p ? 1 : 0;
+        a0 += p ? 0 : 1;
+        n0 -= p ? 0 : 1;
+        const bool live = t < AVFS_INF;
+        bits ^= live ? (p ? tm1 : tm0) : 0u;
+        const uint32_t y = (tt >> bits) & 1u;
+        F.step(t, live, y, p ? (y ? dl.w : dl.z) : (y ? dl.y : dl.x), out);
+    }
+    return F.cnt;
 }
 
-template <int K, bool RERUN>
-__device__ __forceinline__ void eval_gate(const SweepParams& p, const Env& E, const uint4 ins, const uint4 hd,
-                                          const Staged& S) {
-    const int lane = E.lane;
-    const uint32_t out_loc = hd.x, sig = hd.y;
-    const uint32_t tt = hd.z & 0xffffu;
-    const uint32_t in_loc[KMAX] = {ins.x, ins.y, ins.z, ins.w};
-    uint32_t hw[KMAX];
+// Merge of up to four sorted lists (list q = pin q, n[q] = 0 if unused);
+// delays read from the queue entry.
+__device__ __forceinline__ uint32_t merge_four(const float* const (&a_in)[4], const int (&n_in)[4], uint32_t bits,
+                                               uint32_t proj, uint32_t tt, uint32_t dly_s, float* out, uint32_t steps) {
+    float h[4];
+    const float* a[4];
+    int n[4];
 #pragma unroll
-    for (int q = 0; q < K; ++q)
-        hw[q] = S.hdr ? lds_u32(S.hdr_s + 128 * q + 4 * lane)
-                      : __ldcg(reinterpret_cast<const uint32_t*>(region(in_loc[q], E)) + lane);
-    int n[KMAX] = {0, 0, 0, 0};
-    uint32_t bits = 0, orh = 0;
-#pragma unroll
-    for (int q = 0; q < K; ++q) {
-        n[q] = (int)(hw[q] & HDR_N);
-        bits |= ((hw[q] >> HDR_INIT_SHIFT) & 1u) << q;
-        orh |= hw[q];
+    for (int q = 0; q < 4; ++q) {
+        a[q] = a_in[q];
+        n[q] = n_in[q];
+        h[q] = n[q] > 0 ? ld_f32(a[q]) : AVFS_INF;
+        a[q] += 1;
+        n[q] -= 1;
     }
-    if (K == 2 && AVFS_PRUNE) {                          // table lookup (host-built, GateDesc.obs)
-        const uint32_t st = (n[0] == 0 ? 1u : 0u) | (n[1] == 0 ? 2u : 0u);
-        const uint32_t ob = hd.w >> (2 * (st | ((bits & st) << 2)));
-        n[0] = (ob & 1u) ? n[0] : 0;
-        n[1] = (ob & 2u) ? n[1] : 0;
-    } else if (K >= 3 && AVFS_PRUNE) {
-        // Events this slot's output cannot observe: with the stable inputs
-        // (no event) at their values, the truth table restricted to the
-        // remaining minterms does not depend on input q (e.g. AND with another
-        // input stable at 0).  Such events never change the evaluated output
-        // (reading C4), so they are dropped from the merge -- fewer merge
-        // steps and tighter output offsets, identical waveforms.
-        constexpr uint32_t POS[4] = {0xAAAAu, 0xCCCCu, 0xF0F0u, 0xFF00u};
-        uint32_t mt = 0xFFFFu >> (16 - (1 << K));       // minterms consistent with the stable inputs
+    Filt F{proj, 0u, -AVFS_INF};
+#pragma unroll 1
+    for (uint32_t it = 0; it < steps; ++it) {
+        float t = h[0];
+        int pm = 0;
 #pragma unroll
-        for (int q = 0; q < K; ++q)
-            if (n[q] == 0) mt &= ((bits >> q) & 1u) ? POS[q] : ~POS[q];
-#pragma unroll
-        for (int q = 0; q < K; ++q)
-            if ((((tt >> (1 << q)) ^ tt) & mt & ~POS[q]) == 0) n[q] = 0;
-    }
-    int m = 0;
-#pragma unroll
-    for (int q = 0; q < K; ++q) m += n[q];
-    const uint32_t y0 = (tt >> bits) & 1u;
-    uint8_t* ro = region(out_loc, E);
-    uint32_t* ro_hdr = reinterpret_cast<uint32_t*>(ro);
-    auto poison = [&](bool own) {
-        __stcg(ro_hdr + lane, HDR_POISON | (y0 << HDR_INIT_SHIFT));
-        if (lane == 0) {            // poison bitmap bit of this (slot group, gate) in this round
-            const uint32_t gi = lds_u32(S.grp_s);
-            const uint64_t gbit = (uint64_t)gi * (uint32_t)p.n_gates + (sig - (uint32_t)p.n_pi);
-            atomicOr(p.pois + (gbit >> 5), 1u << (gbit & 31u));
-            if (own) p.ovf[gi] = 1;
+        for (int q = 1; q < 4; ++q) {
+            const bool lt = h[q] < t;
+            t = lt ? h[q] : t;
+            pm = lt ? q : pm;
         }
-    };
-    // one warp reduction: upstream poison, any input event
-    const uint32_t R = __reduce_or_sync(FULL, (orh & HDR_POISON) | (m != 0 ? 1u : 0u));
-    if (R & HDR_POISON) {                               // upstream overflow: nothing valid here
-        poison(false);
-        return;
-    }
-    if (!(R & 1u)) {                                    // no input event in any slot: constant output
-        __stcg(ro_hdr + lane, y0 << HDR_INIT_SHIFT);
-        return;
-    }
-    const uint32_t incl = warp_incl_scan((uint32_t)m, lane);
-    const uint32_t total_in = __shfl_sync(FULL, incl, 31);
-    const uint32_t base = incl - (uint32_t)m;
-    const uint32_t maxm = __reduce_max_sync(FULL, (uint32_t)m);
-    // the inputs' events bound the outputs (reading C17): header fields must
-    // hold them; more than W go to the spill heap, and if the heap is
-    // exhausted the slot group is rerun
-    if (total_in > HDR_OFF || maxm > HDR_N) {
-        poison(true);
-        return;
-    }
-    float* out = reinterpret_cast<float*>(ro + 128) + base;
-    uint32_t hdr_part = (base << HDR_OFF_SHIFT) | (y0 << HDR_INIT_SHIFT);
-    if (total_in > (uint32_t)p.W) {
-        const uint32_t need = (total_in + 3u) & ~3u;
-        unsigned long long wb = 0;
-        if (lane == 0) wb = atomicAdd(p.spill_top, (unsigned long long)need);
-        wb = __shfl_sync(FULL, wb, 0);
-        if (wb + need > p.spill_words) {
-            poison(true);
-            return;
-        }
-        if (lane == 0) __stcg(reinterpret_cast<unsigned long long*>(ro + 128), reinterpret_cast<unsigned long long>(p.spill + wb));
-        out = p.spill + wb + base;
-        hdr_part |= HDR_SPILL;
-    }
-    MergeIn M;
-    M.bits = bits;
-    M.proj = y0;
-    M.tt = tt;
-    M.dly_s = S.dly_s;
-    if (K <= 2) M.d01 = lds_f32x4(S.dly_s);
+        const float* ap = a[0];
+        int np = n[0];
 #pragma unroll
-    for (int q = 0; q < KMAX; ++q) M.n[q] = n[q];
-    uint32_t my_n;
-    if (S.ev) {
+        for (int q = 1; q < 4; ++q)
+            if (pm == q) { ap = a[q]; np = n[q]; }
+        const float nx = np > 0 ? ld_f32(ap) : AVFS_INF;
 #pragma unroll
-        for (int q = 0; q < K; ++q)
-            M.ev[q] = S.ev_s[0] + (uint32_t)(4 * EV_STAGE / (K > 2 ? 4 : K)) * q + 4 * ((hw[q] >> HDR_OFF_SHIFT) & HDR_OFF);
-        my_n = merge_slot<K, true>(M, out, maxm);
-    } else {
-#pragma unroll
-        for (int q = 0; q < K; ++q)
-            M.ev[q] = reinterpret_cast<uint64_t>(ev_base(region(in_loc[q], E), hw[q])) + 4 * ((hw[q] >> HDR_OFF_SHIFT) & HDR_OFF);
-        my_n = merge_slot<K, false>(M, out, maxm);
+        for (int q = 0; q < 4; ++q)
+            if (pm == q) { h[q] = nx; a[q] = ap + 1; n[q] = np - 1; }
+        const bool live = t < AVFS_INF;
+        bits ^= live ? (1u << pm) : 0u;
+        const uint32_t y = (tt >> bits) & 1u;
+        F.step(t, live, y, lds_f32(dly_s + 8 * pm + 4 * y), out);
     }
-    __stcg(reinterpret_cast<uint32_t*>(region(out_loc, E)) + lane, my_n | hdr_part);
-    // activity (reading C15) and latest PO arrival: counted once per
-    // slot across rerun rounds -- only where the previous round poisoned this
-    // gate of this slot group (pass 0: everywhere)
-    bool prev = true;
-    if (RERUN) {
-        const uint64_t b = (uint64_t)__ldg(p.prev_idx + p.i_base + E.i) * (uint32_t)p.n_gates + (sig - (uint32_t)p.n_pi);
-        prev = (__ldg(p.pois_prev + (b >> 5)) >> (b & 31u)) & 1u;
-    }
-    if (prev) {
-        const uint32_t total = __reduce_add_sync(FULL, my_n);
-        if (lane == 0 && total) atomicAdd(E.act_kv + (size_t)sig * (uint32_t)p.n_vdd, (unsigned long long)total);
-        if (hd.z & (1u << 24)) {
-            const float last = my_n ? __ldcg(out + my_n - 1) : 0.0f;
-            const uint32_t mx = __reduce_max_sync(FULL, __float_as_uint(last));
-            if (lane == 0 && mx) atomicMax(p.latest + E.kv, mx);
-        }
-    }
+    return F.cnt;
 }
 
+// Phase B over the nq queued gates, then their records.
 template <bool RERUN>
-__device__ __forceinline__ void eval_dispatch(const SweepParams& p, const Env& E, const uint4 ins, const uint4 hd,
-                                              const Staged& S) {
-    // compare chain in order of frequency (2-input cells first) instead of a
-    // jump table
-    const uint32_t k = (hd.z >> 16) & 0xffu;
-    if (k == 2) eval_gate<2, RERUN>(p, E, ins, hd, S);
-    else if (k == 1) eval_gate<1, RERUN>(p, E, ins, hd, S);
-    else if (k == 3) eval_gate<3, RERUN>(p, E, ins, hd, S);
-    else eval_gate<4, RERUN>(p, E, ins, hd, S);
-}
-
-__device__ __forceinline__ void slot_group(const SweepParams& p, int64_t i, int lane, Env& E) {
-    const int64_t sw = p.sw_list ? (int64_t)p.sw_list[i] : p.sw_first + i;
-    E.kv = (int)(sw / p.n_pw);
-    E.i = i;
-    E.lane = lane;
-    E.act_kv = p.act + E.kv;
-    E.row = p.arena + (p.i_base + i) * p.region_bytes;
-}
-
-// Per-warp shared memory (words): two descriptor windows of DW gates
-// (GateDesc 8 words each, then the gates' delays 8 words each), a header ring
-// 4 x 128 (4 input rows of 32 header words), an event ring 2 x EV_STAGE
-// (input q of a K-input gate owns EV_STAGE / K' words, K' = K rounded up to a
-// power of two), staged flags.
-constexpr int DW = 16;                                // gates per descriptor window
-constexpr int OFF_DESC = 0, OFF_HDR = OFF_DESC + 2 * 16 * DW, OFF_EV = OFF_HDR + 4 * 128,
-              OFF_META = OFF_EV + 2 * EV_STAGE;
-constexpr int WARP_SMEM_WORDS = OFF_META + 4;
-constexpr int LEVEL_SMEM_WORDS = 12;                  // delays of the current gate, group index
-
-__device__ __forceinline__ float* warp_smem(int warp, int words) {
-    extern __shared__ __align__(16) float smem[];
-    return smem + 4 + (size_t)warp * words;
-}
-
-// Persistent level sweep (pass 0): one CTA owns one 32-slot group at a time
-// and walks all levels with a CTA barrier between levels.  Warp w
-// evaluates a contiguous block of each level's gates through a software
-// pipeline of asynchronous copies into shared memory (cp.async): descriptors
-// and delays arrive 16 gates at a time; at gate j the warp fetches the input
-// header rows of gate j+2 and the input event lists of gate j+1, so the
-// evaluation of gate j never waits for DRAM.  Event lists larger than the
-// stage are read from L2 by the evaluation instead.
-__global__ void __launch_bounds__(AVFS_SWEEP_THREADS, AVFS_SWEEP_MINB) sweep_kernel(const SweepParams p) {
-    const int lane = threadIdx.x & 31;
-    const int warp = threadIdx.x >> 5;
-    const int nw = blockDim.x >> 5;
-    Env E;
-    // shared addresses only (no generic pointers into the warp's area)
-    const uint32_t ws_s = smem_u32(warp_smem(0, 0)) + 4u * (uint32_t)(warp * WARP_SMEM_WORDS);
-    const uint32_t s_desc = ws_s + 4 * OFF_DESC, s_hdr = ws_s + 4 * OFF_HDR, s_evr = ws_s + 4 * OFF_EV;
-    const uint32_t s_grp = ws_s + 4 * (OFF_META + 2);
-    E.stride = (uint32_t)(p.pin_n_sw * p.region_bytes);
-    const uint4* gd = reinterpret_cast<const uint4*>(p.gates);
-    // narrow netlists: the CTA walks G slot groups at once, nw / G warps each
-    const int G = p.grp_per_cta, wpg = nw / G;
-    const int sg = warp / wpg, wl = warp % wpg;
-    for (int64_t i0 = (int64_t)blockIdx.x * G; i0 < p.n_sw; i0 += (int64_t)gridDim.x * G) {
-        const int64_t i = i0 + sg;
-        const bool valid = i < p.n_sw;                 // idle warps still meet every level barrier
-        slot_group(p, valid ? i : i0, lane, E);
-        __syncwarp();
-        if (lane == 0) sts_u32(s_grp, (uint32_t)(p.i_base + (valid ? i : i0)));
-        const float4* dt = p.dtab + (int64_t)E.kv * p.n_gates * 2;
-        for (int L = 0; L < p.depth; ++L) {
-            const int ls = __ldg(p.level_ptr + L), le = __ldg(p.level_ptr + L + 1);
-            const int B = (le - ls + wpg - 1) / wpg;
-            const int g0 = ls + wl * B;
-            const int nj = valid ? max(0, min(B, le - g0)) : 0;
-            // descriptor window k (gates g0 + 16k ..): lane copies 16 B of the
-            // descriptors (lanes 0..31 = 16 gates x 2) and 16 B of the delays
-            // descriptor ring of 2 DW gates (32 B each), delay ring behind it
-            auto issue_win = [&](int k) {
-                const int g = g0 + DW * k + (lane >> 1);
-                const uint32_t w = s_desc + 32 * ((uint32_t)(DW * k + (lane >> 1)) & (2 * DW - 1)) + 16 * (lane & 1);
-                if (g < le) {
-                    cp_async16(w, gd + 2 * g + (lane & 1));
-                    cp_async16(w + 32 * 2 * DW, dt + 2 * g + (lane & 1));
-                }
-            };
-            auto desc_at = [&](uint32_t j) { return s_desc + 32 * (j & (2 * DW - 1)); };
-            auto issue_hdr = [&](uint32_t j) {
-                const uint32_t d = desc_at(j);
-                const uint32_t q = (uint32_t)lane >> 3;
-                if (q < ((lds_u32(d + 24) >> 16) & 0xffu))
-                    cp_async16(s_hdr + 512 * (j & 3) + 128 * q + 16 * (lane & 7),
-                               region(lds_u32(d + 4 * q), E) + 16 * (lane & 7));
-            };
-            // input q's events (extent = lane 31's offset + count) -> slot q of
-            // the stage (EV_STAGE / K' words, 32 / K' lanes per input, <= 2
-            // chunks of 16 B per lane); staged only if every input fits
-            bool staged_next = false, staged_cur = false;
-            auto issue_ev = [&](uint32_t j) {
-                const uint32_t d = desc_at(j);
-                const uint32_t k = (lds_u32(d + 24) >> 16) & 0xffu;
-                const uint32_t sh = k > 2 ? 2u : (k > 1 ? 1u : 0u);      // log2 K'
-                const uint32_t q = (uint32_t)lane >> (5 - sh), sub = (uint32_t)lane & (31u >> sh);
-                uint32_t c = 0, w = 0;
-                if (q < k) {
-                    w = lds_u32(s_hdr + 512 * (j & 3) + 128 * q + 124);
-                    c = (((w >> HDR_OFF_SHIFT) & HDR_OFF) + (w & HDR_N) + 3) >> 2;
-                }
-                const uint32_t cap = (uint32_t)(EV_STAGE / 4) >> sh;   // chunks per input
-                const bool staged = __all_sync(FULL, c <= cap);
-                staged_next = staged;
-                if (staged && sub < c) {
-                    const uint8_t* src = ev_base(region(lds_u32(d + 4 * q), E), w) + 16 * sub;
-                    const uint32_t dst = s_evr + 4 * EV_STAGE * (j & 1) + (4 * EV_STAGE >> sh) * q + 16 * sub;
-                    cp_async16(dst, src);
-                    const uint32_t st = 512u >> sh;                     // bytes covered by one pass of the lanes
-                    if (sub + (32u >> sh) < c) cp_async16(dst + st, src + st);
-                }
-            };
-            if (nj > 0) {
-                // prologue: descriptor windows 0, 1; header rows 0, 1; events of gate 0
-                issue_win(0);
-                if (nj > DW) issue_win(1);
-                cp_async_commit();
-                cp_async_wait_all();
-                __syncwarp();
-                issue_hdr(0);
-                if (nj > 1) issue_hdr(1);
-                cp_async_commit();
-                cp_async_wait_all();
-                __syncwarp();
-                issue_ev(0);
-                staged_cur = staged_next;
-                cp_async_commit();
-                const uint32_t nju = (uint32_t)nj;
-#pragma unroll 1
-                for (uint32_t j = 0; j < nju; ++j) {
-                    cp_async_wait_all();
-                    __syncwarp();
-                    if (j % DW == 0 && j > 0 && j + DW < nju) issue_win((int)(j / DW) + 1);
-                    if (j + 2 < nju) issue_hdr(j + 2);
-                    const bool st_j = staged_cur;
-                    if (j + 1 < nju) issue_ev(j + 1);
-                    staged_cur = staged_next;
-                    cp_async_commit();
-                    const uint32_t d = desc_at(j);
-                    const uint4 dv0 = lds_u32x4(d), dv1 = lds_u32x4(d + 16);
-                    Staged S;
-                    S.hdr = true;
-                    S.hdr_s = s_hdr + 512 * (j & 3);
-                    S.ev = st_j;
-                    S.dly_s = d + 32 * 2 * DW;
-                    S.grp_s = s_grp;
-                    S.ev_s[0] = s_evr + 4 * EV_STAGE * (j & 1);
-                    eval_dispatch<false>(p, E, dv0, dv1, S);
+__device__ __forceinline__ void phase_b(const SweepParams& p, const Grp& G, int nq, uint32_t q_s, uint32_t it_s,
+                                        int lane, unsigned long long& enc) {
+    // item list: entry e's slots in ascending order, entries in queue order
+    uint32_t T = 0;
+    for (int e = 0; e < nq; ++e) {
+        const uint32_t A = lds_u32(q_s + 4u * (QW * e + Q_A));
+        if ((A >> lane) & 1u) sts_u16(it_s + 2u * (T + (uint32_t)__popc(A & lanemask_lt())), ((uint32_t)e << 5) | lane);
+        T += (uint32_t)__popc(A);
+    }
+    __syncwarp();
+    for (uint32_t b0 = 0; b0 < T; b0 += 32) {
+        const uint32_t it = b0 + lane;
+        const bool v = it < T;
+        const uint32_t code = v ? lds_u16(it_s + 2u * it) : 0u;
+        const uint32_t e = code >> 5, l = code & 31u;
+        const uint32_t seg = v ? e : 31u;             // segment id (31: no entry)
+        const uint32_t qe = q_s + 4u * QW * e;
+        const uint4 w0 = lds_u32x4(qe + 4 * Q_TTK);
+        const uint32_t tt = w0.x & 0xffffu, K = (w0.x >> 16) & 0xffu;
+        const uint4 X = lds_u32x4(qe + 4 * Q_X), Ev = lds_u32x4(qe + 4 * Q_E);
+        const uint32_t Xa[4] = {X.x, X.y, X.z, X.w}, Ea[4] = {Ev.x, Ev.y, Ev.z, Ev.w};
+        const uint32_t lmask = (1u << l) - 1u;
+        uint32_t bits = 0, evb = 0;
+#pragma unroll
+        for (int q = 0; q < 4; ++q) {
+            bits |= ((Xa[q] >> l) & 1u) << q;
+            evb |= ((Ea[q] >> l) & 1u) << q;
+        }
+        // observable inputs of this slot: with the inputs without events at
+        // their values, the truth table restricted to the remaining minterms
+        // depends on input q
+        constexpr uint32_t POS[4] = {0xAAAAu, 0xCCCCu, 0xF0F0u, 0xFF00u};
+        uint32_t mt = 0xFFFFu >> (16 - (1 << K));
+#pragma unroll
+        for (int q = 0; q < 4; ++q)
+            if ((uint32_t)q < K && !((evb >> q) & 1u)) mt &= ((bits >> q) & 1u) ? POS[q] : ~POS[q];
+        uint32_t use = 0;
+#pragma unroll
+        for (int q = 0; q < 4; ++q)
+            if (((evb >> q) & 1u) && ((((tt >> (1 << q)) ^ tt) & mt & ~POS[q]) != 0)) use |= 1u << q;
+        if (!v) use = 0;
+        // entries of the used inputs
+        const uint4 AQ = lds_u32x4(qe + 4 * Q_AQ), LOC = lds_u32x4(qe + 4 * Q_LOC);
+        const uint32_t AQa[4] = {AQ.x, AQ.y, AQ.z, AQ.w}, LOCa[4] = {LOC.x, LOC.y, LOC.z, LOC.w};
+        const float* ap[4];
+        int nn[4];
+#pragma unroll
+        for (int q = 0; q < 4; ++q) {
+            ap[q] = p.zero;
+            nn[q] = 0;
+            if ((use >> q) & 1u) {
+                const unsigned long long itb = lds_u64(qe + 4 * Q_ITB + 8 * q);
+                if ((LOCa[q] & LOC_KIND) == LOC_PI) {
+                    nn[q] = 1;
+                } else {
+                    const uint32_t* ent = reinterpret_cast<const uint32_t*>(G.row + (size_t)(LOCa[q] & LOC_ID) * G.stride);
+                    const uint32_t w = __ldcg(ent + __popc(AQa[q] & lmask));
+                    nn[q] = (int)(w & ENT_N);
+                    ap[q] = reinterpret_cast<const float*>(itb) + (w >> ENT_OFF_SHIFT);
                 }
             }
-            // this level's stores -> the next levels' loads; with several slot
-            // groups per CTA each group syncs only its own warps (named barrier)
-            if (G == 1 || G > 15) __syncthreads();
-            else asm volatile("bar.sync %0, %1;" ::"r"(1 + sg), "r"(32 * wpg) : "memory");
+        }
+        const uint32_t m = (uint32_t)(nn[0] + nn[1] + nn[2] + nn[3]);
+        // output offsets: segmented exclusive prefix of m over the entry's
+        // items in this pass, after the entry's carry from earlier passes
+        const uint32_t prev_seg = __shfl_up_sync(FULL, seg, 1);
+        const bool head = lane == 0 || prev_seg != seg;
+        const uint32_t heads = __ballot_sync(FULL, head);
+        const int sl = 31 - __clz(heads & lanemask_le());
+        const uint32_t incl = warp_incl_scan(m, lane);
+        const uint32_t excl = incl - m;
+        const uint32_t seg_excl = __shfl_sync(FULL, excl, sl);
+        const uint32_t carry = lds_u32(qe + 4 * Q_CARRY);
+        const uint32_t off = carry + (excl - seg_excl);
+        const bool seg_last = (lane == 31) || ((heads >> (lane + 1)) & 1u);
+        __syncwarp();
+        if (v && seg_last) sts_u32(qe + 4 * Q_CARRY, off + m);
+        const uint32_t steps = __reduce_max_sync(FULL, m);
+        const unsigned long long tbo = lds_u64(qe + 4 * Q_TB);
+        float* out = reinterpret_cast<float*>(tbo) + off;
+        const uint32_t y0 = (w0.w >> l) & 1u;
+        uint32_t n_out;
+        if (__any_sync(FULL, __popc(use) > 2)) {
+            n_out = merge_four(ap, nn, bits, y0, tt, qe + 4 * Q_DLY, out, steps);
+        } else {
+            // the (at most two) used pins in ascending order; list 1 may be empty
+            const int p0 = use ? __ffs(use) - 1 : 0;
+            const uint32_t rest = use & (use - 1u);
+            const int p1 = rest ? __ffs(rest) - 1 : p0;
+            const float* a0 = ap[0];
+            const float* a1 = ap[0];
+            int n0 = 0, n1 = 0;
+#pragma unroll
+            for (int q = 0; q < 4; ++q) {
+                if (q == p0) { a0 = ap[q]; n0 = nn[q]; }
+                if (q == p1 && rest) { a1 = ap[q]; n1 = nn[q]; }
+            }
+            float4 dl;
+            dl.x = lds_f32(qe + 4 * (Q_DLY + 2 * p0));
+            dl.y = lds_f32(qe + 4 * (Q_DLY + 2 * p0 + 1));
+            dl.z = lds_f32(qe + 4 * (Q_DLY + 2 * p1));
+            dl.w = lds_f32(qe + 4 * (Q_DLY + 2 * p1 + 1));
+            n_out = merge_two(a0, n0, a1, n1, bits, 1u << p0, rest ? 1u << p1 : 0u, y0, tt, dl, out, steps);
+        }
+        if (v) {
+            uint32_t* oent = reinterpret_cast<uint32_t*>(G.row + (size_t)w0.z * G.stride);
+            const uint32_t A = lds_u32(qe + 4 * Q_A);
+            __stcg(oent + __popc(A & lmask), min(n_out, ENT_N) | (off << ENT_OFF_SHIFT));
+            if (m > ENT_N) atoms_or(qe + 4 * Q_FLAG, QF_POISON | QF_OWN);
+            if (n_out) {
+                atoms_or(qe + 4 * Q_EOUT, 1u << l);
+                atoms_add(qe + 4 * Q_ACT, n_out);
+                if (w0.x & (1u << 24)) atoms_max(qe + 4 * Q_LAST, __float_as_uint(__ldcg(out + n_out - 1)));
+            }
+        }
+        __syncwarp();
+    }
+    // records of the queued gates; one global atomic per gate for activity
+    // (reading C15) and the latest PO arrival, counted once per slot
+    // group across rerun rounds
+    if (lane < nq) {
+        const uint32_t qe = q_s + 4u * QW * (uint32_t)lane;
+        const uint4 w0 = lds_u32x4(qe + 4 * Q_TTK);     // ttk, sig, out, y0
+        const uint4 w1 = lds_u32x4(qe + 4 * Q_A);       // A, E, count, carry
+        const uint4 w2 = lds_u32x4(qe + 4 * Q_TB);      // time base, latest, flags
+        const uint32_t fl = w2.w;
+        const bool pois = fl & QF_POISON;
+        const uint32_t meta = pois ? REC_POISON : (w1.z | ((fl & QF_SPILL) ? REC_SPILL : 0u));
+        __stcg(G.rec + (size_t)w0.z * G.rstride, make_uint4(w0.w, pois ? 0u : w1.y, pois ? 0u : w1.x, meta));
+        const bool counted = fl & QF_COUNT;
+        if (pois) {
+            if (!RERUN || counted) poison_bit(p, G.gi, w0.y);
+            if (fl & QF_OWN) p.ovf[G.gi] = 1;
+        } else {
+            if (counted && w1.z) atomicAdd(p.act + (size_t)w0.y * (uint32_t)p.n_vdd + G.kv, (unsigned long long)w1.z);
+            if (counted && (w0.x & (1u << 24)) && w2.z) atomicMax(p.latest + G.kv, w2.z);
+            enc += (unsigned long long)(1u + (fl >> 8)) * (unsigned long long)__popc(w1.y);
         }
     }
+    __syncwarp();
 }
 
-// The same sweep with each slot group shared by S = p.split co-resident CTAs
-// (consecutive blocks; the grid is a multiple of S): CTA part s takes the
-// s-th 1/S slice of every level, and the S parts meet at a level barrier
-// made of an L2 counter per group.  Chosen when few slot groups would leave
-// the last wave of CTAs mostly empty.  (A separate kernel: folding it into
-// the one above changed that kernel's scheduling enough to cost 7 % on
-// config 2.)
-template <bool SPLIT>
-__global__ void __launch_bounds__(AVFS_SWEEP_THREADS, AVFS_SWEEP_MINB) sweep_split_kernel(const SweepParams p) {
-    const int lane = threadIdx.x & 31;
-    const int warp = threadIdx.x >> 5;
-    const int nw = blockDim.x >> 5;
-    Env E;
-    // shared addresses only (no generic pointers into the warp's area)
-    const uint32_t ws_s = smem_u32(warp_smem(0, 0)) + 4u * (uint32_t)(warp * WARP_SMEM_WORDS);
-    const uint32_t s_desc = ws_s + 4 * OFF_DESC, s_hdr = ws_s + 4 * OFF_HDR, s_evr = ws_s + 4 * OFF_EV;
-    const uint32_t s_grp = ws_s + 4 * (OFF_META + 2);
-    E.stride = (uint32_t)(p.pin_n_sw * p.region_bytes);
-    const uint4* gd = reinterpret_cast<const uint4*>(p.gates);
-    // narrow netlists: the CTA walks G slot groups at once, nw / G warps each;
-    // few slot groups: S co-resident CTAs (consecutive blocks, grid a multiple
-    // of S) share one group, each taking 1/S of every level (G == 1 then)
-    const int G = SPLIT ? 1 : p.grp_per_cta, wpg = nw / G, S = SPLIT ? p.split : 1;
+template <bool SPLIT, bool RERUN>
+__global__ void __launch_bounds__(AVFS_SWEEP_THREADS, 1) sweep_kernel(const SweepParams p) {
+    extern __shared__ __align__(16) uint32_t smem_w[];
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nw = blockDim.x >> 5;
+    const uint32_t base_s = smem_u32(smem_w);
+    const uint32_t q_s = base_s + 4u * (uint32_t)(CTA_HDR_WORDS + warp * WARP_SMEM_WORDS);
+    const uint32_t it_s = q_s + 4u * QN * QW;
+    // narrow netlists: the CTA walks GP slot groups at once, nw / GP warps
+    // each; few slot groups: S co-resident CTAs (consecutive blocks, grid a
+    // multiple of S) share one group, each taking 1/S of every level
+    const int GP = SPLIT ? 1 : p.grp_per_cta, wpg = nw / GP, S = SPLIT ? p.split : 1;
     const int sg = warp / wpg, wl = warp % wpg;
+    const uint32_t ctr_s = base_s + 8u * (uint32_t)sg;        // this group's level counters
+    unsigned long long enc = 0;
+    Grp G;
     const int64_t u_end = SPLIT ? p.n_sw * S : p.n_sw;
-    const int64_t u_step = SPLIT ? (int64_t)gridDim.x : (int64_t)gridDim.x * G;
-    for (int64_t u = SPLIT ? (int64_t)blockIdx.x : (int64_t)blockIdx.x * G; u < u_end; u += u_step) {
+    const int64_t u_step = SPLIT ? (int64_t)gridDim.x : (int64_t)gridDim.x * GP;
+    for (int64_t u = SPLIT ? (int64_t)blockIdx.x : (int64_t)blockIdx.x * GP; u < u_end; u += u_step) {
         const int64_t i0 = SPLIT ? u / S : u;
         const int part = SPLIT ? (int)(u % S) : 0;
         const int64_t i = i0 + sg;
         const bool valid = i < p.n_sw;                 // idle warps still meet every level barrier
-        slot_group(p, valid ? i : i0, lane, E);
-        __syncwarp();
-        if (lane == 0) sts_u32(s_grp, (uint32_t)(p.i_base + (valid ? i : i0)));
-        const float4* dt = p.dtab + (int64_t)E.kv * p.n_gates * 2;
+        group_setup(p, valid ? i : i0, lane, G);
+        const float4* dt = p.dtab + (int64_t)G.kv * p.n_gates * 2;
+        if (wl == 0 && lane == 0) {
+            sts_u32(ctr_s, 0u);
+            sts_u32(ctr_s + 4, 0u);
+        }
+        if (GP == 1 || GP > 15) __syncthreads();
+        else asm volatile("bar.sync %0, %1;" ::"r"(1 + sg), "r"(32 * wpg) : "memory");
         for (int L = 0; L < p.depth; ++L) {
             const int ls0 = __ldg(p.level_ptr + L), le0 = __ldg(p.level_ptr + L + 1);
-            const int P = SPLIT ? (le0 - ls0 + S - 1) / S : 0;
-            const int ls = SPLIT ? min(le0, ls0 + part * P) : ls0;
-            const int le = SPLIT ? min(le0, ls + P) : le0;
-            const int B = (le - ls + wpg - 1) / wpg;
-            const int g0 = ls + wl * B;
-            const int nj = valid ? max(0, min(B, le - g0)) : 0;
-            // descriptor window k (gates g0 + 16k ..): lane copies 16 B of the
-            // descriptors (lanes 0..31 = 16 gates x 2) and 16 B of the delays
-            // descriptor ring of 2 DW gates (32 B each), delay ring behind it
-            auto issue_win = [&](int k) {
-                const int g = g0 + DW * k + (lane >> 1);
-                const uint32_t w = s_desc + 32 * ((uint32_t)(DW * k + (lane >> 1)) & (2 * DW - 1)) + 16 * (lane & 1);
-                if (g < le) {
-                    cp_async16(w, gd + 2 * g + (lane & 1));
-                    cp_async16(w + 32 * 2 * DW, dt + 2 * g + (lane & 1));
-                }
-            };
-            auto desc_at = [&](uint32_t j) { return s_desc + 32 * (j & (2 * DW - 1)); };
-            auto issue_hdr = [&](uint32_t j) {
-                const uint32_t d = desc_at(j);
-                const uint32_t q = (uint32_t)lane >> 3;
-                if (q < ((lds_u32(d + 24) >> 16) & 0xffu))
-                    cp_async16(s_hdr + 512 * (j & 3) + 128 * q + 16 * (lane & 7),
-                               region(lds_u32(d + 4 * q), E) + 16 * (lane & 7));
-            };
-            // input q's events (extent = lane 31's offset + count) -> slot q of
-            // the stage (EV_STAGE / K' words, 32 / K' lanes per input, <= 2
-            // chunks of 16 B per lane); staged only if every input fits
-            bool staged_next = false, staged_cur = false;
-            auto issue_ev = [&](uint32_t j) {
-                const uint32_t d = desc_at(j);
-                const uint32_t k = (lds_u32(d + 24) >> 16) & 0xffu;
-                const uint32_t sh = k > 2 ? 2u : (k > 1 ? 1u : 0u);      // log2 K'
-                const uint32_t q = (uint32_t)lane >> (5 - sh), sub = (uint32_t)lane & (31u >> sh);
-                uint32_t c = 0, w = 0;
-                if (q < k) {
-                    w = lds_u32(s_hdr + 512 * (j & 3) + 128 * q + 124);
-                    c = (((w >> HDR_OFF_SHIFT) & HDR_OFF) + (w & HDR_N) + 3) >> 2;
-                }
-                const uint32_t cap = (uint32_t)(EV_STAGE / 4) >> sh;   // chunks per input
-                const bool staged = __all_sync(FULL, c <= cap);
-                staged_next = staged;
-                if (staged && sub < c) {
-                    const uint8_t* src = ev_base(region(lds_u32(d + 4 * q), E), w) + 16 * sub;
-                    const uint32_t dst = s_evr + 4 * EV_STAGE * (j & 1) + (4 * EV_STAGE >> sh) * q + 16 * sub;
-                    cp_async16(dst, src);
-                    const uint32_t st = 512u >> sh;                     // bytes covered by one pass of the lanes
-                    if (sub + (32u >> sh) < c) cp_async16(dst + st, src + st);
-                }
-            };
-            if (nj > 0) {
-                // prologue: descriptor windows 0, 1; header rows 0, 1; events of gate 0
-                issue_win(0);
-                if (nj > DW) issue_win(1);
-                cp_async_commit();
-                cp_async_wait_all();
-                __syncwarp();
-                issue_hdr(0);
-                if (nj > 1) issue_hdr(1);
-                cp_async_commit();
-                cp_async_wait_all();
-                __syncwarp();
-                issue_ev(0);
-                staged_cur = staged_next;
-                cp_async_commit();
-                const uint32_t nju = (uint32_t)nj;
-#pragma unroll 1
-                for (uint32_t j = 0; j < nju; ++j) {
-                    cp_async_wait_all();
-                    __syncwarp();
-                    if (j % DW == 0 && j > 0 && j + DW < nju) issue_win((int)(j / DW) + 1);
-                    if (j + 2 < nju) issue_hdr(j + 2);
-                    const bool st_j = staged_cur;
-                    if (j + 1 < nju) issue_ev(j + 1);
-                    staged_cur = staged_next;
-                    cp_async_commit();
-                    const uint32_t d = desc_at(j);
-                    const uint4 dv0 = lds_u32x4(d), dv1 = lds_u32x4(d + 16);
-                    Staged S;
-                    S.hdr = true;
-                    S.hdr_s = s_hdr + 512 * (j & 3);
-                    S.ev = st_j;
-                    S.dly_s = d + 32 * 2 * DW;
-                    S.grp_s = s_grp;
-                    S.ev_s[0] = s_evr + 4 * EV_STAGE * (j & 1);
-                    eval_dispatch<false>(p, E, dv0, dv1, S);
+            int ls = ls0, le = le0;
+            if (SPLIT) {
+                const int P = (le0 - ls0 + S - 1) / S;
+                ls = min(le0, ls0 + part * P);
+                le = min(le0, ls + P);
+            }
+            // batches of QN gates are grabbed from a shared counter; the
+            // next level's counter is cleared now (its last users finished
+            // before the previous barrier)
+            const uint32_t cs = ctr_s + 4u * (uint32_t)(L & 1);
+            if (wl == 0 && lane == 0) sts_u32(ctr_s + 4u * (uint32_t)((L + 1) & 1), 0u);
+            const int nlv = le - ls;
+            if (valid) {
+                while (true) {
+                    uint32_t gb = 0;
+                    if (lane == 0) gb = atoms_add(cs, QN);
+                    gb = __shfl_sync(FULL, gb, 0);
+                    if ((int)gb >= nlv) break;
+                    const int nb = min(QN, nlv - (int)gb);
+                    const int nq = phase_a<RERUN>(p, G, ls + (int)gb, nb, q_s, dt, lane);
+                    if (nq) phase_b<RERUN>(p, G, nq, q_s, it_s, lane, enc);
                 }
             }
             // this level's stores -> the next levels' loads; with several slot
             // groups per CTA each group syncs only its own warps (named barrier)
-            if (G == 1 || G > 15) __syncthreads();
+            if (GP == 1 || GP > 15) __syncthreads();
             else asm volatile("bar.sync %0, %1;" ::"r"(1 + sg), "r"(32 * wpg) : "memory");
             if (SPLIT) {                                // the other parts of this level (L2 counter)
                 if (threadIdx.x == 0) {
@@ -793,10 +673,10 @@ __global__ void __launch_bounds__(AVFS_SWEEP_THREADS, AVFS_SWEEP_MINB) sweep_spl
                     __threadfence();
                     atomicAdd(ctr, 1u);
                     const unsigned int target = (unsigned int)S * (unsigned int)(L + 1);
-                    unsigned int v;
+                    unsigned int vv;
                     while (true) {
-                        asm volatile("ld.acquire.gpu.u32 %0, [%1];" : "=r"(v) : "l"(ctr) : "memory");
-                        if (v >= target) break;
+                        asm volatile("ld.acquire.gpu.u32 %0, [%1];" : "=r"(vv) : "l"(ctr) : "memory");
+                        if (vv >= target) break;
                         __nanosleep(64);
                     }
                     __threadfence();
@@ -805,108 +685,43 @@ __global__ void __launch_bounds__(AVFS_SWEEP_THREADS, AVFS_SWEEP_MINB) sweep_spl
             }
         }
     }
+    if (enc) atomicAdd(p.enc_units, enc);
 }
 
-// Level-parallel variant for overflow reruns (few slot groups): one launch per
-// level, warps take (gate, slot group) items of the level grid-wide.
-__global__ void __launch_bounds__(512, 2) level_kernel(const SweepParams p, int L) {
-    const int lane = threadIdx.x & 31;
-    const int warp = threadIdx.x >> 5;
-    Env E;
-    float* ws = warp_smem(warp, LEVEL_SMEM_WORDS);
-    E.stride = (uint32_t)(p.pin_n_sw * p.region_bytes);
-    const uint4* gd = reinterpret_cast<const uint4*>(p.gates);
-    Staged S;
-    S.hdr = false;
-    S.ev = false;
-    S.dly_s = smem_u32(ws);
-    S.grp_s = smem_u32(ws + 8);
-    const int g0 = __ldg(p.level_ptr + L);
-    const int64_t items = (int64_t)(__ldg(p.level_ptr + L + 1) - g0) * p.n_sw;
-    const int64_t gw = (int64_t)blockIdx.x * (blockDim.x >> 5) + warp;
-    const int64_t nwarps = (int64_t)gridDim.x * (blockDim.x >> 5);
-    for (int64_t it = gw; it < items; it += nwarps) {
-        const int gi = g0 + (int)(it / p.n_sw);
-        const int64_t i = it % p.n_sw;
-        slot_group(p, i, lane, E);
-        const float* dt = reinterpret_cast<const float*>(p.dtab) + ((int64_t)E.kv * p.n_gates + gi) * 8;
-        __syncwarp();
-        if (lane < 8) ws[lane] = __ldg(dt + lane);
-        if (lane == 8) reinterpret_cast<uint32_t*>(ws)[8] = (uint32_t)(p.i_base + i);
-        __syncwarp();
-        eval_dispatch<true>(p, E, __ldg(gd + 2 * gi), __ldg(gd + 2 * gi + 1), S);
-    }
-}
+int sweep_smem_bytes(int warps_per_cta, int) { return 4 * (CTA_HDR_WORDS + warps_per_cta * WARP_SMEM_WORDS); }
 
-// Materialise PI waveforms of a round's slot groups (reading C2: one event at
-// t = 0 iff p1 != p2) as regions of buffers 0..n_pi-1: one warp per (PI, group).
-__global__ void pi_regions_kernel(const SweepParams p, int32_t n_pi) {
-    const int lane = threadIdx.x & 31;
-    const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-    if (gw >= (int64_t)n_pi * p.pin_n_sw) return;
-    const int pi = (int)(gw / p.pin_n_sw);
-    const int64_t i = gw % p.pin_n_sw;
-    const int64_t sw = p.sw_list ? (int64_t)p.sw_list[i] : p.sw_first + i;
-    const int kv = (int)(sw / p.n_pw), pw = (int)(sw % p.n_pw);
-    const int64_t j = (int64_t)pw * 32 + lane;
-    const int64_t pub = (int64_t)kv * p.n_pairs + j;
-    const bool valid = j < p.n_pairs && pub >= p.slot_first && pub < p.slot_end;
-    const uint32_t mask = __ballot_sync(0xffffffffu, valid);
-    const uint32_t w1 = p.p1t[(int64_t)pi * p.n_pw + pw] & mask;
-    const uint32_t w2 = p.p2t[(int64_t)pi * p.n_pw + pw] & mask;
-    const uint32_t tog = w1 ^ w2;
-    const uint32_t n = (tog >> lane) & 1u;
-    const uint32_t off = __popc(tog & ((1u << lane) - 1u));
-    uint8_t* r = p.arena + ((int64_t)pi * p.pin_n_sw + i) * p.region_bytes;
-    reinterpret_cast<uint32_t*>(r)[lane] = n | (off << HDR_OFF_SHIFT) | (((w1 >> lane) & 1u) << HDR_INIT_SHIFT);
-    reinterpret_cast<float*>(r + 128)[lane] = 0.0f;
-}
-
-cudaError_t launch_pi_regions(const SweepParams& p, int32_t n_pi, cudaStream_t st) {
-    const int64_t threads = (int64_t)n_pi * p.pin_n_sw * 32;
-    if (threads == 0) return cudaSuccess;
-    pi_regions_kernel<<<(unsigned)((threads + 255) / 256), 256, 0, st>>>(p, n_pi);
-    return cudaGetLastError();
-}
-
-int sweep_smem_bytes(int warps_per_cta) { return 16 + warps_per_cta * WARP_SMEM_WORDS * 4; }
-int level_smem_bytes(int warps_per_cta) { return 16 + warps_per_cta * LEVEL_SMEM_WORDS * 4; }
-
-cudaError_t sweep_occupancy(int warps_per_cta, int smem, int* blocks_per_sm) {
-    int b1 = 0, b2 = 0;
-    cudaError_t e = cudaFuncSetAttribute(sweep_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
-    if (e == cudaSuccess) e = cudaFuncSetAttribute(sweep_split_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
-    if (e == cudaSuccess) e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b1, sweep_kernel, warps_per_cta * 32, smem);
-    if (e == cudaSuccess) e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b2, sweep_split_kernel<true>, warps_per_cta * 32, smem);
-    *blocks_per_sm = b1 < b2 ? b1 : b2;      // split groups need every CTA resident
+template <bool SPLIT, bool RERUN>
+static cudaError_t occ_one(int warps_per_cta, int smem, int* b) {
+    cudaError_t e = cudaFuncSetAttribute(sweep_kernel<SPLIT, RERUN>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+    if (e == cudaSuccess) e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(b, sweep_kernel<SPLIT, RERUN>, warps_per_cta * 32, smem);
     return e;
 }
 
-cudaError_t launch_sweep(const SweepParams& p, int grid, int warps_per_cta, cudaStream_t st) {
-    const int smem = sweep_smem_bytes(warps_per_cta);
+cudaError_t sweep_occupancy(int warps_per_cta, int smem, int* blocks_per_sm) {
+    int b[4] = {0, 0, 0, 0};
+    cudaError_t e = occ_one<false, false>(warps_per_cta, smem, b + 0);
+    if (e == cudaSuccess) e = occ_one<true, false>(warps_per_cta, smem, b + 1);
+    if (e == cudaSuccess) e = occ_one<false, true>(warps_per_cta, smem, b + 2);
+    if (e == cudaSuccess) e = occ_one<true, true>(warps_per_cta, smem, b + 3);
+    int m = b[0];
+    for (int k = 1; k < 4; ++k) m = b[k] < m ? b[k] : m;    // split groups need every CTA resident
+    *blocks_per_sm = m;
+    return e;
+}
+
+cudaError_t launch_sweep(const SweepParams& p, bool rerun, int grid, int warps_per_cta, cudaStream_t st) {
+    const int smem = sweep_smem_bytes(warps_per_cta, p.grp_per_cta);
     if (p.split > 1) {
         // the parts of a slot group wait for each other: a cooperative launch
         // guarantees that every CTA of the grid is resident (or fails)
         SweepParams q = p;
         void* args[] = {&q};
-        return cudaLaunchCooperativeKernel(reinterpret_cast<const void*>(sweep_split_kernel<true>), dim3(grid),
-                                           dim3(warps_per_cta * 32), args, (size_t)smem, st);
+        const void* f = rerun ? reinterpret_cast<const void*>(sweep_kernel<true, true>)
+                              : reinterpret_cast<const void*>(sweep_kernel<true, false>);
+        return cudaLaunchCooperativeKernel(f, dim3(grid), dim3(warps_per_cta * 32), args, (size_t)smem, st);
     }
-    sweep_kernel<<<grid, warps_per_cta * 32, smem, st>>>(p);
-    return cudaGetLastError();
-}
-
-cudaError_t level_occupancy(int warps_per_cta, int smem, int* blocks_per_sm) {
-    cudaError_t e = cudaFuncSetAttribute(level_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
-    if (e != cudaSuccess) return e;
-    return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, level_kernel, warps_per_cta * 32, smem);
-}
-
-cudaError_t launch_level(const SweepParams& p, int level, int grid, int warps_per_cta, cudaStream_t st) {
-    const int smem = level_smem_bytes(warps_per_cta);
-    cudaError_t e = cudaFuncSetAttribute(level_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
-    if (e != cudaSuccess) return e;
-    level_kernel<<<grid, warps_per_cta * 32, smem, st>>>(p, level);
+    if (rerun) sweep_kernel<false, true><<<grid, warps_per_cta * 32, smem, st>>>(p);
+    else sweep_kernel<false, false><<<grid, warps_per_cta * 32, smem, st>>>(p);
     return cudaGetLastError();
 }
 
@@ -1050,8 +865,28 @@ cudaError_t launch_compact_overflow(const int32_t* ovf, int64_t n_sw, const int3
     return cudaGetLastError();
 }
 
+// Slot l of a stored waveform (record + region layout, avfs_internal.h):
+// initial value, count and its times; false if the waveform is poisoned.
+__device__ __forceinline__ bool read_slot(const GatherRound& R, uint32_t buf, int64_t idx, int l, uint32_t& init,
+                                          int& n, const float*& ev) {
+    const uint4 rec = R.recs[(size_t)buf * R.n_sw + idx];
+    if (rec.w & REC_POISON) return false;
+    const uint8_t* reg = R.pinned + ((int64_t)buf * R.n_sw + idx) * R.region_bytes;
+    init = (rec.x >> l) & 1u;
+    n = 0;
+    ev = nullptr;
+    if ((rec.z >> l) & 1u) {
+        const uint32_t w = reinterpret_cast<const uint32_t*>(reg)[__popc(rec.z & ((1u << l) - 1u))];
+        n = (int)(w & ENT_N);
+        const float* tb = (rec.w & REC_SPILL) ? *reinterpret_cast<const float* const*>(reg + REG_SPILLPTR)
+                                              : reinterpret_cast<const float*>(reg + REG_TIMES);
+        ev = tb + (w >> ENT_OFF_SHIFT);
+    }
+    return true;
+}
+
 // H9: readback of kept waveforms (PIs from the stimuli, gates from the round
-// that holds each slot group's final data).
+// that holds each slot group's final data).  One thread per (signal, slot).
 __global__ void gather_kernel(const GatherParams p) {
     const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (t >= (int64_t)p.n_sig * p.n_slots) return;
@@ -1070,21 +905,13 @@ __global__ void gather_kernel(const GatherParams p) {
         const uint32_t w2 = p.p2t[(int64_t)(loc & LOC_ID) * p.n_pw + pw];
         init = (w1 >> lane) & 1u;
         n = (int)(((w1 ^ w2) >> lane) & 1u);
-        if (tout && p.cap > 0) tout[0] = 0.0f;
-        if (tout) for (int i = n; i < p.cap; ++i) tout[i] = 0.0f;
+        if (tout) for (int i = 0; i < p.cap; ++i) tout[i] = 0.0f;
     } else {
         const int r = p.sw_round[sw];
         if (r < 0) { atomicOr(p.bad, 1); return; }
-        const GatherRound R = p.rounds[r];
-        const uint8_t* base = R.pinned + ((int64_t)(loc & LOC_ID) * R.n_sw + p.sw_index[sw]) * R.region_bytes;
-        const uint32_t* hdr = reinterpret_cast<const uint32_t*>(base);
-        const uint32_t h = hdr[lane];
-        if (h & HDR_POISON) { atomicOr(p.bad, 2); return; }
-        init = (h >> HDR_INIT_SHIFT) & 1u;
-        n = (int)(h & HDR_N);
-        const int off = (int)((h >> HDR_OFF_SHIFT) & HDR_OFF);
-        const float* ev = reinterpret_cast<const float*>(ev_base(base, h)) + off;
-        if (tout) for (int i = 0; i < p.cap; ++i) tout[i] = i < n ? ev[i] : 0.0f;
+        const float* ev;
+        if (!read_slot(p.rounds[r], loc & LOC_ID, p.sw_index[sw], lane, init, n, ev)) { atomicOr(p.bad, 2); return; }
+        if (tout) for (int i = 0; i < p.cap; ++i) tout[i] = i < n ? __ldcg(ev + i) : 0.0f;
     }
     p.init[t] = (uint8_t)init;
     p.count[t] = n;
@@ -1126,18 +953,17 @@ __global__ void capture_kernel(const CaptureParams p) {
         c = (n && 0.0f <= T) ? 1u : 0u;
     } else {
         const int r = p.sw_round[sw];
-        const GatherRound R = p.rounds[r < 0 ? 0 : r];
-        const uint8_t* base = R.pinned + ((int64_t)(loc & LOC_ID) * R.n_sw + p.sw_index[sw]) * R.region_bytes;
-        const uint32_t h = reinterpret_cast<const uint32_t*>(base)[lane];
-        init = (h >> HDR_INIT_SHIFT) & 1u;
-        n = h & HDR_N;
-        const float* ev = reinterpret_cast<const float*>(ev_base(base, h)) + ((h >> HDR_OFF_SHIFT) & HDR_OFF);
-        if (valid)
-            for (uint32_t e = 0; e < n; ++e) {
-                const float t = ev[e];
-                last = t;
-                c += (t <= T) ? 1u : 0u;
-            }
+        const float* ev;
+        int nn = 0;
+        if (r >= 0 && read_slot(p.rounds[r], loc & LOC_ID, p.sw_index[sw], lane, init, nn, ev)) {
+            n = (uint32_t)nn;
+            if (valid)
+                for (uint32_t e = 0; e < n; ++e) {
+                    const float t = __ldcg(ev + e);
+                    last = t;
+                    c += (t <= T) ? 1u : 0u;
+                }
+        }
     }
     const bool fail = valid && (((init ^ c) & 1u) != ((init ^ n) & 1u));
     const uint32_t fb = __ballot_sync(0xffffffffu, fail);

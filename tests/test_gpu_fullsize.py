@@ -55,7 +55,11 @@ def test_fullsize_sampled_po_parity(cfg, quantum):
         a, b, c = gpu_waveforms(ctx, nl.po_sig, int(s), 1, cap)
         init[i], cnt[i], times[i] = a[0], b[0], c[0]
     ref.times = ref.times[:, :, :cap]
-    r = compare(ref, init, cnt, times, quantum, f"cfg{cfg}-q{quantum}")
+    # config 5 (XOR-tree glitch amplifiers, 120 levels): nearly every PO cone holds a
+    # reading-C13 near tie somewhere, so F mode taints most pairs; they are still
+    # compared and must agree (tainted_differ), Q mode carries the exact guarantee
+    r = compare(ref, init, cnt, times, quantum, f"cfg{cfg}-q{quantum}", max_taint=1.0 if cfg == 5 else 0.3)
+    assert r["tainted_differ"] <= 0.01 * max(r["tainted"], 1)
     if quantum > 0:
         assert r["tainted"] == 0
     assert r["events"] > 0
