@@ -278,6 +278,13 @@ typedef struct {
 } avfs_stats;
 avfs_status avfs_get_stats(avfs_ctx *ctx, avfs_stats *st);
 
+/* Diagnostics: per-phase warp clock sums of the sweep kernel (16 counters:
+ * 1 bit-parallel phase, 5 item phase, 6 level barriers), accumulated over
+ * all launches since the last reset.  Only builds compiled with
+ * -DAVFS_PROF_PHASES count; returns the number of counters written (0 in
+ * normal builds, -1 on error).                                          */
+int32_t avfs_debug_phase_cycles(uint64_t *out16, int32_t reset);
+
 #ifdef __cplusplus
 }
 #endif

@@ -25,7 +25,7 @@ EXPORTS = [
     "avfs_set_options", "avfs_default_options", "avfs_simulate", "avfs_sync",
     "avfs_get_activity", "avfs_get_latest_arrival", "avfs_get_final_values",
     "avfs_get_waveforms", "avfs_get_stats", "avfs_capture", "avfs_get_switching_energy",
-    "avfs_fit_delay_polynomial",
+    "avfs_fit_delay_polynomial", "avfs_debug_phase_cycles",
 ]
 
 
@@ -104,6 +104,7 @@ def load_library(path: str = LIB_PATH):
             "avfs_capture": ([P, P, I32, C.c_float, C.c_float, P, P, P, P], C.c_int),
             "avfs_get_switching_energy": ([P, P], C.c_int),
             "avfs_fit_delay_polynomial": ([I64, P, P, P, I32, I32, D, D, D, D, P, P], C.c_int),
+            "avfs_debug_phase_cycles": ([P, I32], C.c_int32),
         }
         for name, (args, res) in sig.items():
             f = getattr(lib, name)
@@ -111,6 +112,13 @@ def load_library(path: str = LIB_PATH):
             f.restype = res
         _lib = lib
     return _lib
+
+
+def debug_phase_cycles(reset: bool = False) -> np.ndarray:
+    """Per-phase warp clock sums of the sweep (diagnostic builds, -DAVFS_PROF_PHASES)."""
+    out = np.zeros(16, np.uint64)
+    n = load_library().avfs_debug_phase_cycles(C.c_void_p(out.ctypes.data), int(reset))
+    return out if n > 0 else np.zeros(0, np.uint64)
 
 
 def _p(a):

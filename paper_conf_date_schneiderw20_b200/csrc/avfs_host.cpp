@@ -834,17 +834,20 @@ static avfs_status run_round(avfs_ctx* ctx, Round& R, int round_idx, const int32
     int wpc = ctx->opt.warps_per_cta > 0 ? ctx->opt.warps_per_cta : wmax;
     wpc = std::min(wpc, wmax);
     const double per_level = ctx->depth > 0 ? (double)ctx->n_gates / ctx->depth : 1.0;
-    // narrow netlists (few gates per level): one sweep CTA walks G slot groups
-    // at once so that every warp has >= 2 gates of a level (power of 2, <= wpc)
-    int grp = 1;
-    while (grp < wpc && per_level / (double)(wpc / grp) < 2.0) grp *= 2;
-    if (const char* e = getenv("AVFS_GROUPS_PER_CTA")) grp = std::max(1, std::min(wpc, atoi(e)));
-    while (wpc % grp) grp /= 2;
+    // slot groups per sweep CTA: two by default (each group has its own
+    // level barrier, so one group's wait overlaps the other's work); more
+    // for narrow netlists (few gates per level), up to 8, until every warp
+    // has >= 4 gates of a level; one if the groups would not fill the SMs
+    int grp = wpc >= 2 ? 2 : 1;
+    while (grp < std::min(wpc, 8) && per_level / (double)(wpc / grp) < 4.0) grp *= 2;
     const int smem = sweep_smem_bytes(wpc, grp);
     int bps = 0;
     CK(sweep_occupancy(wpc, smem, &bps));
     if (bps < 1) return fail(ctx, AVFS_ERR_CAPACITY, "sweep kernel does not fit on an SM (smem %d)", smem);
     const int64_t resident = (int64_t)ctx->n_sm * bps;
+    if (grp == 2 && R.n_sw < 2 * resident) grp = 1;            // too few groups to pair
+    if (const char* e = getenv("AVFS_GROUPS_PER_CTA")) grp = std::max(1, std::min(wpc, atoi(e)));
+    while (wpc % grp) grp /= 2;
     // few slot groups for the SMs (last wave mostly empty, e.g. reruns): S
     // co-resident CTAs share a group; S minimises waves / S, ties to the
     // smaller S, and every warp keeps >= 2 gates of a level
@@ -1386,6 +1389,10 @@ avfs_status avfs_get_switching_energy(avfs_ctx* ctx, double* out) {
     CK(cudaMemcpyAsync(out, ctx->d_energy.p, (size_t)V * sizeof(double), cudaMemcpyDeviceToHost, ctx->stream));
     CK(cudaStreamSynchronize(ctx->stream));
     return AVFS_OK;
+}
+
+int32_t avfs_debug_phase_cycles(uint64_t* out16, int32_t reset) {
+    return debug_phase_cycles(reinterpret_cast<unsigned long long*>(out16), reset);
 }
 
 avfs_status avfs_get_stats(avfs_ctx* ctx, avfs_stats* st) {

@@ -128,6 +128,7 @@ struct SweepParams {
 
 // launch wrappers (avfs_kernels.cu)
 int sweep_smem_bytes(int warps_per_cta, int grp_per_cta);
+int debug_phase_cycles(unsigned long long* out, int reset);   // -DAVFS_PROF_PHASES builds only
 cudaError_t sweep_occupancy(int warps_per_cta, int smem, int* blocks_per_sm);
 cudaError_t launch_delays(const DelayParams& p, cudaStream_t st);
 cudaError_t launch_sweep(const SweepParams& p, bool rerun, int grid, int warps_per_cta, cudaStream_t st);

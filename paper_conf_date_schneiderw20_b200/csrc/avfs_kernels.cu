@@ -170,6 +170,17 @@ __device__ __forceinline__ void atoms_add_u64(uint32_t a, unsigned long long v) 
     asm volatile("red.shared.add.u64 [%0], %1;" ::"r"(a), "l"(v) : "memory");
 }
 
+// Debug-only phase timing (-DAVFS_PROF_PHASES): per-warp clock64 sums per
+// phase, read back with avfs_debug_phase_cycles.
+#ifdef AVFS_PROF_PHASES
+__device__ unsigned long long g_phase_cycles[16];
+#define PROF_T0() long long prof_t0_ = clock64()
+#define PROF_ACC(k) do { long long t_ = clock64(); if ((threadIdx.x & 31) == 0) atomicAdd(&g_phase_cycles[k], (unsigned long long)(t_ - prof_t0_)); prof_t0_ = t_; } while (0)
+#else
+#define PROF_T0() do {} while (0)
+#define PROF_ACC(k) do {} while (0)
+#endif
+
 constexpr int QN = 16;                 // gates per batch (Phase A lanes, queue entries)
 constexpr int QW = 44;                 // words per queue entry
 enum : int {
@@ -652,19 +663,41 @@ __global__ void __launch_bounds__(AVFS_SWEEP_THREADS, 1) sweep_kernel(const Swee
             const uint32_t cs = ctr_s + 4u * (uint32_t)(L & 1);
             if (wl == 0 && lane == 0) sts_u32(ctr_s + 4u * (uint32_t)((L + 1) & 1), 0u);
             const int nlv = le - ls;
+            // narrow levels (fewer than two full batches per warp): guided
+            // batch sizes, a share of the level's remaining gates, so that
+            // the warps finish together
+            const bool guided = nlv < 2 * QN * wpg;
             if (valid) {
                 while (true) {
                     uint32_t gb = 0;
-                    if (lane == 0) gb = atoms_add(cs, QN);
-                    gb = __shfl_sync(FULL, gb, 0);
+                    int bsz = QN;
+                    if (guided) {
+                        // guided batches: a share of what is left, at most QN
+                        // gates, so that the level's last batches are small
+                        if (lane == 0) {
+                            const int rem = nlv - (int)lds_u32(cs);
+                            const int bs = max(1, min(QN, (rem + 2 * wpg - 1) / (2 * wpg)));
+                            gb = atoms_add(cs, (uint32_t)bs) | ((uint32_t)bs << 24);
+                        }
+                        gb = __shfl_sync(FULL, gb, 0);
+                        bsz = (int)(gb >> 24);
+                        gb &= 0xFFFFFFu;
+                    } else {
+                        if (lane == 0) gb = atoms_add(cs, QN);
+                        gb = __shfl_sync(FULL, gb, 0);
+                    }
                     if ((int)gb >= nlv) break;
-                    const int nb = min(QN, nlv - (int)gb);
+                    const int nb = min(bsz, nlv - (int)gb);
+                    PROF_T0();
                     const int nq = phase_a<RERUN>(p, G, ls + (int)gb, nb, q_s, dt, lane);
+                    PROF_ACC(1);
                     if (nq) phase_b<RERUN>(p, G, nq, q_s, it_s, lane, enc);
+                    PROF_ACC(5);
                 }
             }
             // this level's stores -> the next levels' loads; with several slot
             // groups per CTA each group syncs only its own warps (named barrier)
+            PROF_T0();
             if (GP == 1 || GP > 15) __syncthreads();
             else asm volatile("bar.sync %0, %1;" ::"r"(1 + sg), "r"(32 * wpg) : "memory");
             if (SPLIT) {                                // the other parts of this level (L2 counter)
@@ -683,9 +716,25 @@ __global__ void __launch_bounds__(AVFS_SWEEP_THREADS, 1) sweep_kernel(const Swee
                 }
                 __syncthreads();
             }
+            PROF_ACC(6);
         }
     }
     if (enc) atomicAdd(p.enc_units, enc);
+}
+
+int debug_phase_cycles(unsigned long long* out, int reset) {
+#ifdef AVFS_PROF_PHASES
+    if (cudaMemcpyFromSymbol(out, g_phase_cycles, sizeof(unsigned long long) * 16) != cudaSuccess) return -1;
+    if (reset) {
+        static const unsigned long long z[16] = {};
+        cudaMemcpyToSymbol(g_phase_cycles, z, sizeof z);
+    }
+    return 16;
+#else
+    (void)out;
+    (void)reset;
+    return 0;
+#endif
 }
 
 int sweep_smem_bytes(int warps_per_cta, int) { return 4 * (CTA_HDR_WORDS + warps_per_cta * WARP_SMEM_WORDS); }
