@@ -271,11 +271,12 @@ def main():
     flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
 
     def step():
-        ctx.simulate(stream)
+        ctx.simulate(stream)      # asynchronous; sync settles overflow reruns (none expected)
+        ctx.sync()
         if world > 1:
             import torch.distributed as dist
             ctx.activity(act_dev)
-            lat_dev.copy_(torch.from_numpy(ctx.latest_arrival()))
+            ctx.latest_arrival(lat_dev)                       # device copy, no host round trip
             with torch.cuda.stream(stream):
                 _reduce(act_dev, dist.ReduceOp.SUM)          # the only collective
                 _reduce(lat_dev, dist.ReduceOp.MAX)

@@ -190,12 +190,16 @@ avfs_status avfs_set_options(avfs_ctx *ctx, const avfs_options *opt);
 avfs_status avfs_default_options(avfs_options *opt);
 
 /* Simulate every slot in range on `cuda_stream` (cudaStream_t; NULL = the
- * legacy default stream).  Launches the stimulus expansion, the persistent
- * level-sweep kernel and, if some 32-slot region overflowed its capacity,
- * reruns of just those slot groups at 4x capacity.  Returns after the work
- * has completed (one host synchronisation reads the overflow count).
- * Activity and latest arrival are accumulated over the slot range and reset
- * at the start of each call.                                             */
+ * legacy default stream) -- asynchronous (P:L141 step 3):
+ * enqueues the delay evaluation, the stimulus expansion, the persistent
+ * level-sweep kernel and the overflow check, and returns.  avfs_sync waits
+ * for the work; if some slot group overflowed its waveform storage it then
+ * reruns just those groups (H7) before returning, and errors (non-positive
+ * delay, capacity still exceeded) are reported by avfs_sync.  Every get_*
+ * call, and the next simulate, settle an outstanding simulate the same way.
+ * Runs that need several slot batches settle each batch but the last
+ * inside avfs_simulate.  Activity and latest arrival are accumulated over
+ * the slot range and reset at the start of each call.                    */
 avfs_status avfs_simulate(avfs_ctx *ctx, void *cuda_stream);
 avfs_status avfs_sync(avfs_ctx *ctx);
 
@@ -205,8 +209,10 @@ avfs_status avfs_sync(avfs_ctx *ctx);
  * out_is_device = 1: `out` is a device pointer (e.g. for an NCCL reduce). */
 avfs_status avfs_get_activity(avfs_ctx *ctx, uint64_t *out, int32_t out_is_device);
 /* Latest transition time at any primary output per operating point, max
- * over simulated pairs (Table II measurement); 0 if none.        */
-avfs_status avfs_get_latest_arrival(avfs_ctx *ctx, float *out);
+ * over simulated pairs (Table II measurement); 0 if none.
+ * out[n_vdd]; out_is_device = 1: `out` is a device pointer (a MAX reduce
+ * over ranks then needs no host round trip).                              */
+avfs_status avfs_get_latest_arrival(avfs_ctx *ctx, float *out, int32_t out_is_device);
 /* Final logic value (init xor count parity) of signals sig[n_sig] at public
  * slots [slot0, slot0 + n_slots): out[n_sig][n_slots].  Signals must be
  * PIs, POs, probes (or any, with keep_all).                               */

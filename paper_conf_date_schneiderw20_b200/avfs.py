@@ -97,7 +97,7 @@ def load_library(path: str = LIB_PATH):
             "avfs_simulate": ([P, P], C.c_int),
             "avfs_sync": ([P], C.c_int),
             "avfs_get_activity": ([P, P, I32], C.c_int),
-            "avfs_get_latest_arrival": ([P, P], C.c_int),
+            "avfs_get_latest_arrival": ([P, P, I32], C.c_int),
             "avfs_get_final_values": ([P, I32, P, I64, I64, P], C.c_int),
             "avfs_get_waveforms": ([P, I32, P, I64, I64, I32, P, P, P], C.c_int),
             "avfs_get_stats": ([P, P], C.c_int),
@@ -293,9 +293,16 @@ class Context:
         self._ck(self.lib.avfs_get_activity(self.h, _p(a), 0))
         return a
 
-    def latest_arrival(self) -> np.ndarray:
+    def latest_arrival(self, out=None) -> np.ndarray:
+        """[n_vdd] float32 ps; `out` may be a contiguous CUDA float32 tensor (device copy)."""
+        if out is not None:
+            import torch
+            if not out.is_cuda or out.dtype != torch.float32 or tuple(out.shape) != (self.n_vdd,) or not out.is_contiguous():
+                raise ValueError("latest_arrival out tensor must be a contiguous CUDA float32 [n_vdd]")
+            self._ck(self.lib.avfs_get_latest_arrival(self.h, C.c_void_p(out.data_ptr()), 1))
+            return out
         a = np.zeros(self.n_vdd, np.float32)
-        self._ck(self.lib.avfs_get_latest_arrival(self.h, _p(a)))
+        self._ck(self.lib.avfs_get_latest_arrival(self.h, _p(a), 0))
         return a
 
     def final_values(self, sig, slot0: int, n_slots: int) -> np.ndarray:

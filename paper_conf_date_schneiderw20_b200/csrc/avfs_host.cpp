@@ -142,10 +142,25 @@ struct avfs_ctx {
 
     // last simulation
     bool sim_done = false, map_valid = false;
+    // an asynchronous simulate whose overflow check is still outstanding
+    // (settled by avfs_sync or any call that needs the results)
+    bool pending = false;
+    int pend_r = 0, pend_cur = 0;
+    int64_t pend_r0n = 1, pend_hint = 0, pend_slots = 0;
+    double pend_sweep_ms = 0;
+    std::chrono::steady_clock::time_point pend_t0;
     std::vector<Round> rounds;
     int64_t sim_first = 0, sim_end = 0;
     avfs_stats stats{};
 };
+
+static avfs_status finish_pending(avfs_ctx* ctx);   // settles an asynchronous simulate (defined below)
+
+#define SETTLE()                                                                                   \
+    do {                                                                                           \
+        avfs_status s_ = finish_pending(ctx);                                                      \
+        if (s_ != AVFS_OK) return s_;                                                              \
+    } while (0)
 
 namespace {
 
@@ -381,7 +396,13 @@ avfs_status upload_netlist(avfs_ctx* ctx) {
     return AVFS_OK;
 }
 
+// inputs change: settle an outstanding simulate first (its errors, if any,
+// stay in avfs_last_error), then drop its results
 void invalidate_sim(avfs_ctx* ctx) {
+    if (ctx->pending) {
+        const std::string keep = ctx->err;
+        if (finish_pending(ctx) == AVFS_OK) ctx->err = keep;
+    }
     ctx->sim_done = false;
     ctx->map_valid = false;
 }
@@ -823,6 +844,7 @@ avfs_status avfs_set_options(avfs_ctx* ctx, const avfs_options* o) {
 avfs_status avfs_sync(avfs_ctx* ctx) {
     CHECK_CTX();
     if (!has_dev(ctx)) return AVFS_OK;
+    SETTLE();
     CK(cudaStreamSynchronize(ctx->stream));
     return AVFS_OK;
 }
@@ -955,11 +977,115 @@ static avfs_status run_round(avfs_ctx* ctx, Round& R, int round_idx, const int32
     return AVFS_OK;
 }
 
+}  // extern "C"
+
+// Overflow check of the last round: compaction of the overflowed slot groups
+// and asynchronous copies of their count, the delay error flag and the
+// round's heap request into pinned host memory.
+static avfs_status issue_checks(avfs_ctx* ctx, int r, int cur) {
+    Round& prev = ctx->rounds.back();
+    CK(ctx->d_list[cur].ensure(std::max<int64_t>(prev.n_sw, 1) * sizeof(int32_t)));
+    CK(ctx->d_prev[cur].ensure(std::max<int64_t>(prev.n_sw, 1) * sizeof(int32_t)));
+    CK(cudaMemsetAsync(ctx->d_count.p, 0, 16, ctx->stream));
+    CK(launch_compact_overflow(ctx->d_ovf.as<int32_t>(), prev.n_sw,
+                               r == 0 ? nullptr : ctx->d_list[cur ^ 1].as<int32_t>(), prev.sw_first,
+                               ctx->d_list[cur].as<int32_t>(), ctx->d_prev[cur].as<int32_t>(),
+                               ctx->d_count.as<int32_t>(), ctx->stream));
+    ctx->stats.launches++;
+    CK(cudaMemcpyAsync(ctx->h_pinned, ctx->d_count.p, 4, cudaMemcpyDeviceToHost, ctx->stream));
+    CK(cudaMemcpyAsync(ctx->h_pinned + 1, ctx->d_err.p, 4, cudaMemcpyDeviceToHost, ctx->stream));
+    CK(cudaMemcpyAsync(ctx->h_pinned + 2, ctx->d_spill_top.as<unsigned long long>() + r, 8,
+                       cudaMemcpyDeviceToHost, ctx->stream));
+    return AVFS_OK;
+}
+
+// Wait for the outstanding overflow check of the current batch; rerun the
+// overflowed slot groups (H7) until none is left, then fold the batch's heap
+// requests into the sizing hints.
+static avfs_status settle_batch(avfs_ctx* ctx) {
+    avfs_status st = AVFS_OK;
+    for (;;) {
+        const int r = ctx->pend_r;
+        const int cur = ctx->pend_cur;
+        Round& prev = ctx->rounds.back();
+        CK(cudaStreamSynchronize(ctx->stream));
+        {
+            unsigned long long req = 0;
+            std::memcpy(&req, ctx->h_pinned + 2, 8);
+            prev.spill_req = (int64_t)req;
+            ctx->stats.spill_bytes += 4 * std::min<int64_t>(prev.spill_req, prev.spill_words);
+            ctx->stats.spill_heap_bytes += 4 * prev.spill_words;
+        }
+        if (ctx->h_pinned[1] & 1)
+            return fail(ctx, AVFS_ERR_DELAY_NONPOS, "a delay d' = d_nom (1 + f(P)) evaluated to <= 0");
+        const int32_t n_ovf = ctx->h_pinned[0];
+        if (n_ovf == 0) break;
+        if (r >= ctx->opt.max_rerun_rounds)
+            return fail(ctx, AVFS_ERR_CAPACITY, "%d slot groups still overflow at capacity %d after %d reruns",
+                        n_ovf, prev.capacity, r);
+        Round Rn;
+        Rn.n_sw = n_ovf;
+        Rn.sws.resize(n_ovf);
+        CK(cudaMemcpy(Rn.sws.data(), ctx->d_list[cur].p, n_ovf * sizeof(int32_t), cudaMemcpyDeviceToHost));
+        // with a spill heap the overflow was heap exhaustion: same capacity, a
+        // heap 4x what was asked for (poisoned cones asked for nothing), at
+        // least 64 MiB; without one, 4x capacity
+        if (prev.spill_want > 0) {
+            Rn.capacity = prev.capacity;
+            Rn.spill_want = std::max<int64_t>(4 * std::max<int64_t>(prev.spill_req, prev.spill_words), (64ll << 20) / 4);
+        } else {
+            Rn.capacity = std::min(prev.capacity * 4, 1024);
+        }
+        Rn.W = 32 * Rn.capacity;
+        Rn.region_bytes = REG_TIMES + 4 * (int64_t)Rn.W;
+        ctx->stats.overflow_slot_warps += n_ovf;
+        ctx->stats.rerun_rounds++;
+        st = run_round(ctx, Rn, r + 1, ctx->d_list[cur].as<int32_t>(), ctx->d_prev[cur].as<int32_t>(), false);
+        if (st != AVFS_OK) return st;
+        ctx->rounds.push_back(std::move(Rn));
+        ctx->pend_r = r + 1;
+        ctx->pend_cur = cur ^ 1;
+        st = issue_checks(ctx, ctx->pend_r, ctx->pend_cur);
+        if (st != AVFS_OK) return st;
+    }
+    int64_t req = 0;
+    for (const Round& R : ctx->rounds) req += R.spill_req;
+    ctx->pend_hint = std::max(ctx->pend_hint, req);
+    ctx->spill_per_group = std::max<int64_t>(ctx->spill_per_group, (req + ctx->pend_r0n - 1) / ctx->pend_r0n);
+    if (ctx->opt.profile) {
+        float ms = 0;
+        CK(cudaEventElapsedTime(&ms, ctx->ev0, ctx->ev1));
+        ctx->pend_sweep_ms += ms;
+    }
+    return AVFS_OK;
+}
+
+// Settle an asynchronous simulate (avfs_sync, and every call that reads its
+// results): overflow reruns, errors, statistics.
+static avfs_status finish_pending(avfs_ctx* ctx) {
+    if (!ctx->pending) return AVFS_OK;
+    ctx->pending = false;
+    avfs_status st = settle_batch(ctx);
+    if (st != AVFS_OK) return st;
+    ctx->spill_hint = ctx->pend_hint;
+    if (ctx->opt.profile) ctx->stats.sweep_ms = ctx->pend_sweep_ms;
+    ctx->stats.batches = ctx->n_batches;
+    int64_t ab = 0;
+    for (size_t r = 0; r < ctx->rounds.size(); ++r) ab += (int64_t)ctx->arena[r].n;
+    ctx->stats.arena_bytes = ab;
+    ctx->stats.sim_ms = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - ctx->pend_t0).count();
+    ctx->sim_done = true;
+    return AVFS_OK;
+}
+
+extern "C" {
+
 avfs_status avfs_simulate(avfs_ctx* ctx, void* cuda_stream) {
     CHECK_CTX();
     if (!has_dev(ctx)) return fail(ctx, AVFS_ERR_STATE, "host-only context");
     if (!ctx->net_loaded || !ctx->stim_set || ctx->vdd.empty())
         return fail(ctx, AVFS_ERR_STATE, "netlist, stimuli and operating points must be set");
+    SETTLE();                                          // a previous simulate's reruns (same stream)
     const auto t0 = std::chrono::steady_clock::now();
     CK(cudaSetDevice(ctx->dev));
     ctx->stream = static_cast<cudaStream_t>(cuda_stream);
@@ -1065,8 +1191,8 @@ avfs_status avfs_simulate(avfs_ctx* ctx, void* cuda_stream) {
     }
     nb = std::min(nb, n_sw_all);
     ctx->n_batches = 0;
-    double sweep_ms_sum = 0;
-    int64_t hint = 0;
+    ctx->pend_sweep_ms = 0;
+    ctx->pend_hint = 0;
     for (int64_t b0 = sw_lo; b0 < sw_hi; b0 += nb) {
     if (b0 > sw_lo) {                                   // earlier batches' rerun memory is not kept
         for (size_t r = 1; r < ctx->arena.size(); ++r) ctx->arena[r].release();
@@ -1097,91 +1223,32 @@ avfs_status avfs_simulate(avfs_ctx* ctx, void* cuda_stream) {
     }
     st = run_round(ctx, R0, 0, nullptr, nullptr, ctx->opt.profile != 0);
     if (st != AVFS_OK) return st;
-    const int64_t R0n = std::max<int64_t>(R0.n_sw, 1);
     ctx->rounds.push_back(R0);
-    int cur = 0;
-    for (int r = 0;; ++r) {
-        Round& prev = ctx->rounds.back();
-        CK(ctx->d_list[cur].ensure(std::max<int64_t>(prev.n_sw, 1) * sizeof(int32_t)));
-        CK(ctx->d_prev[cur].ensure(std::max<int64_t>(prev.n_sw, 1) * sizeof(int32_t)));
-        CK(cudaMemsetAsync(ctx->d_count.p, 0, 16, ctx->stream));
-        CK(launch_compact_overflow(ctx->d_ovf.as<int32_t>(), prev.n_sw,
-                                   r == 0 ? nullptr : ctx->d_list[cur ^ 1].as<int32_t>(), prev.sw_first,
-                                   ctx->d_list[cur].as<int32_t>(), ctx->d_prev[cur].as<int32_t>(),
-                                   ctx->d_count.as<int32_t>(), ctx->stream));
-        ctx->stats.launches++;
-        CK(cudaMemcpyAsync(ctx->h_pinned, ctx->d_count.p, 4, cudaMemcpyDeviceToHost, ctx->stream));
-        CK(cudaMemcpyAsync(ctx->h_pinned + 1, ctx->d_err.p, 4, cudaMemcpyDeviceToHost, ctx->stream));
-        CK(cudaMemcpyAsync(ctx->h_pinned + 2, ctx->d_spill_top.as<unsigned long long>() + r, 8,
-                           cudaMemcpyDeviceToHost, ctx->stream));
-        CK(cudaStreamSynchronize(ctx->stream));
-        {
-            unsigned long long req = 0;
-            std::memcpy(&req, ctx->h_pinned + 2, 8);
-            prev.spill_req = (int64_t)req;
-            ctx->stats.spill_bytes += 4 * std::min<int64_t>(prev.spill_req, prev.spill_words);
-            ctx->stats.spill_heap_bytes += 4 * prev.spill_words;
-        }
-        if (ctx->h_pinned[1] & 1)
-            return fail(ctx, AVFS_ERR_DELAY_NONPOS, "a delay d' = d_nom (1 + f(P)) evaluated to <= 0");
-        const int32_t n_ovf = ctx->h_pinned[0];
-        if (n_ovf == 0) break;
-        if (r >= ctx->opt.max_rerun_rounds)
-            return fail(ctx, AVFS_ERR_CAPACITY, "%d slot groups still overflow at capacity %d after %d reruns",
-                        n_ovf, prev.capacity, r);
-        Round Rn;
-        Rn.n_sw = n_ovf;
-        Rn.sws.resize(n_ovf);
-        CK(cudaMemcpy(Rn.sws.data(), ctx->d_list[cur].p, n_ovf * sizeof(int32_t), cudaMemcpyDeviceToHost));
-        // with a spill heap the overflow was heap exhaustion: same capacity, a
-        // heap 4x what was asked for (poisoned cones asked for nothing), at
-        // least 64 MiB; without one, 4x capacity
-        if (prev.spill_want > 0) {
-            Rn.capacity = prev.capacity;
-            Rn.spill_want = std::max<int64_t>(4 * std::max<int64_t>(prev.spill_req, prev.spill_words), (64ll << 20) / 4);
-        } else {
-            Rn.capacity = std::min(prev.capacity * 4, 1024);
-        }
-        Rn.W = 32 * Rn.capacity;
-        Rn.region_bytes = REG_TIMES + 4 * (int64_t)Rn.W;
-        ctx->stats.overflow_slot_warps += n_ovf;
-        ctx->stats.rerun_rounds++;
-        st = run_round(ctx, Rn, r + 1, ctx->d_list[cur].as<int32_t>(), ctx->d_prev[cur].as<int32_t>(), false);
+    st = issue_checks(ctx, 0, 0);
+    if (st != AVFS_OK) return st;
+    ctx->pend_r = 0;
+    ctx->pend_cur = 0;
+    ctx->pend_r0n = std::max<int64_t>(R0.n_sw, 1);
+    if (b0 + nb < sw_hi) {                              // more batches follow: settle this one now
+        st = settle_batch(ctx);
         if (st != AVFS_OK) return st;
-        ctx->rounds.push_back(std::move(Rn));
-        cur ^= 1;
-    }
-    {
-        int64_t req = 0;
-        for (const Round& R : ctx->rounds) req += R.spill_req;
-        hint = std::max(hint, req);
-        ctx->spill_per_group = std::max<int64_t>(ctx->spill_per_group, (req + R0n - 1) / R0n);
-    }
-    if (ctx->opt.profile) {
-        float ms = 0;
-        CK(cudaEventElapsedTime(&ms, ctx->ev0, ctx->ev1));
-        sweep_ms_sum += ms;
     }
     }  // batches
-    ctx->spill_hint = hint;
-    if (ctx->opt.profile) ctx->stats.sweep_ms = sweep_ms_sum;
-    ctx->sim_done = true;
+    ctx->pend_t0 = t0;
+    ctx->pend_slots = end - first;
     ctx->stats.slots = end - first;
     ctx->stats.evals = (int64_t)ctx->n_gates * (end - first);
     ctx->stats.slot_warps = sw_hi - sw_lo;
     ctx->stats.grid = ctx->rounds[0].grid;
-    ctx->stats.batches = ctx->n_batches;
     ctx->stats.n_scratch_buffers = ctx->n_scratch;
     ctx->stats.n_pinned = ctx->n_pinned;
-    int64_t ab = 0;
-    for (size_t r = 0; r < ctx->rounds.size(); ++r) ab += (int64_t)ctx->arena[r].n;
-    ctx->stats.arena_bytes = ab;
-    ctx->stats.sim_ms = std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+    ctx->pending = true;                               // the last batch's overflow check is outstanding
     return AVFS_OK;
 }
 
 avfs_status avfs_get_activity(avfs_ctx* ctx, uint64_t* out, int32_t out_is_device) {
     CHECK_CTX();
+    SETTLE();
     if (!out) return fail(ctx, AVFS_ERR_ARG, "null output");
     if (!ctx->sim_done) return fail(ctx, AVFS_ERR_STATE, "simulate first");
     const size_t n = (size_t)(ctx->n_pi + ctx->n_gates) * ctx->vdd.size() * sizeof(uint64_t);
@@ -1191,12 +1258,14 @@ avfs_status avfs_get_activity(avfs_ctx* ctx, uint64_t* out, int32_t out_is_devic
     return AVFS_OK;
 }
 
-avfs_status avfs_get_latest_arrival(avfs_ctx* ctx, float* out) {
+avfs_status avfs_get_latest_arrival(avfs_ctx* ctx, float* out, int32_t out_is_device) {
     CHECK_CTX();
+    SETTLE();
     if (!out) return fail(ctx, AVFS_ERR_ARG, "null output");
     if (!ctx->sim_done) return fail(ctx, AVFS_ERR_STATE, "simulate first");
-    CK(cudaMemcpyAsync(out, ctx->d_latest.p, ctx->vdd.size() * 4, cudaMemcpyDeviceToHost, ctx->stream));
-    CK(cudaStreamSynchronize(ctx->stream));
+    CK(cudaMemcpyAsync(out, ctx->d_latest.p, ctx->vdd.size() * 4,
+                       out_is_device ? cudaMemcpyDeviceToDevice : cudaMemcpyDeviceToHost, ctx->stream));
+    if (!out_is_device) CK(cudaStreamSynchronize(ctx->stream));
     return AVFS_OK;
 }
 
@@ -1290,6 +1359,7 @@ static avfs_status gather(avfs_ctx* ctx, int32_t n_sig, const int32_t* sig, int6
 avfs_status avfs_get_final_values(avfs_ctx* ctx, int32_t n_sig, const int32_t* sig, int64_t slot0,
                                   int64_t n_slots, uint8_t* out) {
     CHECK_CTX();
+    SETTLE();
     if (!out) return fail(ctx, AVFS_ERR_ARG, "null output");
     const size_t n = (size_t)std::max(n_sig, 0) * std::max<int64_t>(n_slots, 0);
     std::vector<uint8_t> init(n);
@@ -1303,6 +1373,7 @@ avfs_status avfs_get_final_values(avfs_ctx* ctx, int32_t n_sig, const int32_t* s
 avfs_status avfs_get_waveforms(avfs_ctx* ctx, int32_t n_sig, const int32_t* sig, int64_t slot0, int64_t n_slots,
                                int32_t cap, uint8_t* init, int32_t* count, float* times) {
     CHECK_CTX();
+    SETTLE();
     if (!init || !count || (cap > 0 && !times)) return fail(ctx, AVFS_ERR_ARG, "null output");
     return gather(ctx, n_sig, sig, slot0, n_slots, cap, init, count, cap > 0 ? times : nullptr);
 }
@@ -1310,6 +1381,7 @@ avfs_status avfs_get_waveforms(avfs_ctx* ctx, int32_t n_sig, const int32_t* sig,
 avfs_status avfs_capture(avfs_ctx* ctx, const float* t_clk, int32_t n_bins, float lo_ps, float width_ps,
                          uint32_t* fail_pairs, uint32_t* fail_po, uint32_t* slack_hist, uint8_t* fail_bits) {
     CHECK_CTX();
+    SETTLE();
     if (!ctx->sim_done) return fail(ctx, AVFS_ERR_STATE, "simulate first");
     if (!t_clk || !fail_pairs) return fail(ctx, AVFS_ERR_ARG, "null t_clk / fail_pairs");
     if (slack_hist && (n_bins < 1 || !(width_ps > 0))) return fail(ctx, AVFS_ERR_ARG, "bad histogram bins");
@@ -1378,6 +1450,7 @@ avfs_status avfs_capture(avfs_ctx* ctx, const float* t_clk, int32_t n_bins, floa
 
 avfs_status avfs_get_switching_energy(avfs_ctx* ctx, double* out) {
     CHECK_CTX();
+    SETTLE();
     if (!out) return fail(ctx, AVFS_ERR_ARG, "null output");
     if (!ctx->sim_done) return fail(ctx, AVFS_ERR_STATE, "simulate first");
     const int32_t V = (int32_t)ctx->vdd.size();
@@ -1397,6 +1470,7 @@ int32_t avfs_debug_phase_cycles(uint64_t* out16, int32_t reset) {
 
 avfs_status avfs_get_stats(avfs_ctx* ctx, avfs_stats* st) {
     CHECK_CTX();
+    SETTLE();
     if (!st) return fail(ctx, AVFS_ERR_ARG, "null output");
     if (!ctx->sim_done) return fail(ctx, AVFS_ERR_STATE, "simulate first");
     // algorithmic bytes of the sweep: every signal's

@@ -111,11 +111,17 @@ def test_overflow_exact_across_runs(spill_bytes):
 def test_capacity_exhausted_reports_error():
     from paper_conf_date_schneiderw20_b200 import AvfsError
     w = make_config(2, n_pairs=32, n_vdd=1)
+    # simulate is asynchronous: the capacity error surfaces on sync
     with pytest.raises(AvfsError) as e:
-        gpu_run(w, capacity=1, max_rerun_rounds=0, spill_bytes=-1)
+        gpu_run(w, capacity=1, max_rerun_rounds=0, spill_bytes=-1).sync()
     assert e.value.status == 7
     with pytest.raises(AvfsError) as e:
-        gpu_run(w, capacity=1, max_rerun_rounds=0, spill_bytes=64)
+        gpu_run(w, capacity=1, max_rerun_rounds=0, spill_bytes=64).sync()
+    assert e.value.status == 7
+    # ... and so does any call that reads the results
+    ctx = gpu_run(w, capacity=1, max_rerun_rounds=0, spill_bytes=-1)
+    with pytest.raises(AvfsError) as e:
+        ctx.activity()
     assert e.value.status == 7
 
 
@@ -213,7 +219,7 @@ def test_nonpositive_delay_reported():
     w = make_config(1)
     w.library = make_library(0, deg_v=1, const=-2.0)     # d' = -d_nom
     with pytest.raises(AvfsError) as e:
-        gpu_run(w)
+        gpu_run(w).sync()                                   # surfaced on sync (asynchronous simulate)
     assert e.value.status == 6
 
 
