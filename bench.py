@@ -12,8 +12,10 @@ the measurement through the public API with host buffers (H2D of the stimuli,
 D2H of activity + latest arrival inside the timed region).
 For N > 1 launch with torchrun (one rank per GPU).  Slots are independent
 problems, so they shard with no data-path exchange; by default the
-scaling is weak: the pair count grows with N (N x the config's pairs) and each
-rank simulates one config-sized shard ("--scaling strong" fixes the total).
+scaling is strong: BASELINE's config at every N, its slot space split into N
+contiguous shards ("--scaling weak" grows the pairs N-fold instead).  Config 5
+(specified on 8 x B200) runs as one shard of 8 per GPU with --gpus 8, or
+--shard-of 8 on one GPU.
 """
 from __future__ import annotations
 
@@ -212,6 +214,7 @@ def config_dict(w, args):
     n = getattr(args, "shard_slots", None) or w.n_slots
     d.update({"slots": n, "evals_per_step": w.netlist.n_gates * n,
               "mode": "F (FP64 delay polynomials, FP32 times)" if args.quantum == 0 else f"Q (quantum {args.quantum} ps)",
+              "delays": "evaluated in the sweep" if getattr(args, "delay_in_sweep", False) else "delay table",
               "l2": "flushed by a 256 MiB write between timed steps; waveform arena >> L2",
               "parallelism": (f"one slot shard of {args.shard_of} (rank 0), 1 GPU" if args.shard_of > 1 else
                               f"slot-shard x{args.gpus} ({args.scaling})")})
@@ -230,7 +233,13 @@ def main():
     ap.add_argument("--impl", default="avfs", choices=["avfs", "reference"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
-    ap.add_argument("--scaling", default="weak", choices=["weak", "strong"])
+    ap.add_argument("--scaling", default="strong", choices=["weak", "strong"],
+                    help="strong (default): BASELINE's config at every N, slots sharded over ranks; "
+                         "weak: N x the pairs")
+    ap.add_argument("--deg-c", type=int, default=0,
+                    help="N_c of the delay polynomial (3 = the paper's 2-D Table I model, N_v = N_c = 3)")
+    ap.add_argument("--delay-in-sweep", action="store_true",
+                    help="evaluate Eq. (4)/(9) inside the sweep instead of tabulating delays")
     ap.add_argument("--shard-of", type=int, default=0,
                     help="N=1 only: simulate rank 0's shard of an N-GPU run (e.g. config 5, "
                          "specified on 8 x B200, does not fit one GPU whole)")
@@ -239,9 +248,9 @@ def main():
 
     from workloads import make_config
     world, rank, local = dist_setup(args.gpus)
-    w = make_config(args.config)
+    w = make_config(args.config, deg_c=args.deg_c)
     if args.scaling == "weak" and world > 1:
-        w = make_config(args.config, n_pairs=w.stimuli.n_pairs * world)
+        w = make_config(args.config, n_pairs=w.stimuli.n_pairs * world, deg_c=args.deg_c)
     if args.impl == "reference":
         run_reference(args, w, world, rank)
         if world > 1:
@@ -257,7 +266,8 @@ def main():
     ctx = Context(local)
     load_workload(ctx, w.netlist, w.library, w.stimuli, w.vdd)
     cap = args.capacity or w.capacity
-    ctx.set_options(capacity=cap, quantum_ps=args.quantum, warps_per_cta=args.warps_per_cta, profile=True)
+    ctx.set_options(capacity=cap, quantum_ps=args.quantum, warps_per_cta=args.warps_per_cta, profile=True,
+                    delay_in_sweep=args.delay_in_sweep)
     total_slots = w.n_slots
     first, n_local = shard_range(total_slots, rank, world)
     if args.shard_of > 1 and world == 1:

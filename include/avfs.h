@@ -185,6 +185,14 @@ typedef struct {
                                   arrival and energy cover every slot;
                                   waveforms / final values only the last
                                   batch's slots, and capture is refused.   */
+    int32_t delay_in_sweep;    /* 0: a delay kernel tabulates d'(Vdd, gate,
+                                  arc) in binary32 before the sweep (G x V x
+                                  32 B); 1: the sweep evaluates Eq. (4)/(9)
+                                  in FP64 on the fly for the gates that have
+                                  observable input events ("threads
+                                  of the simulation kernels independently
+                                  compute modified delays on-the-fly"), no
+                                  table.  Identical results.               */
 } avfs_options;
 avfs_status avfs_set_options(avfs_ctx *ctx, const avfs_options *opt);
 avfs_status avfs_default_options(avfs_options *opt);

@@ -49,7 +49,7 @@ class avfs_options(C.Structure):
     _fields_ = [("capacity", C.c_int32), ("quantum_ps", C.c_double), ("n_probe", C.c_int32),
                 ("probe_sig", C.POINTER(C.c_int32)), ("keep_all", C.c_int32),
                 ("max_rerun_rounds", C.c_int32), ("warps_per_cta", C.c_int32), ("profile", C.c_int32),
-                ("spill_bytes", C.c_int64), ("max_batch_slots", C.c_int64)]
+                ("spill_bytes", C.c_int64), ("max_batch_slots", C.c_int64), ("delay_in_sweep", C.c_int32)]
 
 
 class avfs_stats(C.Structure):
@@ -248,7 +248,8 @@ class Context:
         self._ck(self.lib.avfs_set_slot_range(self.h, int(first), int(n)))
 
     def set_options(self, capacity=8, quantum_ps=0.0, probes=None, keep_all=False,
-                    max_rerun_rounds=3, warps_per_cta=0, profile=False, spill_bytes=0, max_batch_slots=0):
+                    max_rerun_rounds=3, warps_per_cta=0, profile=False, spill_bytes=0, max_batch_slots=0,
+                    delay_in_sweep=False):
         o = avfs_options()
         self._ck(self.lib.avfs_default_options(C.byref(o)))
         o.capacity = int(capacity)
@@ -263,6 +264,7 @@ class Context:
         o.profile = int(bool(profile))
         o.spill_bytes = int(spill_bytes)
         o.max_batch_slots = int(max_batch_slots)
+        o.delay_in_sweep = int(bool(delay_in_sweep))
         self._ck(self.lib.avfs_set_options(self.h, C.byref(o)))
 
     def simulate(self, stream=None):

@@ -106,7 +106,8 @@ struct avfs_ctx {
     std::vector<uint8_t> is_po;       // per signal
     int32_t depth = 0, kmax = 1, n_dangling = 0;
     std::vector<double> coef;         // coefficient blocks
-    std::vector<uint32_t> coef_off;   // per gate
+    std::vector<uint32_t> coef_off;   // per gate: its cell's coefficient block
+    std::vector<double> phi_c;        // per gate: phi_C(c_load) (0 when deg_c = 0)
 
     // plan (options dependent)
     bool plan_valid = false;
@@ -152,6 +153,7 @@ struct avfs_ctx {
     std::vector<Round> rounds;
     int64_t sim_first = 0, sim_end = 0;
     avfs_stats stats{};
+    DelayParams dparams{};            // delay model of the last simulate (the sweep may evaluate it)
 };
 
 static avfs_status finish_pending(avfs_ctx* ctx);   // settles an asynchronous simulate (defined below)
@@ -262,40 +264,19 @@ avfs_status levelize(avfs_ctx* ctx) {
 }
 
 // ---------------------------------------------------------------- coefficient store
+// The device evaluates Eq. (4) in both variables (NEXT-2): the cells'
+// coefficients go to the device unchanged ([cell][pin][pol][deg_v+1][deg_c+1],
+// P:L139 "stored in the GPU memory"); per gate only z = phi_C(c_g) is
+// precomputed here (P:L117 normalisation of the gate's load).
 void build_coef(avfs_ctx* ctx) {
-    const int dv = ctx->deg_v, dc = ctx->deg_c;
-    const size_t blk = 8 * (size_t)(dv + 1);
-    auto b = [&](int cell, int pin, int pol, int i, int j) {
-        return ctx->beta[((((size_t)cell * 4 + pin) * 2 + pol) * (dv + 1) + i) * (dc + 1) + j];
-    };
+    const size_t nb = (size_t)(ctx->deg_v + 1) * (ctx->deg_c + 1);
+    ctx->coef = ctx->beta;
     ctx->coef_off.assign(ctx->n_gates, 0);
-    if (dc == 0) {
-        const int nc = (int)ctx->cell_nin.size();
-        ctx->coef.assign(nc * blk, 0.0);
-        for (int c = 0; c < nc; ++c)
-            for (int pin = 0; pin < 4; ++pin)
-                for (int pol = 0; pol < 2; ++pol)
-                    for (int i = 0; i <= dv; ++i)
-                        ctx->coef[c * blk + (pin * 2 + pol) * (dv + 1) + i] = b(c, pin, pol, i, 0);
-        for (int32_t g = 0; g < ctx->n_gates; ++g) ctx->coef_off[g] = (uint32_t)(ctx->gate_cell[g] * blk);
-    } else {
-        // Load-time fold of the load capacitance (deg_c > 0): phi_C and
-        // the inner Horner in phi_C with fma, so the kernel's Horner in phi_V
-        // evaluates exactly the nested Horner of Eq. (4).
-        ctx->coef.assign((size_t)ctx->n_gates * blk, 0.0);
-        const double lc0 = std::log2(ctx->c_min), lc1 = std::log2(ctx->c_max);
-        for (int32_t g = 0; g < ctx->n_gates; ++g) {
-            const double z = (std::log2(ctx->c_load[g]) - lc0) / (lc1 - lc0);
-            const int c = ctx->gate_cell[g];
-            for (int pin = 0; pin < 4; ++pin)
-                for (int pol = 0; pol < 2; ++pol)
-                    for (int i = 0; i <= dv; ++i) {
-                        double a = b(c, pin, pol, i, dc);
-                        for (int j = dc - 1; j >= 0; --j) a = std::fma(a, z, b(c, pin, pol, i, j));
-                        ctx->coef[g * blk + (pin * 2 + pol) * (dv + 1) + i] = a;
-                    }
-            ctx->coef_off[g] = (uint32_t)(g * blk);
-        }
+    ctx->phi_c.assign(ctx->n_gates, 0.0);
+    const double lc0 = std::log2(ctx->c_min), lc1 = std::log2(ctx->c_max);
+    for (int32_t g = 0; g < ctx->n_gates; ++g) {
+        ctx->coef_off[g] = (uint32_t)((size_t)ctx->gate_cell[g] * 8 * nb);
+        if (ctx->deg_c > 0) ctx->phi_c[g] = (std::log2(ctx->c_load[g]) - lc0) / (lc1 - lc0);
     }
 }
 
@@ -372,6 +353,7 @@ avfs_status upload_netlist(avfs_ctx* ctx) {
         d.ttk = ttm | ((uint32_t)k << 16) | ((ctx->is_po[ctx->n_pi + g] ? 1u : 0u) << 24);
         d.fanout = (uint32_t)std::min<int64_t>(ctx->fanout[ctx->n_pi + g], 0xFFFFFF);
         e.coef_off = ctx->coef_off[g];
+        e.z = ctx->phi_c[g];
         e.k = (uint32_t)k;
         e.island = (uint32_t)ctx->island[g];
         for (int p = 0; p < k; ++p)
@@ -933,7 +915,8 @@ static avfs_status run_round(avfs_ctx* ctx, Round& R, int round_idx, const int32
     p.level_ptr = ctx->d_level_ptr.as<int32_t>();
     p.depth = ctx->depth;
     p.n_gates = ctx->n_gates;
-    p.dtab = ctx->d_dtab.as<float4>();
+    p.dtab = ctx->opt.delay_in_sweep ? nullptr : ctx->d_dtab.as<float4>();
+    p.dp = ctx->dparams;
     p.p1t = ctx->d_p1t.as<uint32_t>();
     p.p2t = ctx->d_p2t.as<uint32_t>();
     p.n_pw = (int32_t)((ctx->n_pairs + 31) / 32);
@@ -1124,21 +1107,27 @@ avfs_status avfs_simulate(avfs_ctx* ctx, void* cuda_stream) {
     CK(cudaMemsetAsync(ctx->d_err.p, 0, 16, ctx->stream));
     CK(ctx->d_enc.ensure(8));
     CK(cudaMemsetAsync(ctx->d_enc.p, 0, 8, ctx->stream));
-    // delay computation kernel: d'(gate, pin, pol, Vdd) in FP64 -> binary32 table
-    CK(ctx->d_dtab.ensure((size_t)V * std::max(ctx->n_gates, 1) * 8 * sizeof(float)));
+    // delay computation kernel: d'(gate, pin, pol, Vdd) in FP64 ->
+    // binary32 table, or (delay_in_sweep) only the d' > 0 check, the sweep
+    // then evaluating Eq. (4)/(9) itself for the gates that need delays
+    const bool in_sweep = ctx->opt.delay_in_sweep != 0;
+    if (!in_sweep) CK(ctx->d_dtab.ensure((size_t)V * std::max(ctx->n_gates, 1) * 8 * sizeof(float)));
+    else ctx->d_dtab.release();
     {
-        DelayParams dp{};
+        DelayParams& dp = ctx->dparams;
+        dp = DelayParams{};
         dp.dd = ctx->d_ddesc.as<DelayDesc>();
         dp.n_gates = ctx->n_gates;
         dp.coef = ctx->d_coef.as<double>();
         dp.deg_v = ctx->deg_v;
+        dp.deg_c = ctx->deg_c;
         dp.vdd = ctx->d_vdd.as<double>();
         dp.n_vdd = V;
         dp.n_isl = ctx->n_isl;
         dp.v_min = ctx->v_min;
         dp.v_max = ctx->v_max;
         dp.quantum = ctx->opt.quantum_ps;
-        dp.dtab = ctx->d_dtab.as<float>();
+        dp.dtab = in_sweep ? nullptr : ctx->d_dtab.as<float>();
         dp.err = ctx->d_err.as<int32_t>();
         CK(launch_delays(dp, ctx->stream));
         ctx->stats.launches++;

@@ -57,27 +57,32 @@ struct alignas(16) GateDesc {
 };
 static_assert(sizeof(GateDesc) == 32, "GateDesc layout");
 
-// Inputs of the delay computation kernel: per sorted gate.
+// Inputs of the delay computation: per sorted gate.  The delay of
+// arc (pin, pol) at supply v is Eq. (4)/(9) with the cell's coefficients
+// beta[deg_v+1][deg_c+1] (block at coef_off + (2 pin + pol) nb, nb =
+// (deg_v+1)(deg_c+1)), x = phi_V(v) and the gate's z = phi_C(c_load)
+// (computed at load from the gate's load, 0 when deg_c = 0).
 struct alignas(16) DelayDesc {
     double dnom[2 * KMAX];   // [pin][pol] nominal delay, ps
-    uint32_t coef_off;       // offset (doubles) of the [pin][pol][deg_v+1] coefficient block
+    double z;                // phi_C(c_g)
+    uint32_t coef_off;       // offset (doubles) of the cell's [pin][pol][deg_v+1][deg_c+1] block
     uint32_t k;
     uint32_t island;         // voltage island (NEXT-2)
-    uint32_t pad;
+    uint32_t pad[3];
 };
-static_assert(sizeof(DelayDesc) == 80, "DelayDesc layout");
+static_assert(sizeof(DelayDesc) == 96, "DelayDesc layout");
 
 struct DelayParams {
     const DelayDesc* __restrict__ dd;
     int32_t n_gates;
-    const double* __restrict__ coef;
-    int32_t deg_v;
+    const double* __restrict__ coef;         // [cell][pin][pol][deg_v+1][deg_c+1]
+    int32_t deg_v, deg_c;
     const double* __restrict__ vdd;          // [n_vdd][n_isl] volts
     int32_t n_vdd;
     int32_t n_isl;
     double v_min, v_max;
     double quantum;                          // 0: F mode
-    float* dtab;                             // [n_vdd][n_gates][8] delays (binary32), ps
+    float* dtab;                             // [n_vdd][n_gates][8] delays (binary32), ps; null: check only
     int32_t* err;                            // bit 0: non-positive delay
 };
 
@@ -86,7 +91,8 @@ struct SweepParams {
     const int32_t* __restrict__ level_ptr;  // [depth+1] offsets into gates (level 1..depth)
     int32_t depth;
     int32_t n_gates;
-    const float4* __restrict__ dtab;        // [n_vdd][n_gates][2] float4 delays
+    const float4* __restrict__ dtab;        // [n_vdd][n_gates][2] float4 delays, or null: evaluated in the sweep
+    DelayParams dp;                         // delay model (used when dtab is null)
     const uint32_t* __restrict__ p1t;       // [n_pi][n_pw] bit-transposed stimuli
     const uint32_t* __restrict__ p2t;
     int32_t n_pw;                           // pair-warps (ceil(n_pairs/32))

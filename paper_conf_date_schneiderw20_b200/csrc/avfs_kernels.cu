@@ -267,6 +267,25 @@ __device__ __forceinline__ void eval_masks(uint32_t tt, const uint32_t (&X)[4], 
     A = c0 & c1;
 }
 
+// Eq. (4) by nested Horner in FP64 with FMA, outer in x = phi_V(v) from
+// i = deg_v down, inner in z = phi_C(c), then
+// Eq. (9) d' = d_nom (1 + f), Q-mode rounding (reading C12), one rounding to
+// binary32 (reading C11).  cf: [deg_v+1][deg_c+1].
+__device__ __forceinline__ float arc_delay(const double* __restrict__ cf, int dv, int dc, double x, double z,
+                                           double dnom, double q, bool& bad) {
+    double f = 0.0;
+    for (int i = dv; i >= 0; --i) {
+        const double* row = cf + i * (dc + 1);
+        double a = __ldg(row + dc);
+        for (int j = dc - 1; j >= 0; --j) a = fma(a, z, __ldg(row + j));
+        f = (i == dv) ? a : fma(f, x, a);
+    }
+    double d = dnom * (1.0 + f);
+    if (q > 0.0) d = q * rint(d / q);
+    bad = !(d > 0.0);
+    return __double2float_rn(d);
+}
+
 __device__ __forceinline__ void poison_bit(const SweepParams& p, int64_t gi, uint32_t sig) {
     const uint64_t gbit = (uint64_t)gi * (uint32_t)p.n_gates + (sig - (uint32_t)p.n_pi);
     atomicOr(p.pois + (gbit >> 5), 1u << (gbit & 31u));
@@ -284,8 +303,10 @@ __device__ __forceinline__ int phase_a(const SweepParams& p, const Grp& G, int g
     if (on) {
         d0 = __ldg(gd + 2 * g);
         d1 = __ldg(gd + 2 * g + 1);
-        dl0 = __ldg(dt + 2 * g);
-        dl1 = __ldg(dt + 2 * g + 1);
+        if (dt) {
+            dl0 = __ldg(dt + 2 * g);
+            dl1 = __ldg(dt + 2 * g + 1);
+        }
     }
     const uint32_t tt = d1.z & 0xffffu, K = on ? (d1.z >> 16) & 0xffu : 0u;
     const uint32_t loc[4] = {d0.x, d0.y, d0.z, d0.w};
@@ -352,6 +373,27 @@ __device__ __forceinline__ int phase_a(const SweepParams& p, const Grp& G, int g
             if (!RERUN || counted) poison_bit(p, G.gi, sig);
             if (own) p.ovf[G.gi] = 1;
         }
+    }
+    if (!dt && active) {                      // Eq. (4)/(9) evaluated here, for the gates that need delays
+        const DelayParams& P = p.dp;
+        const DelayDesc& D = P.dd[g];
+        const double v = __ldg(P.vdd + (size_t)G.kv * P.n_isl + D.island);
+        const double x = (v - P.v_min) / (P.v_max - P.v_min);
+        const int nb = (P.deg_v + 1) * (P.deg_c + 1);
+        float dd[8];
+        bool bad = false;
+#pragma unroll
+        for (int e = 0; e < 8; ++e) {
+            dd[e] = 1.0f;
+            if ((uint32_t)e < 2 * K) {
+                bool b;
+                dd[e] = arc_delay(P.coef + D.coef_off + e * nb, P.deg_v, P.deg_c, x, D.z, D.dnom[e], P.quantum, b);
+                bad |= b;
+            }
+        }
+        if (bad) atomicOr(P.err, 1);
+        dl0 = make_float4(dd[0], dd[1], dd[2], dd[3]);
+        dl1 = make_float4(dd[4], dd[5], dd[6], dd[7]);
     }
     const uint32_t bal = __ballot_sync(FULL, active);
     if (active) {
@@ -642,7 +684,7 @@ __global__ void __launch_bounds__(AVFS_SWEEP_THREADS, 1) sweep_kernel(const Swee
         const int64_t i = i0 + sg;
         const bool valid = i < p.n_sw;                 // idle warps still meet every level barrier
         group_setup(p, valid ? i : i0, lane, G);
-        const float4* dt = p.dtab + (int64_t)G.kv * p.n_gates * 2;
+        const float4* dt = p.dtab ? p.dtab + (int64_t)G.kv * p.n_gates * 2 : nullptr;
         if (wl == 0 && lane == 0) {
             sts_u32(ctr_s, 0u);
             sts_u32(ctr_s + 4, 0u);
@@ -776,11 +818,8 @@ cudaError_t launch_sweep(const SweepParams& p, bool rerun, int grid, int warps_p
 
 // ---------------------------------------------------------------------------
 // Delay computation kernel (P:L139, P:L152-L160 steps 3-5): one thread per
-// (operating point, gate, pin, polarity).  f(P) of Eq. (4) by Horner with FMA
-// in FP64, d' = d_nom (1 + f) (Eq. 9), optional Q-mode rounding
-// (reading C12), rounded once to binary32 (reading C11).  The sweep reads the
-// 8 delays of a gate as two uniform float4 loads per 32 slots.
-// ---------------------------------------------------------------------------
+// (operating point, gate, pin, polarity); fills the table the sweep reads,
+// or (dtab null) only checks every delay for d' > 0 (reading C14).
 __global__ void delay_kernel(const DelayParams p) {
     const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     const int64_t total = (int64_t)p.n_vdd * p.n_gates * 8;
@@ -794,15 +833,12 @@ __global__ void delay_kernel(const DelayParams p) {
     if (e < 2 * (int)D.k) {
         const double v = p.vdd[(size_t)kv * p.n_isl + D.island];           // gate's island supply (NEXT-2)
         const double x = (v - p.v_min) / (p.v_max - p.v_min);                // phi_V
-        const double* cf = p.coef + D.coef_off + e * (p.deg_v + 1);
-        double f = cf[p.deg_v];
-        for (int i = p.deg_v - 1; i >= 0; --i) f = fma(f, x, cf[i]);
-        double d = D.dnom[e] * (1.0 + f);
-        if (p.quantum > 0.0) d = p.quantum * rint(d / p.quantum);
-        if (!(d > 0.0)) atomicOr(p.err, 1);
-        out = __double2float_rn(d);
+        const int nb = (p.deg_v + 1) * (p.deg_c + 1);
+        bool bad;
+        out = arc_delay(p.coef + D.coef_off + e * nb, p.deg_v, p.deg_c, x, D.z, D.dnom[e], p.quantum, bad);
+        if (bad) atomicOr(p.err, 1);
     }
-    p.dtab[t] = out;
+    if (p.dtab) p.dtab[t] = out;
 }
 
 cudaError_t launch_delays(const DelayParams& p, cudaStream_t st) {

@@ -17,7 +17,8 @@ REPORT = []          # per-compare taint summaries, printed by conftest at sessi
 
 
 def gpu_run(w_or_parts, quantum=0.0, capacity=None, keep_all=True, probes=None, slot_range=None,
-            stream=None, warps_per_cta=0, max_rerun_rounds=3, netlist=None, spill_bytes=0, max_batch_slots=0):
+            stream=None, warps_per_cta=0, max_rerun_rounds=3, netlist=None, spill_bytes=0, max_batch_slots=0,
+            delay_in_sweep=False):
     from paper_conf_date_schneiderw20_b200 import Context, load_workload
     nl = netlist if netlist is not None else w_or_parts.netlist
     ctx = Context(0)
@@ -25,7 +26,7 @@ def gpu_run(w_or_parts, quantum=0.0, capacity=None, keep_all=True, probes=None, 
     ctx.set_options(capacity=capacity or w_or_parts.capacity, quantum_ps=quantum, keep_all=keep_all,
                     probes=probes, warps_per_cta=warps_per_cta, max_rerun_rounds=max_rerun_rounds,
                     spill_bytes=spill_bytes, max_batch_slots=max_batch_slots,
-                    profile=True)
+                    delay_in_sweep=delay_in_sweep, profile=True)
     if slot_range is not None:
         ctx.set_slot_range(*slot_range)
     ctx.simulate(stream)

@@ -71,6 +71,31 @@ def test_fullsize_sampled_po_parity(cfg, quantum):
     ctx.close()
 
 
+@pytest.mark.parametrize("quantum,in_sweep", [(2.0 ** -8, False), (0.0, True)])
+def test_fullsize_config3_2d_polynomial(quantum, in_sweep):
+    """NEXT-2 at full size: config 3 (b17-shaped, 4096 x 16 slots) with the
+    paper's N_v = N_c = 3 two-dimensional delay model evaluated on the device
+    (delay kernel / inside the sweep); sampled PO waveforms vs the oracle."""
+    w = make_config(3, deg_c=3)
+    nl = w.netlist
+    ctx = gpu_run(w, keep_all=False, quantum=quantum, delay_in_sweep=in_sweep)
+    slots = sample_slots(w, 64)
+    P = w.stimuli.n_pairs
+    ref = oracle.simulate(nl, w.library, w.stimuli, w.vdd, slots % P, slots // P, quantum=quantum,
+                          cap=64, out_sig=nl.po_sig)
+    cap = max(1, min(64, int(ref.count.max())))
+    init = np.zeros((len(slots), len(nl.po_sig)), np.uint8)
+    cnt = np.zeros((len(slots), len(nl.po_sig)), np.int32)
+    times = np.zeros((len(slots), len(nl.po_sig), cap), np.float32)
+    for i, s in enumerate(slots):
+        a, b, c = gpu_waveforms(ctx, nl.po_sig, int(s), 1, cap)
+        init[i], cnt[i], times[i] = a[0], b[0], c[0]
+    ref.times = ref.times[:, :, :cap]
+    r = compare(ref, init, cnt, times, quantum, f"cfg3-2d-q{quantum}-{'sweep' if in_sweep else 'table'}")
+    assert r["events"] > 0
+    ctx.close()
+
+
 @pytest.mark.parametrize("cfg", [2, 3, 4])
 def test_fullsize_window_activity(cfg):
     w = make_config(cfg)

@@ -70,12 +70,31 @@ def test_random_dag_four_input_cells(quantum):
     full_compare(w, quantum, label="rdag4")
 
 
-def test_deg_c_folded_polynomial_q_mode():
-    """Full 2-D (v, c) polynomial (Eq. 4) with load folding: bit-exact in Q mode."""
-    nl = random_dag(99, 1500, 40, 18)
-    w = Workload(0, "rdag-2d", nl, make_library(98, deg_v=3, deg_c=3), make_stimuli(97, nl.n_pi, 64),
+@pytest.mark.parametrize("quantum,in_sweep", [(Q, False), (0.0, False), (Q, True), (0.0, True)])
+def test_2d_polynomial_on_device(quantum, in_sweep):
+    """NEXT-2: the full 2-D (v, c) polynomial of Eq. (4) (N_v = N_c = 3, the
+    paper's 16 coefficients) evaluated on the device -- by the
+    delay kernel or inside the sweep -- on a mid-size DAG: Q mode bit-exact,
+    F mode within the time tolerance."""
+    nl = random_dag(99, 6000, 120, 30)
+    w = Workload(0, "rdag-2d", nl, make_library(98, deg_v=3, deg_c=3), make_stimuli(97, nl.n_pi, 96),
                  np.array([0.62, 0.8, 1.05]), 8)
-    full_compare(w, Q, label="2d")
+    full_compare(w, quantum, label=f"2d-{'sweep' if in_sweep else 'table'}", delay_in_sweep=in_sweep)
+
+
+@pytest.mark.parametrize("quantum", [Q, 0.0])
+def test_delay_in_sweep_identical_to_table(quantum):
+    """On-the-fly delays in the sweep give bit-identical results to
+    the delay table, with islands, reruns and several groups per CTA."""
+    w = make_config(3, n_pairs=96, n_vdd=4, scale=0.1)
+    outs = []
+    for in_sweep in (False, True):
+        ctx = gpu_run(w, quantum=quantum, capacity=2, delay_in_sweep=in_sweep, spill_bytes=4096)
+        sig = np.arange(w.netlist.n_signals, dtype=np.int32)
+        outs.append((ctx.activity(), ctx.latest_arrival(), *ctx.waveforms(sig, 0, w.n_slots, cap=24)))
+        ctx.close()
+    for a, b in zip(*outs):
+        assert np.array_equal(a, b)
 
 
 @pytest.mark.parametrize("quantum", [Q, 0.0])

@@ -44,13 +44,15 @@ class Workload:
             "workload": self.name, "cfg": self.cfg, "gates": self.netlist.n_gates,
             "pis": self.netlist.n_pi, "pos": int(len(self.netlist.po_sig)),
             "pairs": self.stimuli.n_pairs, "vdd_points": int(len(self.vdd)),
-            "deg_v": self.library.deg_v, "capacity": self.capacity,
+            "deg_v": self.library.deg_v, "deg_c": self.library.deg_c, "capacity": self.capacity,
         }
 
 
 def make_config(i: int, n_pairs: int | None = None, n_vdd: int | None = None,
-                scale: float = 1.0) -> Workload:
-    """Build config i (1..5).  n_pairs / n_vdd / scale shrink it for tests."""
+                scale: float = 1.0, deg_c: int = 0) -> Workload:
+    """Build config i (1..5).  n_pairs / n_vdd / scale shrink it for tests.
+    deg_c > 0 (configs 2-5): the paper's 2-D (v, c) delay model with N_c =
+    deg_c (Table I uses N_v = N_c = 3)."""
     if i == 1:
         nl = c17(seed=2001)
         lib = make_library(2001, deg_v=2, spread=0.1)
@@ -60,7 +62,7 @@ def make_config(i: int, n_pairs: int | None = None, n_vdd: int | None = None,
         cap = 8
     elif i == 2:
         nl = array_multiplier(16, seed=2002)
-        lib = make_library(2002, deg_v=3, spread=0.2)
+        lib = make_library(2002, deg_v=3, deg_c=deg_c, spread=0.2)
         P = n_pairs or 10_000
         stim = make_stimuli(3002, nl.n_pi, P, toggle=0.5)
         vdd = np.linspace(0.6, 1.1, 8)
@@ -82,7 +84,7 @@ def make_config(i: int, n_pairs: int | None = None, n_vdd: int | None = None,
             mix["XNOR2"] += 0.01
         nl = random_dag(1000 + i, G, PI, L, n_po_min=PO, mix=mix,
                         delay_seed=2000 + i, name=CONFIG_NAMES[i])
-        lib = make_library(2000 + i, deg_v=3, spread=0.2)
+        lib = make_library(2000 + i, deg_v=3, deg_c=deg_c, spread=0.2)
         P = n_pairs or P0
         stim = make_stimuli(3000 + i, nl.n_pi, P, toggle=0.5)
         vdd = (np.linspace(0.6, 1.1, V0) if i != 5 else 0.6 + 0.01 * np.arange(51))
