@@ -96,26 +96,88 @@ def test_fullsize_config3_2d_polynomial(quantum, in_sweep):
     ctx.close()
 
 
-@pytest.mark.parametrize("cfg", [2, 3, 4])
-def test_fullsize_window_activity(cfg):
+def _window_activity(cfg, quantum, first, n, **kw):
     w = make_config(cfg)
     nl = w.netlist
     P, V = w.stimuli.n_pairs, len(w.vdd)
-    first = (P * V) // 2 + 7
-    n = 64
-    ctx = gpu_run(w, keep_all=False, slot_range=(first, n))
+    ctx = gpu_run(w, keep_all=False, slot_range=(first, n), quantum=quantum, **kw)
     act = ctx.activity().astype(np.int64)
+    st = ctx.stats()
     slots = np.arange(first, first + n)
-    ref = oracle.simulate(nl, w.library, w.stimuli, w.vdd, slots % P, slots // P, quantum=0.0, cap=0)
-    cnt = ref.count.sum(0)
+    ref = oracle.simulate(nl, w.library, w.stimuli, w.vdd, slots % P, slots // P, quantum=quantum, cap=0)
     k = slots // P
+    tainted = 0
     for kv in np.unique(k):
         sel = k == kv
-        ok = ref.taint[sel].sum(0) == 0
+        ok = ref.taint[sel].sum(0) == 0                  # every signal in Q mode
+        tainted += int((~ok).sum())
         got = act[:, kv]
         want = ref.count[sel].sum(0)
         assert np.array_equal(got[ok], want[ok]), f"cfg{cfg} vdd{kv}"
     others = np.setdiff1d(np.arange(V), np.unique(k))
     assert np.all(act[:, others] == 0)
-    assert cnt.sum() > 0
+    assert ref.count.sum() > 0
+    if quantum > 0:
+        assert tainted == 0
+    print(f"[window] cfg{cfg} q={quantum} slots [{first}, {first + n}) signals={nl.n_signals} "
+          f"tainted_rows={tainted} batches={st['batches']}")
+    ctx.close()
+    return st
+
+
+@pytest.mark.parametrize("cfg,quantum", [(2, 0.0), (3, 0.0), (4, 0.0),
+                                         (2, 2.0 ** -8), (3, 2.0 ** -8), (4, 2.0 ** -8),
+                                         pytest.param(5, 2.0 ** -8, marks=pytest.mark.slow)])
+def test_fullsize_window_activity(cfg, quantum):
+    """Activity of EVERY signal over a 64-slot window of the full-size config
+    (the shard mechanism) equals the oracle's counts; Q mode: no exclusions."""
+    w = make_config(cfg)
+    _window_activity(cfg, quantum, w.n_slots // 2 + 7, 64)
+
+
+@pytest.mark.slow
+def test_config5_multibatch_window_activity():
+    """Whole-config-5 netlist (2M gates) in forced slot batches: a 160-slot
+    window across two Vdd points run as five 32-slot batches on one reused
+    arena; activity of every signal equals the oracle's (Q mode)."""
+    first = 1024 * 30 - 64                               # straddles Vdd points 29 / 30
+    st = _window_activity(5, 2.0 ** -8, first, 160, max_batch_slots=32)
+    assert st["batches"] == 5
+
+
+@pytest.mark.slow
+@pytest.mark.parametrize("quantum", [2.0 ** -8, 0.0])
+def test_config5_all_shards(quantum):
+    """Config 5 as its 8 GPU shards, run one after another on this GPU: two
+    sampled slots per shard (all 51 Vdd points 0.60-1.10 V are covered by the
+    shards), PO waveforms vs the oracle."""
+    from paper_conf_date_schneiderw20_b200 import Context, load_workload, shard_range
+    w = make_config(5)
+    nl = w.netlist
+    P = w.stimuli.n_pairs
+    ctx = Context(0)
+    load_workload(ctx, nl, w.library, w.stimuli, w.vdd)
+    ctx.set_options(capacity=w.capacity, quantum_ps=quantum, keep_all=False)
+    rng = np.random.default_rng(55)
+    all_slots, rows = [], []
+    for r in range(8):
+        first, cnt = shard_range(w.n_slots, r, 8)
+        ctx.set_slot_range(first, cnt)
+        ctx.simulate()
+        slots = np.sort(first + rng.choice(cnt, size=2, replace=False))
+        for s in slots:
+            rows.append(gpu_waveforms(ctx, nl.po_sig, int(s), 1, 64))
+        all_slots.extend(slots.tolist())
+    slots = np.array(all_slots)
+    assert len(np.unique(slots // P)) >= 8
+    ref = oracle.simulate(nl, w.library, w.stimuli, w.vdd, slots % P, slots // P, quantum=quantum,
+                          cap=64, out_sig=nl.po_sig)
+    cap = max(1, min(64, int(ref.count.max())))
+    init = np.stack([a[0] for a, _, _ in rows])
+    cnt = np.stack([b[0] for _, b, _ in rows])
+    times = np.stack([c[0][:, :cap] for _, _, c in rows])
+    ref.times = ref.times[:, :, :cap]
+    r = compare(ref, init, cnt, times, quantum, f"cfg5-8shards-q{quantum}", max_taint=1.0)
+    assert r["tainted_differ"] <= 0.01 * max(r["tainted"], 1)
+    assert r["events"] > 0
     ctx.close()
