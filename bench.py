@@ -238,6 +238,8 @@ def main():
                          "weak: N x the pairs")
     ap.add_argument("--deg-c", type=int, default=0,
                     help="N_c of the delay polynomial (3 = the paper's 2-D Table I model, N_v = N_c = 3)")
+    ap.add_argument("--spill-bytes", type=int, default=0,
+                    help="pass-0 spill heap bytes (0 auto, <0 none): a capped heap forces overflow reruns (H7)")
     ap.add_argument("--delay-in-sweep", action="store_true",
                     help="evaluate Eq. (4)/(9) inside the sweep instead of tabulating delays")
     ap.add_argument("--shard-of", type=int, default=0,
@@ -267,7 +269,7 @@ def main():
     load_workload(ctx, w.netlist, w.library, w.stimuli, w.vdd)
     cap = args.capacity or w.capacity
     ctx.set_options(capacity=cap, quantum_ps=args.quantum, warps_per_cta=args.warps_per_cta, profile=True,
-                    delay_in_sweep=args.delay_in_sweep)
+                    delay_in_sweep=args.delay_in_sweep, spill_bytes=args.spill_bytes)
     total_slots = w.n_slots
     first, n_local = shard_range(total_slots, rank, world)
     if args.shard_of > 1 and world == 1:
@@ -302,14 +304,16 @@ def main():
     clocks = ClockSampler(local)
     clocks.start()
     ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
-    sweep_ms = []
+    sweep_ms, rerun_ms = [], []
     for i in range(args.steps):
         with torch.cuda.stream(stream):
             flush.zero_()
         ev[i][0].record(stream)
         step()
         ev[i][1].record(stream)
-        sweep_ms.append(ctx.stats()["sweep_ms"])
+        st_i = ctx.stats()
+        sweep_ms.append(st_i["sweep_ms"])
+        rerun_ms.append(st_i["rerun_ms"])
     torch.cuda.synchronize()
     ck = clocks.stop()
     step_ms = [a.elapsed_time(b) for a, b in ev]
@@ -383,7 +387,11 @@ def main():
             "clocks": ck,
             "stats": {k: stats[k] for k in ("evals", "slot_warps", "overflow_slot_warps", "rerun_rounds", "spill_bytes", "batches",
                                             "grid", "warps_per_cta", "n_scratch_buffers", "n_pinned",
-                                            "arena_bytes", "launches")},
+                                            "arena_bytes", "launches", "enc_bytes")},
+            "overflow": {"groups_rerun": stats["overflow_slot_warps"], "groups": stats["slot_warps"],
+                         "rerun_fraction": stats["overflow_slot_warps"] / max(stats["slot_warps"], 1),
+                         "rerun_ms": float(np.mean(rerun_ms)),
+                         "rerun_share_of_step": float(np.mean(rerun_ms)) / (t_total / args.steps)},
             "paper_context": "P100 (CUDA 10): 1186 MEPS average at one Vdd, 310-1785x over a serial "
                              "commercial event-driven simulator on a Xeon E5-2687W v2 core (PAPER.md L203)",
         }

@@ -289,6 +289,8 @@ typedef struct {
     int64_t batches;             /* slot batches of the last simulate         */
     int64_t enc_bytes;           /* algorithmic bytes of the stored encoding
                                     (records, entries, times)  */
+    double rerun_ms;             /* CUDA-event time of the overflow reruns
+                                    (profile=1), all batches                  */
 } avfs_stats;
 avfs_status avfs_get_stats(avfs_ctx *ctx, avfs_stats *st);
 

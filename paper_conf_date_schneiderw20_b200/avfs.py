@@ -58,7 +58,8 @@ class avfs_stats(C.Structure):
                 ("arena_bytes", C.c_int64), ("alg_bytes", C.c_int64), ("grid", C.c_int32),
                 ("warps_per_cta", C.c_int32), ("n_scratch_buffers", C.c_int32), ("n_pinned", C.c_int32),
                 ("sim_ms", C.c_double), ("sweep_ms", C.c_double), ("spill_bytes", C.c_int64),
-                ("spill_heap_bytes", C.c_int64), ("batches", C.c_int64), ("enc_bytes", C.c_int64)]
+                ("spill_heap_bytes", C.c_int64), ("batches", C.c_int64), ("enc_bytes", C.c_int64),
+                ("rerun_ms", C.c_double)]
 
     def as_dict(self) -> dict:
         return {f: getattr(self, f) for f, _ in self._fields_}

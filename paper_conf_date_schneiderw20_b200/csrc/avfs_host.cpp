@@ -66,6 +66,7 @@ struct Round {
     int64_t spill_words = 0;         // heap words allocated for this round
     int64_t spill_req = 0;           // words requested by the round's gate-warps (incl. failed)
     int32_t grp = 1;                 // slot groups per sweep CTA
+    bool spill_exact = false;        // the caller fixed the heap size (options.spill_bytes > 0): no headroom
     int32_t split = 1;               // sweep CTAs per slot group
 };
 
@@ -139,7 +140,7 @@ struct avfs_ctx {
     int64_t spill_per_group = 0;      // largest heap words per slot group asked for so far (sizing hint)
     int32_t n_batches = 1;            // slot batches of the last simulate (readback keeps the last)
     int32_t* h_pinned = nullptr;      // small pinned host buffer (count, err)
-    cudaEvent_t ev0 = nullptr, ev1 = nullptr;
+    cudaEvent_t ev0 = nullptr, ev1 = nullptr, ev2 = nullptr, ev3 = nullptr;   // pass-0 sweep; reruns
 
     // last simulation
     bool sim_done = false, map_valid = false;
@@ -450,7 +451,8 @@ avfs_status avfs_create(int cuda_device, avfs_ctx** out) {
         if (cudaSetDevice(cuda_device) != cudaSuccess ||
             cudaDeviceGetAttribute(&ctx->n_sm, cudaDevAttrMultiProcessorCount, cuda_device) != cudaSuccess ||
             cudaMallocHost(&ctx->h_pinned, 64) != cudaSuccess ||
-            cudaEventCreate(&ctx->ev0) != cudaSuccess || cudaEventCreate(&ctx->ev1) != cudaSuccess) {
+            cudaEventCreate(&ctx->ev0) != cudaSuccess || cudaEventCreate(&ctx->ev1) != cudaSuccess ||
+            cudaEventCreate(&ctx->ev2) != cudaSuccess || cudaEventCreate(&ctx->ev3) != cudaSuccess) {
             cudaGetLastError();
             delete ctx;
             return AVFS_ERR_CUDA;
@@ -467,6 +469,8 @@ void avfs_destroy(avfs_ctx* ctx) {
         if (ctx->h_pinned) cudaFreeHost(ctx->h_pinned);
         if (ctx->ev0) cudaEventDestroy(ctx->ev0);
         if (ctx->ev1) cudaEventDestroy(ctx->ev1);
+        if (ctx->ev2) cudaEventDestroy(ctx->ev2);
+        if (ctx->ev3) cudaEventDestroy(ctx->ev3);
     }
     delete ctx;
 }
@@ -831,6 +835,12 @@ avfs_status avfs_sync(avfs_ctx* ctx) {
     return AVFS_OK;
 }
 
+static void release_rerun_memory(avfs_ctx* ctx) {
+    for (size_t r = 1; r < ctx->arena.size(); ++r) ctx->arena[r].release();
+    for (size_t r = 1; r < ctx->recs.size(); ++r) ctx->recs[r].release();
+    for (size_t r = 1; r < ctx->spill.size(); ++r) ctx->spill[r].release();
+}
+
 static avfs_status run_round(avfs_ctx* ctx, Round& R, int round_idx, const int32_t* d_sw_list,
                              const int32_t* d_prev_idx, bool timed) {
     const bool rerun = round_idx > 0;
@@ -853,18 +863,19 @@ static avfs_status run_round(avfs_ctx* ctx, Round& R, int round_idx, const int32
     if (const char* e = getenv("AVFS_GROUPS_PER_CTA")) grp = std::max(1, std::min(wpc, atoi(e)));
     while (wpc % grp) grp /= 2;
     // few slot groups for the SMs (last wave mostly empty, e.g. reruns): S
-    // co-resident CTAs share a group; S minimises waves / S, ties to the
-    // smaller S, and every warp keeps >= 2 gates of a level
+    // co-resident CTAs share a group; S minimises waves / S, with 5 % per
+    // doubling of S for the cross-CTA level barriers, ties to the smaller S,
+    // and every warp keeps >= 2 gates of a level
     int split = 1;
     if (grp == 1) {
         double best = 1e300;
-        for (int S = 1; S <= 4; S *= 2) {
+        for (int S = 1, lg = 0; S <= 16; S *= 2, ++lg) {
             if (S > 1 && per_level / S / wpc < 2.0) break;
             const int64_t g = std::max<int64_t>(resident / S * S, S);
-            const double cost = (double)((R.n_sw * S + g - 1) / g) / S;
+            const double cost = (double)((R.n_sw * S + g - 1) / g) / S * (1.0 + 0.05 * lg);
             if (cost < best - 1e-9) { best = cost; split = S; }
         }
-        if (const char* e = getenv("AVFS_SPLIT")) split = std::max(1, std::min(4, atoi(e)));
+        if (const char* e = getenv("AVFS_SPLIT")) split = std::max(1, std::min(16, atoi(e)));
     }
     R.grp = grp;
     R.split = split;
@@ -880,7 +891,16 @@ static avfs_status run_round(avfs_ctx* ctx, Round& R, int round_idx, const int32
     const int64_t n_buf = (int64_t)ctx->n_pinned + ctx->n_scratch;
     if ((uint64_t)R.n_sw * R.region_bytes >= (1ull << 32))
         return fail(ctx, AVFS_ERR_NOMEM, "slot-group stride exceeds 4 GiB; restrict the slot range");
-    CK(ctx->arena[round_idx].ensure((size_t)std::max<int64_t>(n_buf, 1) * R.n_sw * R.region_bytes));
+    {
+        const size_t bytes = (size_t)std::max<int64_t>(n_buf, 1) * R.n_sw * R.region_bytes;
+        cudaError_t e = ctx->arena[round_idx].ensure(bytes);
+        if (e == cudaErrorMemoryAllocation && round_idx == 0) {   // retained rerun memory: give it back
+            cudaGetLastError();
+            release_rerun_memory(ctx);
+            e = ctx->arena[round_idx].ensure(bytes);
+        }
+        CK(e);
+    }
     CK(ctx->recs[round_idx].ensure((size_t)std::max<int64_t>(n_buf, 1) * R.n_sw * sizeof(uint4)));
     CK(ctx->d_ovf.ensure(std::max<int64_t>(R.n_sw, 1) * sizeof(int32_t)));
     CK(cudaMemsetAsync(ctx->d_ovf.p, 0, R.n_sw * sizeof(int32_t), ctx->stream));
@@ -889,13 +909,15 @@ static avfs_status run_round(avfs_ctx* ctx, Round& R, int round_idx, const int32
     R.spill_words = 0;
     if (R.spill_want > 0 && ctx->spill[round_idx].n >= (size_t)R.spill_want * 4) {
         R.spill_words = (int64_t)(ctx->spill[round_idx].n / 4);     // reuse the heap (with its headroom)
+        if (R.spill_exact) R.spill_words = R.spill_want;
     } else if (R.spill_want > 0) {
+        if (round_idx == 0) release_rerun_memory(ctx);   // pass 0's heap grows: retained rerun memory goes first
         size_t fr = 0, tot = 0;
         CK(cudaMemGetInfo(&fr, &tot));
         const size_t have = ctx->spill[round_idx].n;
         const size_t avail = fr + have > (1ull << 30) ? fr + have - (1ull << 30) : 0;
         // 25 % headroom so that slowly growing requests do not reallocate every run
-        size_t bytes = std::min<size_t>((size_t)R.spill_want * 5, avail) & ~(size_t)15;
+        size_t bytes = std::min<size_t>((size_t)R.spill_want * (R.spill_exact ? 4 : 5), avail) & ~(size_t)15;
         while (bytes >= 16 && ctx->spill[round_idx].ensure(bytes) != cudaSuccess) {
             cudaGetLastError();
             bytes = (bytes / 2) & ~(size_t)15;
@@ -1015,7 +1037,9 @@ static avfs_status settle_batch(avfs_ctx* ctx) {
         // least 64 MiB; without one, 4x capacity
         if (prev.spill_want > 0) {
             Rn.capacity = prev.capacity;
-            Rn.spill_want = std::max<int64_t>(4 * std::max<int64_t>(prev.spill_req, prev.spill_words), (64ll << 20) / 4);
+            int64_t floor_words = (64ll << 20) / 4;
+            if (const char* e = getenv("AVFS_RERUN_HEAP_MIN_BYTES")) floor_words = std::max<int64_t>(16, atoll(e) / 4);
+            Rn.spill_want = std::max<int64_t>(4 * std::max<int64_t>(prev.spill_req, prev.spill_words), floor_words);
         } else {
             Rn.capacity = std::min(prev.capacity * 4, 1024);
         }
@@ -1023,8 +1047,10 @@ static avfs_status settle_batch(avfs_ctx* ctx) {
         Rn.region_bytes = REG_TIMES + 4 * (int64_t)Rn.W;
         ctx->stats.overflow_slot_warps += n_ovf;
         ctx->stats.rerun_rounds++;
+        if (ctx->opt.profile && r == 0) CK(cudaEventRecord(ctx->ev2, ctx->stream));
         st = run_round(ctx, Rn, r + 1, ctx->d_list[cur].as<int32_t>(), ctx->d_prev[cur].as<int32_t>(), false);
         if (st != AVFS_OK) return st;
+        if (ctx->opt.profile) CK(cudaEventRecord(ctx->ev3, ctx->stream));
         ctx->rounds.push_back(std::move(Rn));
         ctx->pend_r = r + 1;
         ctx->pend_cur = cur ^ 1;
@@ -1039,6 +1065,10 @@ static avfs_status settle_batch(avfs_ctx* ctx) {
         float ms = 0;
         CK(cudaEventElapsedTime(&ms, ctx->ev0, ctx->ev1));
         ctx->pend_sweep_ms += ms;
+        if (ctx->pend_r > 0) {                          // this batch reran: time of its rerun rounds
+            CK(cudaEventElapsedTime(&ms, ctx->ev2, ctx->ev3));
+            ctx->stats.rerun_ms += ms;
+        }
     }
     return AVFS_OK;
 }
@@ -1140,11 +1170,9 @@ avfs_status avfs_simulate(avfs_ctx* ctx, void* cuda_stream) {
     ctx->stats.launches += 2;
 
     ctx->rounds.clear();
-    // rerun rounds' arenas and heaps of the previous simulate are stale: give
-    // their memory back so that pass 0 can size its heap from the hint
-    for (size_t r = 1; r < ctx->arena.size(); ++r) ctx->arena[r].release();
-    for (size_t r = 1; r < ctx->recs.size(); ++r) ctx->recs[r].release();
-    for (size_t r = 1; r < ctx->spill.size(); ++r) ctx->spill[r].release();
+    // rerun rounds' arenas and heaps of the previous simulate are kept for
+    // the next one (repeated runs rerun the same groups without reallocating
+    // inside the step); pass 0 takes their memory back if it needs it
     // slot batching: when the arena for every slot group would not
     // fit, the groups run in batches on the same arena and heap; activity,
     // latest arrival and energy accumulate over all batches, waveform readback
@@ -1209,6 +1237,7 @@ avfs_status avfs_simulate(avfs_ctx* ctx, void* cuda_stream) {
                       : ctx->opt.spill_bytes < 0 ? 0
                       : std::max<int64_t>({arena_words / 4, (256ll << 20) / 4,
                                            ctx->spill_per_group * R0.n_sw + ctx->spill_per_group * R0.n_sw / 4});
+        R0.spill_exact = ctx->opt.spill_bytes > 0;
     }
     st = run_round(ctx, R0, 0, nullptr, nullptr, ctx->opt.profile != 0);
     if (st != AVFS_OK) return st;

@@ -181,3 +181,32 @@ def test_config5_all_shards(quantum):
     assert r["tainted_differ"] <= 0.01 * max(r["tainted"], 1)
     assert r["events"] > 0
     ctx.close()
+
+
+@pytest.mark.slow
+def test_config5_overflow_reruns_at_scale():
+    """H7 at full size: config 5's first shard (2M gates, 204 slot groups)
+    with the pass-0 spill heap capped so that part of the groups exhaust it
+    and rerun.  Activity of every signal, latest arrival and the PO final
+    values of 2048 slots equal the uncapped run bit for bit (Q mode)."""
+    from paper_conf_date_schneiderw20_b200 import Context, load_workload, shard_range
+    w = make_config(5)
+    nl = w.netlist
+    first, cnt = shard_range(w.n_slots, 0, 8)
+    res = []
+    for spill in (0, 20 << 30):
+        ctx = Context(0)
+        load_workload(ctx, nl, w.library, w.stimuli, w.vdd)
+        ctx.set_options(capacity=w.capacity, quantum_ps=2.0 ** -8, keep_all=False, spill_bytes=spill, profile=True)
+        ctx.set_slot_range(first, cnt)
+        ctx.simulate()
+        st = ctx.stats()
+        fv = ctx.final_values(nl.po_sig, first, 2048)
+        res.append((ctx.activity(), ctx.latest_arrival(), fv, st))
+        ctx.close()
+    print(f"[overflow] uncapped spill {res[0][3]['spill_bytes']} B; capped: {res[1][3]['overflow_slot_warps']} "
+          f"of {res[1][3]['slot_warps']} groups rerun in {res[1][3]['rerun_rounds']} rounds, "
+          f"rerun {res[1][3]['rerun_ms']:.1f} ms vs sweep {res[1][3]['sweep_ms']:.1f} ms")
+    assert res[1][3]["overflow_slot_warps"] > 0
+    for a, b in zip(res[0][:3], res[1][:3]):
+        assert np.array_equal(a, b)

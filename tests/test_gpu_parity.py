@@ -343,3 +343,24 @@ def test_slot_batching(quantum):
     assert np.array_equal(b.activity().astype(np.int64)[ok], ra[ok])
     a.close()
     b.close()
+
+
+def test_repeated_heap_exhaustion_counts_activity_once(monkeypatch):
+    """a gate counted in round r-1 that is poisoned again in round
+    r must not be counted twice.  A 4 KiB pass-0 heap and no floor on the
+    rerun heaps force several heap-exhausting rerun rounds; activity, latest
+    arrival and waveforms equal the run without any heap (capacity reruns)
+    and the run with an ample heap."""
+    monkeypatch.setenv("AVFS_RERUN_HEAP_MIN_BYTES", "16")
+    w = make_config(3, n_pairs=64, n_vdd=3, scale=0.08)
+    sig = np.arange(w.netlist.n_signals, dtype=np.int32)
+    outs, stats = [], []
+    for spill in (4096, -1, 0):
+        ctx = gpu_run(w, quantum=Q, capacity=1, spill_bytes=spill, max_rerun_rounds=6)
+        outs.append((ctx.activity(), ctx.latest_arrival(), *ctx.waveforms(sig, 0, w.n_slots, cap=40)))
+        stats.append(ctx.stats())
+        ctx.close()
+    assert stats[0]["rerun_rounds"] >= 2, stats[0]
+    for other in outs[1:]:
+        for a, b in zip(outs[0], other):
+            assert np.array_equal(a, b)
