@@ -147,28 +147,74 @@ def host_cores() -> int:
         return os.cpu_count() or 1
 
 
-def cpu_baseline(w, target_s=15.0):
-    """The oracle as it stands, on this host's cores, on a bounded slot sample."""
-    import oracle
-    P, V = w.stimuli.n_pairs, len(w.vdd)
-    rng = np.random.default_rng(12345)
-    threads = host_cores()
+def collective_info(world, args):
+    """What the multi-GPU step exchanges: nothing during the
+    simulation; one reduce of the activity counters (SUM) and of the latest
+    arrival (MAX) to rank 0 per step."""
+    if world <= 1:
+        return None
+    import torch
+    import torch.distributed as dist
+    info = {"backend": dist.get_backend(), "world_size": dist.get_world_size(),
+            "ops": ["reduce(activity u64 [signals x Vdd], SUM)", "reduce(latest f32 [Vdd], MAX)"],
+            "scaling": args.scaling}
+    try:
+        info["nccl_version"] = ".".join(str(x) for x in torch.cuda.nccl.version())
+    except Exception:
+        pass
+    return info
 
-    def run(n):
-        s = np.sort(rng.choice(P * V, size=n, replace=False))
+
+def cpu_model() -> str:
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.lower().startswith("model name"):
+                return line.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return "unknown"
+
+
+def parity_sample(w):
+    """BASELINE.md / SURVEY §8(d) deterministic oracle sample (also the GPU
+    parity set): cfgs 1-2 every slot; cfg 3 pairs j mod 64 = 0; cfg 4 pairs
+    j mod 256 = 0; cfg 5 pair 0 at all 51 Vdd points.  Returns (pairs, vdd
+    indices, description)."""
+    P, V = w.stimuli.n_pairs, len(w.vdd)
+    step = {1: 1, 2: 1, 3: 64, 4: 256}.get(w.cfg)
+    if step is None:                                    # cfg 5
+        j = np.zeros(V, np.int64)
+        k = np.arange(V, dtype=np.int32)
+        return j, k, f"pair 0 x all {V} Vdd points"
+    jj = np.arange(0, P, step, dtype=np.int64)
+    k, j = np.meshgrid(np.arange(V, dtype=np.int32), jj, indexing="ij")
+    return j.ravel(), k.ravel(), (f"pairs j mod {step} = 0 ({len(jj)} pairs) x {V} Vdd" if step > 1
+                                  else f"every slot ({P} pairs x {V} Vdd)")
+
+
+def cpu_baseline(w):
+    """The oracle as it stands, on this host's cores and on one core, on the
+    deterministic sample of BASELINE.md's CPU-baseline plan."""
+    import oracle
+    threads = host_cores()
+    j, k, desc = parity_sample(w)
+
+    def run(nth, jj, kk):
         t0 = time.perf_counter()
-        oracle.simulate(w.netlist, w.library, w.stimuli, w.vdd, s % P, s // P, quantum=0.0, cap=0,
-                        out_sig=w.netlist.po_sig, threads=threads)
+        oracle.simulate(w.netlist, w.library, w.stimuli, w.vdd, jj, kk, quantum=0.0, cap=0,
+                        out_sig=w.netlist.po_sig, threads=nth)
         return time.perf_counter() - t0
 
-    n0 = max(threads, 4)
-    t0 = run(n0)
-    n = int(min(P * V, max(n0, n0 * target_s / max(t0, 1e-3))))
-    t = run(n) if n > n0 else t0
-    n = n if n > n0 else n0
-    return {"value": w.netlist.n_gates * n / t, "unit": UNIT, "cores": threads, "kind": "oracle",
-            "sample": f"{n} random slots of {P * V} (all {w.netlist.n_gates} gates each), "
-                      f"{t:.1f} s wall, OpenMP over slots"}
+    t_all = run(threads, j, k)
+    # 1 thread: the whole sample if it takes <= ~20 s at the all-core rate x cores, else a prefix
+    n1 = int(min(len(j), max(1, 20.0 / max(t_all * threads / len(j), 1e-6))))
+    t_one = run(1, j[:n1], k[:n1])
+    G = w.netlist.n_gates
+    return {"value": G * len(j) / t_all, "unit": UNIT, "cores": threads, "kind": "oracle",
+            "cpu_model": cpu_model(),
+            "sample": f"{desc}: {len(j)} slots (all {G} gates each), {t_all:.2f} s wall, OpenMP over slots",
+            "one_thread": {"value": G * n1 / t_one, "unit": UNIT, "cores": 1,
+                           "sample": f"first {n1} slots of that sample, {t_one:.2f} s wall"}}
 
 
 def run_reference(args, w, world, rank):
@@ -178,20 +224,22 @@ def run_reference(args, w, world, rank):
     import oracle
     P, V = w.stimuli.n_pairs, len(w.vdd)
     threads = host_cores()
-    rng = np.random.default_rng(777)
-    # size each step so the whole --steps K --warmup W run stays within a few minutes
-    probe = np.sort(rng.choice(P * V, size=max(threads, 4), replace=False))
+    # each step: the deterministic parity sample, or an evenly
+    # spaced subset of it that keeps the whole --steps K --warmup W run within
+    # a few minutes
+    js, ks, desc = parity_sample(w)
+    probe = np.linspace(0, len(js) - 1, min(len(js), max(threads, 4))).astype(int)
     t0 = time.perf_counter()
-    oracle.simulate(w.netlist, w.library, w.stimuli, w.vdd, probe % P, probe // P, cap=0,
+    oracle.simulate(w.netlist, w.library, w.stimuli, w.vdd, js[probe], ks[probe], cap=0,
                     out_sig=w.netlist.po_sig, threads=threads)
     per_slot = (time.perf_counter() - t0) / len(probe)
     budget = 150.0 / max(1, args.steps + args.warmup)
-    n = int(max(len(probe), min(P * V, budget / max(per_slot, 1e-6))))
+    n = int(max(len(probe), min(len(js), budget / max(per_slot, 1e-6))))
+    sel = np.linspace(0, len(js) - 1, n).astype(int)
     times = []
     for it in range(args.warmup + args.steps):
-        s = np.sort(rng.choice(P * V, size=n, replace=False))
         t0 = time.perf_counter()
-        oracle.simulate(w.netlist, w.library, w.stimuli, w.vdd, s % P, s // P, cap=0,
+        oracle.simulate(w.netlist, w.library, w.stimuli, w.vdd, js[sel], ks[sel], cap=0,
                         out_sig=w.netlist.po_sig, threads=threads)
         if it >= args.warmup:
             times.append(time.perf_counter() - t0)
@@ -202,8 +250,8 @@ def run_reference(args, w, world, rank):
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * t / args.steps,
         "higher_is_better": True, "scaling": args.scaling, "vs_baseline": None, "dtype": "f64",
         "data": "synthetic", "config": config_dict(w, args),
-        "cpu_baseline": {"value": value, "unit": UNIT, "cores": threads, "kind": "oracle",
-                         "sample": f"{n} random slots per step of {P * V}"},
+        "cpu_baseline": {"value": value, "unit": UNIT, "cores": threads, "kind": "oracle", "cpu_model": cpu_model(),
+                         "sample": f"{n} slots per step of the parity sample ({desc}) of {P * V}"},
         "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }
     print(json.dumps(line), flush=True)
@@ -384,6 +432,7 @@ def main():
             "cpu_baseline": cpu,
             "e2e": e2e,
             "gpu_launches": int(stats["launches"] * args.steps),
+            "collective": collective_info(world, args),
             "clocks": ck,
             "stats": {k: stats[k] for k in ("evals", "slot_warps", "overflow_slot_warps", "rerun_rounds", "spill_bytes", "batches",
                                             "grid", "warps_per_cta", "n_scratch_buffers", "n_pinned",
