@@ -442,26 +442,41 @@ struct Filt {
 
 // Merge of at most two sorted lists (pins p0 < p1; list 1 may be empty), the
 // next element of each list already loaded (one element of lookahead).
+#ifndef AVFS_LOOKAHEAD
+#define AVFS_LOOKAHEAD 3
+#endif
 __device__ __forceinline__ uint32_t merge_two(const float* a0, int n0, const float* a1, int n1, uint32_t bits,
                                               uint32_t tm0, uint32_t tm1, uint32_t proj, uint32_t tt, float4 dl,
                                               float* out, uint32_t steps) {
-    float h0 = n0 > 0 ? ld_f32(a0) : AVFS_INF, g0 = n0 > 1 ? ld_f32(a0 + 1) : AVFS_INF;
-    float h1 = n1 > 0 ? ld_f32(a1) : AVFS_INF, g1 = n1 > 1 ? ld_f32(a1 + 1) : AVFS_INF;
-    a0 += 2;
-    a1 += 2;
-    n0 -= 2;
-    n1 -= 2;
+    // a window of the next AVFS_LOOKAHEAD elements of each list lives in
+    // registers: their loads are issued together up front, and a refill load
+    // is consumed AVFS_LOOKAHEAD advances of its list later (lists of at most
+    // that many events need no load inside the loop)
+    constexpr int D = AVFS_LOOKAHEAD;
+    float w0[D], w1[D];
+#pragma unroll
+    for (int i = 0; i < D; ++i) {
+        w0[i] = n0 > i ? ld_f32(a0 + i) : AVFS_INF;
+        w1[i] = n1 > i ? ld_f32(a1 + i) : AVFS_INF;
+    }
+    a0 += D;
+    a1 += D;
+    n0 -= D;
+    n1 -= D;
     Filt F{proj, 0u, -AVFS_INF};
 #pragma unroll 1
     for (uint32_t it = 0; it < steps; ++it) {
-        const bool p = h1 < h0;                       // ties: the lower pin first (reading C5)
-        const float t = fminf(h0, h1);
+        const bool p = w1[0] < w0[0];                 // ties: the lower pin first (reading C5)
+        const float t = fminf(w0[0], w1[0]);
         const float* a = p ? a1 : a0;
         const float nx = (p ? n1 : n0) > 0 ? ld_f32(a) : AVFS_INF;
-        h1 = p ? g1 : h1;
-        g1 = p ? nx : g1;
-        h0 = p ? h0 : g0;
-        g0 = p ? g0 : nx;
+#pragma unroll
+        for (int i = 0; i + 1 < D; ++i) {
+            w1[i] = p ? w1[i + 1] : w1[i];
+            w0[i] = p ? w0[i] : w0[i + 1];
+        }
+        w1[D - 1] = p ? nx : w1[D - 1];
+        w0[D - 1] = p ? w0[D - 1] : nx;
         a1 += p ? 1 : 0;
         n1 -= p ? 1 : 0;
         a0 += p ? 0 : 1;
