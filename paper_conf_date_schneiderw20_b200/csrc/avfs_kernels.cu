@@ -419,6 +419,7 @@ __device__ __forceinline__ int phase_a(const SweepParams& p, const Grp& G, int g
         sts_f32x4(qe + 4 * Q_DLY, dl0);
         sts_f32x4(qe + 4 * Q_DLY + 16, dl1);
     }
+    __syncwarp();                             // queue entries -> the item phase's lanes
     return __popc(bal);
 }
 

@@ -17,6 +17,17 @@ for r in rows:
         f = lambda x: float(x) if x not in ("", "-") else 0.0
         inst[cur] += f(r[ie]); samp[cur] += f(r[ws])
 tot = sum(inst.values()); ts = sum(samp.values()); gw = a.evals / 32
-print(f"total warp instr {tot:.3e} = {tot/gw:.1f} per gate-warp; stall samples {ts:.0f}")
+# the cuda-line rows of the source page attribute inlined code to several
+# lines; scale to the kernel's executed warp instructions (sass view total)
+raw = subprocess.run(["ncu", "-i", a.rep, "--page", "source", "--csv", "--print-source", "sass"],
+                     capture_output=True, text=True).stdout
+srows = list(csv.reader(io.StringIO(raw)))
+sh = next(r for r in srows if r and "Source" in r and "Instructions Executed" in r)
+k = sh.index("Instructions Executed")
+sass_tot = sum(float(r[k]) for r in srows if len(r) > k and r is not sh and r[k].replace(".", "").isdigit())
+f = sass_tot / tot if tot else 1.0
+print(f"executed warp instructions {sass_tot:.4e} = {sass_tot/gw:.1f} per gate-warp (per-line counts below scaled "
+      f"by {f:.3f} from the cuda-line attribution sum {tot:.4e}); stall samples {ts:.0f}")
+inst = collections.Counter({key: v * f for key, v in inst.items()}); tot = sass_tot
 for k, v in sorted(inst.items(), key=lambda x: -x[1])[:a.top]:
     print(f"{k[0]}:{k[1]:5d} {v/gw:7.1f}/gw {100*v/tot:5.1f}%  samp {100*samp[k]/max(ts,1):5.1f}%  {src[k]}")

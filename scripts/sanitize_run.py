@@ -10,7 +10,8 @@ for cfg, kw in ((1, dict(n_pairs=64)), (2, dict(n_pairs=64, n_vdd=2)), (3, dict(
     for cap, spill in ((1, 0), (1, -1), (1, 4096), (8, 0)):
         ctx = Context(0)
         load_workload(ctx, w.netlist, w.library, w.stimuli, w.vdd)
-        ctx.set_options(capacity=cap, keep_all=(cfg == 1), max_rerun_rounds=4, spill_bytes=spill)
+        ctx.set_options(capacity=cap, keep_all=(cfg == 1), max_rerun_rounds=4, spill_bytes=spill,
+                        delay_in_sweep=(cap == 8))
         ctx.simulate()
         a = ctx.activity()
         ctx.waveforms(w.netlist.po_sig, 0, w.n_slots, cap=8)
@@ -22,7 +23,8 @@ for cfg, kw in ((1, dict(n_pairs=64)), (2, dict(n_pairs=64, n_vdd=2)), (3, dict(
 
 # work-distribution variants: G slot groups per CTA (named barriers), S CTAs per group
 w = make_config(3, n_pairs=96, n_vdd=2, scale=0.05)
-for env in ({"AVFS_GROUPS_PER_CTA": "4"}, {"AVFS_SPLIT": "2"}):
+for env in ({"AVFS_GROUPS_PER_CTA": "4"}, {"AVFS_GROUPS_PER_CTA": "1", "AVFS_SPLIT": "2"},
+            {"AVFS_GROUPS_PER_CTA": "1", "AVFS_SPLIT": "8"}):
     os.environ.pop("AVFS_GROUPS_PER_CTA", None)
     os.environ.pop("AVFS_SPLIT", None)
     os.environ.update(env)
@@ -34,3 +36,11 @@ for env in ({"AVFS_GROUPS_PER_CTA": "4"}, {"AVFS_SPLIT": "2"}):
     ctx.close()
 os.environ.pop("AVFS_GROUPS_PER_CTA", None)
 os.environ.pop("AVFS_SPLIT", None)
+# 2-D (v, c) delay model, voltage islands
+w = make_config(3, n_pairs=64, n_vdd=2, scale=0.03, deg_c=3)
+ctx = Context(0)
+load_workload(ctx, w.netlist, w.library, w.stimuli, w.vdd)
+ctx.set_options(capacity=2, quantum_ps=2.0 ** -8)
+ctx.simulate()
+print("2d", int(ctx.activity().sum()), flush=True)
+ctx.close()
