@@ -954,6 +954,7 @@ static avfs_status run_round(avfs_ctx* ctx, Round& R, int round_idx, const int32
     p.arena = ctx->arena[round_idx].as<uint8_t>();
     p.region_bytes = R.region_bytes;
     p.recs = ctx->recs[round_idx].as<uint4>();
+    p.n_buf = n_buf;
     p.W = R.W;
     p.grp_per_cta = R.grp;
     p.split = R.split;
@@ -1354,7 +1355,7 @@ static avfs_status gather(avfs_ctx* ctx, int32_t n_sig, const int32_t* sig, int6
     g.sw_index = ctx->d_swindex.as<int32_t>();
     for (size_t r = 0; r < ctx->rounds.size(); ++r)
         g.rounds[r] = GatherRound{ctx->arena[r].as<uint8_t>(), ctx->recs[r].as<uint4>(), ctx->rounds[r].region_bytes,
-                                  ctx->rounds[r].n_sw};
+                                  ctx->rounds[r].n_sw, (int64_t)ctx->n_pinned + ctx->n_scratch};
     g.cap = times ? cap : 0;
     g.init = ctx->g_init.as<uint8_t>();
     g.count = ctx->g_count.as<int32_t>();
@@ -1447,7 +1448,7 @@ avfs_status avfs_capture(avfs_ctx* ctx, const float* t_clk, int32_t n_bins, floa
     p.sw_index = ctx->d_swindex.as<int32_t>();
     for (size_t r = 0; r < ctx->rounds.size(); ++r)
         p.rounds[r] = GatherRound{ctx->arena[r].as<uint8_t>(), ctx->recs[r].as<uint4>(), ctx->rounds[r].region_bytes,
-                                  ctx->rounds[r].n_sw};
+                                  ctx->rounds[r].n_sw, (int64_t)ctx->n_pinned + ctx->n_scratch};
     p.slot_fail = ctx->c_slot.as<uint32_t>();
     p.slot_last = ctx->c_slot.as<uint32_t>() + (size_t)n_sw * 32;
     p.fail_po = ctx->c_out.as<uint32_t>();

@@ -27,17 +27,18 @@ constexpr uint32_t LOC_ID = ~LOC_KIND;
 // Waveform of one (signal, 32-slot group) (reading C1), in two parts:
 //
 //  record  uint4 {init, E, A, meta} in the round's record array
-//          [buffer][group]: init = bit l is slot l's value before t = 0,
+//          [group][buffer]: init = bit l is slot l's value before t = 0,
 //          E = slots with >= 1 transition, A = slots that own an entry
 //          (E is a subset of A), meta = total stored transitions (REC_NTOT)
 //          plus REC_POISON / REC_SPILL.  PIs have no record: it is the
 //          stimulus words (init = p1, E = A = p1 xor p2, one event at t = 0).
-//  region  in the round's arena [buffer][group]: 32 entry words, compact in
-//          the order of A's set bits (entry = n | off << ENT_OFF_SHIFT: the
-//          slot's count and the word offset of its first time), then at byte
-//          REG_TIMES the binary32 times (W words); when the record says
-//          REC_SPILL the times live in the spill heap at the 64-bit address
-//          stored at byte REG_SPILLPTR.
+//  region  in the round's arena [buffer][group]: popc(A) entry words, compact
+//          in the order of A's set bits (entry = n | off << ENT_OFF_SHIFT: the
+//          slot's count and the word offset of its first time), then the
+//          binary32 times right after them (byte 4 popc(A)), so a gate's
+//          output is one contiguous extent; when the record says REC_SPILL
+//          the times live in the spill heap at the 64-bit address stored at
+//          byte REG_SPILLPTR.  Regions hold up to W times.
 constexpr uint32_t REC_NTOT = 0x0FFFFFFFu;
 constexpr uint32_t REC_POISON = 1u << 29;    // events not stored here or upstream (overflow)
 constexpr uint32_t REC_SPILL = 1u << 30;
@@ -108,7 +109,8 @@ struct SweepParams {
     // arena of the round: [buffer][pin_n_sw][region]; buffers = kept signals, then scratch
     uint8_t* arena;
     int64_t region_bytes;
-    uint4* recs;                            // [buffer][pin_n_sw] records
+    uint4* recs;                            // [buffer][pin_n_sw] records (or [pin_n_sw][n_buf])
+    int64_t n_buf;                          // arena buffers (kept + scratch)
     int32_t W;                              // in-place time capacity per region (words)
     int32_t grp_per_cta;                    // slot groups a sweep CTA walks at once (power of 2)
     int32_t split;                          // sweep CTAs sharing one slot group (grp_per_cta == 1)
@@ -149,9 +151,10 @@ cudaError_t launch_compact_overflow(const int32_t* ovf, int64_t n_sw, const int3
 
 struct GatherRound {       // one simulated round for readback
     const uint8_t* pinned;      // arena (kept buffers first)
-    const uint4* recs;          // records [buffer][n_sw]
+    const uint4* recs;          // records [buffer][n_sw] (or [n_sw][n_buf])
     int64_t region_bytes;
     int64_t n_sw;
+    int64_t n_buf;
 };
 struct GatherParams {
     const uint32_t* sig_loc;    // [n_sig] location codes (LOC_PI | pi, or LOC_PINNED | arena buffer)

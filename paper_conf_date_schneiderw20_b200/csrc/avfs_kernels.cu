@@ -35,6 +35,28 @@
 
 namespace avfs {
 
+// Byte offset of a region's in-place times (record mask A = the slots that
+// own an entry): right after the popc(A) entry words, so a gate's output is
+// one contiguous extent (AVFS_TIMES_PACKED), or at the fixed REG_TIMES.
+#ifndef AVFS_REC_GROUP_MAJOR
+#define AVFS_REC_GROUP_MAJOR 1     // records [group][buffer] (1) or [buffer][group] (0)
+#endif
+#ifndef AVFS_TIMES_PACKED
+#define AVFS_TIMES_PACKED 1
+#endif
+__host__ __device__ __forceinline__ uint32_t times_off(uint32_t A) {
+#if AVFS_TIMES_PACKED
+#ifdef __CUDA_ARCH__
+    return 4u * (uint32_t)__popc(A);
+#else
+    return 4u * (uint32_t)__builtin_popcount(A);
+#endif
+#else
+    (void)A;
+    return REG_TIMES;
+#endif
+}
+
 // Waveforms are produced and consumed inside one launch: read them at L2
 // (.cg), never through a possibly stale L1 line.
 __device__ __forceinline__ uint32_t ld_u32(const void* p) {
@@ -213,9 +235,17 @@ __device__ __forceinline__ void group_setup(const SweepParams& p, int64_t i, int
     G.pw = (int)(sw % p.n_pw);
     G.gi = p.i_base + i;
     G.row = p.arena + G.gi * p.region_bytes;
+#if AVFS_REC_GROUP_MAJOR
+    G.rec = p.recs + G.gi * (int64_t)p.n_buf;
+#else
     G.rec = p.recs + G.gi;
+#endif
     G.stride = (uint32_t)(p.pin_n_sw * p.region_bytes);
+#if AVFS_REC_GROUP_MAJOR
+    G.rstride = 1u;
+#else
     G.rstride = (uint32_t)p.pin_n_sw;
+#endif
     const int64_t j = (int64_t)G.pw * 32 + lane;
     const int64_t pub = (int64_t)G.kv * p.n_pairs + j;
     G.vmask = __ballot_sync(FULL, j < p.n_pairs && pub >= p.slot_first && pub < p.slot_end);
@@ -350,7 +380,7 @@ __device__ __forceinline__ int phase_a(const SweepParams& p, const Grp& G, int g
         if (U >= OFF_LIMIT) {
             own = true;
         } else if (U <= (uint32_t)p.W) {
-            tb = reinterpret_cast<unsigned long long>(oreg + REG_TIMES);
+            tb = reinterpret_cast<unsigned long long>(oreg + times_off(A));
         } else {
             const unsigned long long need = (U + 3u) & ~3u;
             const unsigned long long wb = atomicAdd(p.spill_top, need);
@@ -412,7 +442,7 @@ __device__ __forceinline__ int phase_a(const SweepParams& p, const Grp& G, int g
             if ((uint32_t)q < K && (loc[q] & LOC_KIND) != LOC_PI) {
                 const uint8_t* r = G.row + (size_t)(loc[q] & LOC_ID) * G.stride;
                 itb = (M[q] & REC_SPILL) ? __ldcg(reinterpret_cast<const unsigned long long*>(r + REG_SPILLPTR))
-                                         : reinterpret_cast<unsigned long long>(r + REG_TIMES);
+                                         : reinterpret_cast<unsigned long long>(r + times_off(AQ[q]));
             }
             sts_u64(qe + 4 * Q_ITB + 8 * q, itb);
         }
@@ -970,7 +1000,11 @@ cudaError_t launch_compact_overflow(const int32_t* ovf, int64_t n_sw, const int3
 // initial value, count and its times; false if the waveform is poisoned.
 __device__ __forceinline__ bool read_slot(const GatherRound& R, uint32_t buf, int64_t idx, int l, uint32_t& init,
                                           int& n, const float*& ev) {
+#if AVFS_REC_GROUP_MAJOR
+    const uint4 rec = R.recs[(size_t)idx * R.n_buf + buf];
+#else
     const uint4 rec = R.recs[(size_t)buf * R.n_sw + idx];
+#endif
     if (rec.w & REC_POISON) return false;
     const uint8_t* reg = R.pinned + ((int64_t)buf * R.n_sw + idx) * R.region_bytes;
     init = (rec.x >> l) & 1u;
@@ -980,7 +1014,7 @@ __device__ __forceinline__ bool read_slot(const GatherRound& R, uint32_t buf, in
         const uint32_t w = reinterpret_cast<const uint32_t*>(reg)[__popc(rec.z & ((1u << l) - 1u))];
         n = (int)(w & ENT_N);
         const float* tb = (rec.w & REC_SPILL) ? *reinterpret_cast<const float* const*>(reg + REG_SPILLPTR)
-                                              : reinterpret_cast<const float*>(reg + REG_TIMES);
+                                              : reinterpret_cast<const float*>(reg + times_off(rec.z));
         ev = tb + (w >> ENT_OFF_SHIFT);
     }
     return true;
