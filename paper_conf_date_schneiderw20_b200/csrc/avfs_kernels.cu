@@ -835,6 +835,15 @@ static cudaError_t occ_one(int warps_per_cta, int smem, int* b) {
 }
 
 cudaError_t sweep_occupancy(int warps_per_cta, int smem, int* blocks_per_sm) {
+    // attributes and occupancy are per (device, shape): computed once, not
+    // inside every simulate (host time between the stream's events)
+    static int c_dev = -1, c_wpc = -1, c_smem = -1, c_bps = 0;
+    int dev = 0;
+    cudaGetDevice(&dev);
+    if (dev == c_dev && warps_per_cta == c_wpc && smem == c_smem) {
+        *blocks_per_sm = c_bps;
+        return cudaSuccess;
+    }
     int b[4] = {0, 0, 0, 0};
     cudaError_t e = occ_one<false, false>(warps_per_cta, smem, b + 0);
     if (e == cudaSuccess) e = occ_one<true, false>(warps_per_cta, smem, b + 1);
@@ -843,6 +852,12 @@ cudaError_t sweep_occupancy(int warps_per_cta, int smem, int* blocks_per_sm) {
     int m = b[0];
     for (int k = 1; k < 4; ++k) m = b[k] < m ? b[k] : m;    // split groups need every CTA resident
     *blocks_per_sm = m;
+    if (e == cudaSuccess) {
+        c_dev = dev;
+        c_wpc = warps_per_cta;
+        c_smem = smem;
+        c_bps = m;
+    }
     return e;
 }
 

@@ -9,9 +9,9 @@ ap = argparse.ArgumentParser(); ap.add_argument("--config", type=int, default=4)
 w = make_config(a.config)
 ctx = Context(0); load_workload(ctx, w.netlist, w.library, w.stimuli, w.vdd)
 ctx.set_options(capacity=w.capacity, profile=True)
-s = torch.cuda.Stream(); ctx.simulate(s); debug_phase_cycles(reset=True); ctx.simulate(s)
+s = torch.cuda.Stream(); ctx.simulate(s); ctx.sync(); debug_phase_cycles(reset=True); ctx.simulate(s); ctx.sync()
 c = debug_phase_cycles().astype(np.float64)
-names = {1: "phaseA", 5: "phaseB", 6: "barrier"}
+names = {1: "phaseA", 2: "item setup", 3: "merge", 4: "item finish", 5: "phaseB total", 6: "barrier"}
 tot = c[1] + c[5] + c[6]
 st = ctx.stats()
 print(f"cfg{a.config} sweep {st['sweep_ms']:.1f} ms; warp-cycles total {tot:.3e}")
