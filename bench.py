@@ -69,7 +69,7 @@ class ClockSampler:
         try:
             self.proc = subprocess.Popen(
                 ["nvidia-smi", "-i", str(self.dev), f"--query-gpu={self.Q}", "--format=csv,noheader,nounits",
-                 "-lms", "100"], stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+                 "-lms", os.environ.get("AVFS_SMI_MS", "250")], stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
             self.t = threading.Thread(target=self._read, daemon=True)
             self.t.start()
         except Exception:
@@ -351,6 +351,9 @@ def main():
     torch.cuda.synchronize()
     clocks = ClockSampler(local)
     clocks.start()
+    import gc
+    gc.collect()
+    gc.disable()                    # no collector pauses between the stream's events
     ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
     sweep_ms, rerun_ms = [], []
     for i in range(args.steps):
@@ -359,10 +362,11 @@ def main():
         ev[i][0].record(stream)
         step()
         ev[i][1].record(stream)
-        st_i = ctx.stats()
-        sweep_ms.append(st_i["sweep_ms"])
-        rerun_ms.append(st_i["rerun_ms"])
+        sw_i, rr_i = ctx.timing()
+        sweep_ms.append(sw_i)
+        rerun_ms.append(rr_i)
     torch.cuda.synchronize()
+    gc.enable()
     ck = clocks.stop()
     step_ms = [a.elapsed_time(b) for a, b in ev]
     t_total = float(np.sum(step_ms))
@@ -424,6 +428,8 @@ def main():
             "warmup": args.warmup, "ms_per_step": t_total / args.steps, "higher_is_better": True,
             "scaling": args.scaling, "vs_baseline": None, "dtype": "f32",
             "data": "synthetic", "config": config_dict(w, args),
+            "step_ms_each": [round(x, 3) for x in step_ms],
+            "sweep_ms_each": [round(x, 3) for x in sweep_ms],
             "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                          "frac": achieved / peak, "traffic": traffic, "peak_source": peak_src,
                          "kernel": "avfs::sweep_kernel", "kernel_ms": sweep_avg,

@@ -294,6 +294,11 @@ typedef struct {
 } avfs_stats;
 avfs_status avfs_get_stats(avfs_ctx *ctx, avfs_stats *st);
 
+/* The CUDA-event times of the last simulate (profile=1): pass-0 sweep and
+ * overflow reruns, ms.  Cheap (no readback), unlike avfs_get_stats, which
+ * also derives the algorithmic bytes from the activity counters.         */
+avfs_status avfs_get_timing(avfs_ctx *ctx, double *sweep_ms, double *rerun_ms);
+
 /* Diagnostics: per-phase warp clock sums of the sweep kernel (16 counters:
  * 1 bit-parallel phase, 5 item phase, 6 level barriers), accumulated over
  * all launches since the last reset.  Only builds compiled with

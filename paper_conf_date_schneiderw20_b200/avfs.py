@@ -25,7 +25,7 @@ EXPORTS = [
     "avfs_set_options", "avfs_default_options", "avfs_simulate", "avfs_sync",
     "avfs_get_activity", "avfs_get_latest_arrival", "avfs_get_final_values",
     "avfs_get_waveforms", "avfs_get_stats", "avfs_capture", "avfs_get_switching_energy",
-    "avfs_fit_delay_polynomial", "avfs_debug_phase_cycles",
+    "avfs_fit_delay_polynomial", "avfs_debug_phase_cycles", "avfs_get_timing",
 ]
 
 
@@ -106,6 +106,7 @@ def load_library(path: str = LIB_PATH):
             "avfs_get_switching_energy": ([P, P], C.c_int),
             "avfs_fit_delay_polynomial": ([I64, P, P, P, I32, I32, D, D, D, D, P, P], C.c_int),
             "avfs_debug_phase_cycles": ([P, I32], C.c_int32),
+            "avfs_get_timing": ([P, P, P], C.c_int),
         }
         for name, (args, res) in sig.items():
             f = getattr(lib, name)
@@ -295,6 +296,12 @@ class Context:
         a = np.zeros((self.n_signals, self.n_vdd), np.uint64)
         self._ck(self.lib.avfs_get_activity(self.h, _p(a), 0))
         return a
+
+    def timing(self):
+        """(pass-0 sweep ms, rerun ms) of the last simulate (profile=True); no readback."""
+        a, b = C.c_double(), C.c_double()
+        self._ck(self.lib.avfs_get_timing(self.h, C.byref(a), C.byref(b)))
+        return a.value, b.value
 
     def latest_arrival(self, out=None) -> np.ndarray:
         """[n_vdd] float32 ps; `out` may be a contiguous CUDA float32 tensor (device copy)."""

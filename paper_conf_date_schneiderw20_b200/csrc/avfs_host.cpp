@@ -1197,9 +1197,13 @@ avfs_status avfs_simulate(avfs_ctx* ctx, void* cuda_stream) {
     bool learn = false;                                 // first batch only one wave: learn the spill per group
     if (ctx->opt.max_batch_slots > 0) {
         nb = std::max<int64_t>(1, ctx->opt.max_batch_slots / 32);
-    } else if (!ctx->arena.empty() && ctx->arena[0].n >= (size_t)(n_sw_all * per_group) &&
+    } else if (!ctx->arena.empty() && !ctx->recs.empty() &&
+               ctx->arena[0].n >= (size_t)(n_sw_all * ((int64_t)ctx->n_pinned + ctx->n_scratch) * region0) &&
+               ctx->recs[0].n >= (size_t)(n_sw_all * ((int64_t)ctx->n_pinned + ctx->n_scratch) * (int64_t)sizeof(uint4)) &&
                ctx->spill_per_group * n_sw_all * 5 / 4 <= (int64_t)(ctx->spill.empty() ? 0 : ctx->spill[0].n / 4)) {
-        nb = n_sw_all;                                  // fits the arena and heap of a previous simulate
+        // fits the arena, records and heap of a previous simulate: no device
+        // memory query (cudaMemGetInfo costs milliseconds at times)
+        nb = n_sw_all;
     } else {
         const int64_t fit = (int64_t)(0.8 * avail_bytes() / std::max(group_bytes(), 1.0));
         if (fit < n_sw_all) {
@@ -1480,6 +1484,16 @@ avfs_status avfs_get_switching_energy(avfs_ctx* ctx, double* out) {
                      ctx->stream));
     CK(cudaMemcpyAsync(out, ctx->d_energy.p, (size_t)V * sizeof(double), cudaMemcpyDeviceToHost, ctx->stream));
     CK(cudaStreamSynchronize(ctx->stream));
+    return AVFS_OK;
+}
+
+avfs_status avfs_get_timing(avfs_ctx* ctx, double* sweep_ms, double* rerun_ms) {
+    CHECK_CTX();
+    SETTLE();
+    if (!sweep_ms || !rerun_ms) return fail(ctx, AVFS_ERR_ARG, "null output");
+    if (!ctx->sim_done) return fail(ctx, AVFS_ERR_STATE, "simulate first");
+    *sweep_ms = ctx->stats.sweep_ms;
+    *rerun_ms = ctx->stats.rerun_ms;
     return AVFS_OK;
 }
 
