@@ -1154,6 +1154,8 @@ avfs_status avfs_simulate(avfs_ctx* ctx, void* cuda_stream) {
         dp.deg_c = ctx->deg_c;
         dp.vdd = ctx->d_vdd.as<double>();
         dp.n_vdd = V;
+        dp.kv_lo = (int32_t)(first / P);
+        dp.kv_hi = (int32_t)((end - 1) / P + 1);
         dp.n_isl = ctx->n_isl;
         dp.v_min = ctx->v_min;
         dp.v_max = ctx->v_max;

@@ -81,6 +81,7 @@ struct DelayParams {
     const double* __restrict__ vdd;          // [n_vdd][n_isl] volts
     int32_t n_vdd;
     int32_t n_isl;
+    int32_t kv_lo, kv_hi;                    // operating points with simulated slots (delay kernel rows)
     double v_min, v_max;
     double quantum;                          // 0: F mode
     float* dtab;                             // [n_vdd][n_gates][8] delays (binary32), ps; null: check only

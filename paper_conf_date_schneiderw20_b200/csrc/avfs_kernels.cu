@@ -882,8 +882,9 @@ cudaError_t launch_sweep(const SweepParams& p, bool rerun, int grid, int warps_p
 // (operating point, gate, pin, polarity); fills the table the sweep reads,
 // or (dtab null) only checks every delay for d' > 0 (reading C14).
 __global__ void delay_kernel(const DelayParams p) {
-    const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-    const int64_t total = (int64_t)p.n_vdd * p.n_gates * 8;
+    // rows kv_lo .. kv_hi-1 only: the operating points the slot range covers
+    const int64_t t = (int64_t)p.kv_lo * p.n_gates * 8 + (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    const int64_t total = (int64_t)p.kv_hi * p.n_gates * 8;
     if (t >= total) return;
     const int e = (int)(t & 7);
     const int64_t vg = t >> 3;
@@ -903,7 +904,7 @@ __global__ void delay_kernel(const DelayParams p) {
 }
 
 cudaError_t launch_delays(const DelayParams& p, cudaStream_t st) {
-    const int64_t n = (int64_t)p.n_vdd * p.n_gates * 8;
+    const int64_t n = (int64_t)(p.kv_hi - p.kv_lo) * p.n_gates * 8;
     if (n == 0) return cudaSuccess;
     delay_kernel<<<(unsigned)((n + 255) / 256), 256, 0, st>>>(p);
     return cudaGetLastError();
