@@ -138,6 +138,7 @@ struct avfs_ctx {
     std::vector<DevBuf> spill;        // per round: spill heap (kept: readback may point into it)
     int64_t spill_hint = 0;           // heap words the last simulate asked for (all rounds)
     int64_t spill_per_group = 0;      // largest heap words per slot group asked for so far (sizing hint)
+    bool spill_known = false;         // spill_per_group measured on this netlist
     int32_t n_batches = 1;            // slot batches of the last simulate (readback keeps the last)
     int32_t* h_pinned = nullptr;      // small pinned host buffer (count, err)
     cudaEvent_t ev0 = nullptr, ev1 = nullptr, ev2 = nullptr, ev3 = nullptr;   // pass-0 sweep; reruns
@@ -569,6 +570,7 @@ avfs_status avfs_load_netlist(avfs_ctx* ctx, int32_t n_pi, int32_t n_gates, cons
     ctx->net_loaded = true;
     ctx->stim_set = false;             // stimuli were packed for the previous netlist's PIs
     ctx->spill_per_group = 0;          // the heap sizing hint belongs to the previous netlist
+    ctx->spill_known = false;
     ctx->spill_hint = 0;
     ctx->plan_valid = false;
     ctx->dev_net_valid = false;
@@ -915,7 +917,9 @@ static avfs_status run_round(avfs_ctx* ctx, Round& R, int round_idx, const int32
         size_t fr = 0, tot = 0;
         CK(cudaMemGetInfo(&fr, &tot));
         const size_t have = ctx->spill[round_idx].n;
-        const size_t avail = fr + have > (1ull << 30) ? fr + have - (1ull << 30) : 0;
+        // keep 1 GiB, and for a rerun room for one more rerun round's arena
+        const size_t keep = (1ull << 30) + (round_idx > 0 ? ctx->arena[round_idx].n + ctx->recs[round_idx].n : 0);
+        const size_t avail = fr + have > keep ? fr + have - keep : 0;
         // 25 % headroom so that slowly growing requests do not reallocate every run
         size_t bytes = std::min<size_t>((size_t)R.spill_want * (R.spill_exact ? 4 : 5), avail) & ~(size_t)15;
         while (bytes >= 16 && ctx->spill[round_idx].ensure(bytes) != cudaSuccess) {
@@ -1025,6 +1029,9 @@ static avfs_status settle_batch(avfs_ctx* ctx) {
         if (ctx->h_pinned[1] & 1)
             return fail(ctx, AVFS_ERR_DELAY_NONPOS, "a delay d' = d_nom (1 + f(P)) evaluated to <= 0");
         const int32_t n_ovf = ctx->h_pinned[0];
+        if (getenv("AVFS_DEBUG"))
+            fprintf(stderr, "[avfs] round %d: %d overflowed groups, heap %.2f GB, requested %.2f GB\n", r, n_ovf,
+                    4e-9 * (double)prev.spill_words, 4e-9 * (double)prev.spill_req);
         if (n_ovf == 0) break;
         if (r >= ctx->opt.max_rerun_rounds)
             return fail(ctx, AVFS_ERR_CAPACITY, "%d slot groups still overflow at capacity %d after %d reruns",
@@ -1062,6 +1069,7 @@ static avfs_status settle_batch(avfs_ctx* ctx) {
     for (const Round& R : ctx->rounds) req += R.spill_req;
     ctx->pend_hint = std::max(ctx->pend_hint, req);
     ctx->spill_per_group = std::max<int64_t>(ctx->spill_per_group, (req + ctx->pend_r0n - 1) / ctx->pend_r0n);
+    ctx->spill_known = true;
     if (ctx->opt.profile) {
         float ms = 0;
         CK(cudaEventElapsedTime(&ms, ctx->ev0, ctx->ev1));
@@ -1207,10 +1215,16 @@ avfs_status avfs_simulate(avfs_ctx* ctx, void* cuda_stream) {
         // memory query (cudaMemGetInfo costs milliseconds at times)
         nb = n_sw_all;
     } else {
-        const int64_t fit = (int64_t)(0.8 * avail_bytes() / std::max(group_bytes(), 1.0));
+        const double av = avail_bytes();
+        const int64_t fit = (int64_t)(0.8 * av / std::max(group_bytes(), 1.0));
         if (fit < n_sw_all) {
             nb = std::max<int64_t>(1, fit);
-            if (ctx->spill_per_group == 0) { nb = std::min<int64_t>(nb, (int64_t)ctx->n_sm); learn = true; }
+            if (!ctx->spill_known) { nb = std::min<int64_t>(nb, (int64_t)ctx->n_sm); learn = true; }
+        } else if (!ctx->spill_known && (double)per_group * (double)n_sw_all > 0.5 * av && n_sw_all > ctx->n_sm) {
+            // the arena alone would take most of the memory and the spill of
+            // this netlist is not known yet: learn it on one wave first
+            nb = (int64_t)ctx->n_sm;
+            learn = true;
         }
     }
     nb = std::min(nb, n_sw_all);
@@ -1231,6 +1245,7 @@ avfs_status avfs_simulate(avfs_ctx* ctx, void* cuda_stream) {
     ctx->n_batches++;
     ctx->rounds.clear();
     Round R0;
+    const bool learning = learn && b0 == sw_lo;
     R0.n_sw = std::min(nb, sw_hi - b0);
     R0.sw_first = b0;
     R0.capacity = ctx->opt.capacity;
@@ -1245,7 +1260,15 @@ avfs_status avfs_simulate(avfs_ctx* ctx, void* cuda_stream) {
                       : std::max<int64_t>({arena_words / 4, (256ll << 20) / 4,
                                            ctx->spill_per_group * R0.n_sw + ctx->spill_per_group * R0.n_sw / 4});
         R0.spill_exact = ctx->opt.spill_bytes > 0;
+        // the first batch of a run that must learn the spill per group (one
+        // wave): give its heap most of the free memory rather than a guess
+        if (learning && ctx->opt.spill_bytes == 0)
+            R0.spill_want = std::max<int64_t>(R0.spill_want, (int64_t)(0.6 * avail_bytes() / 4.0 / 1.25));
     }
+    if (getenv("AVFS_DEBUG"))
+        fprintf(stderr, "[avfs] batch %d: groups [%lld, %lld) of %lld, heap want %.2f GB%s\n", ctx->n_batches,
+                (long long)b0, (long long)(b0 + R0.n_sw), (long long)n_sw_all, 4e-9 * (double)R0.spill_want,
+                learning ? " (learning)" : "");
     st = run_round(ctx, R0, 0, nullptr, nullptr, ctx->opt.profile != 0);
     if (st != AVFS_OK) return st;
     ctx->rounds.push_back(R0);
