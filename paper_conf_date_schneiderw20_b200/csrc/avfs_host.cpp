@@ -305,6 +305,11 @@ avfs_status build_plan(avfs_ctx* ctx) {
     int32_t n_buf = 0;
     for (int32_t L = 1; L <= ctx->depth; ++L) {
         for (int32_t b : release[L]) free_list.push_back(b);
+        // the level's gates take the free buffers in ascending order (the
+        // smallest last in the vector): consecutive gates of a level mostly
+        // get consecutive buffer ids, so their records and regions are adjacent
+        if (getenv("AVFS_SORTED_BUFFERS") == nullptr || atoi(getenv("AVFS_SORTED_BUFFERS")) != 0)
+            std::sort(free_list.begin(), free_list.end(), std::greater<int32_t>());
         for (int32_t i = ctx->level_ptr[L - 1]; i < ctx->level_ptr[L]; ++i) {
             const int32_t s = ctx->n_pi + ctx->order[i];
             if (pinned[s]) continue;

@@ -32,7 +32,7 @@ constexpr uint32_t LOC_ID = ~LOC_KIND;
 //          (E is a subset of A), meta = total stored transitions (REC_NTOT)
 //          plus REC_POISON / REC_SPILL.  PIs have no record: it is the
 //          stimulus words (init = p1, E = A = p1 xor p2, one event at t = 0).
-//  region  in the round's arena [buffer][group]: popc(A) entry words, compact
+//  region  in the round's arena [group][buffer]: popc(A) entry words, compact
 //          in the order of A's set bits (entry = n | off << ENT_OFF_SHIFT: the
 //          slot's count and the word offset of its first time), then the
 //          binary32 times right after them (byte 4 popc(A)), so a gate's

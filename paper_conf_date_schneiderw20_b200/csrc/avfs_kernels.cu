@@ -38,6 +38,9 @@ namespace avfs {
 // Byte offset of a region's in-place times (record mask A = the slots that
 // own an entry): right after the popc(A) entry words, so a gate's output is
 // one contiguous extent (AVFS_TIMES_PACKED), or at the fixed REG_TIMES.
+#ifndef AVFS_REG_GROUP_MAJOR
+#define AVFS_REG_GROUP_MAJOR 1     // regions [group][buffer] (1) or [buffer][group] (0)
+#endif
 #ifndef AVFS_REC_GROUP_MAJOR
 #define AVFS_REC_GROUP_MAJOR 1     // records [group][buffer] (1) or [buffer][group] (0)
 #endif
@@ -234,13 +237,21 @@ __device__ __forceinline__ void group_setup(const SweepParams& p, int64_t i, int
     G.kv = (int)(sw / p.n_pw);
     G.pw = (int)(sw % p.n_pw);
     G.gi = p.i_base + i;
+#if AVFS_REG_GROUP_MAJOR
+    G.row = p.arena + G.gi * p.n_buf * p.region_bytes;
+#else
     G.row = p.arena + G.gi * p.region_bytes;
+#endif
 #if AVFS_REC_GROUP_MAJOR
     G.rec = p.recs + G.gi * (int64_t)p.n_buf;
 #else
     G.rec = p.recs + G.gi;
 #endif
+#if AVFS_REG_GROUP_MAJOR
+    G.stride = (uint32_t)p.region_bytes;
+#else
     G.stride = (uint32_t)(p.pin_n_sw * p.region_bytes);
+#endif
 #if AVFS_REC_GROUP_MAJOR
     G.rstride = 1u;
 #else
@@ -1022,7 +1033,11 @@ __device__ __forceinline__ bool read_slot(const GatherRound& R, uint32_t buf, in
     const uint4 rec = R.recs[(size_t)buf * R.n_sw + idx];
 #endif
     if (rec.w & REC_POISON) return false;
+#if AVFS_REG_GROUP_MAJOR
+    const uint8_t* reg = R.pinned + ((int64_t)idx * R.n_buf + buf) * R.region_bytes;
+#else
     const uint8_t* reg = R.pinned + ((int64_t)buf * R.n_sw + idx) * R.region_bytes;
+#endif
     init = (rec.x >> l) & 1u;
     n = 0;
     ev = nullptr;
