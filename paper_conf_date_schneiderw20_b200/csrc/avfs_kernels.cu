@@ -213,7 +213,7 @@ enum : int {
     Q_A = 4, Q_EOUT = 5, Q_ACT = 6, Q_CARRY = 7,    // entry mask, accumulated event mask / count, next time offset
     Q_TB = 8,                                       // u64 time base of the output
     Q_LAST = 10, Q_FLAG = 11,                       // latest PO time bits; flags | fanout << 8
-    Q_X = 12, Q_E = 16, Q_AQ = 20, Q_LOC = 24,      // per input: init, event, entry masks; location
+    Q_X = 12, Q_E = 16, Q_AQ = 20, Q_LOC = 24,      // per input: init, observable-event, entry masks; location
     Q_ITB = 28,                                     // 4 x u64 time bases of the inputs
     Q_DLY = 36                                      // 8 delays [pin][pol], binary32 ps
 };
@@ -275,7 +275,7 @@ __device__ __forceinline__ uint32_t mux(uint32_t s, uint32_t one, uint32_t zero)
 //          possible values (X fixed where E = 0, free where E = 1)
 template <int KM>
 __device__ __forceinline__ void eval_masks(uint32_t tt, const uint32_t (&X)[4], const uint32_t (&E)[4], uint32_t& y0,
-                                           uint32_t& A) {
+                                           uint32_t& A, uint32_t (&O)[4]) {
     uint32_t lf[1 << KM];
 #pragma unroll
     for (int b = 0; b < (1 << KM); ++b) lf[b] = tt_leaf(tt, b);
@@ -299,13 +299,20 @@ __device__ __forceinline__ void eval_masks(uint32_t tt, const uint32_t (&X)[4], 
             cons[b] = cons[b] & l0;
         }
     }
-    uint32_t c0 = 0, c1 = 0;
+    // O[q]: slots where input q has events and the truth table restricted to
+    // the consistent input vectors depends on q (its events are observable)
 #pragma unroll
-    for (int b = 0; b < (1 << KM); ++b) {
-        c1 |= cons[b] & lf[b];
-        c0 |= cons[b] & ~lf[b];
+    for (int q = 0; q < 4; ++q) O[q] = 0;
+#pragma unroll
+    for (int q = 0; q < KM; ++q) {
+        const uint32_t dq = tt ^ (tt >> (1 << q));     // bit b (b_q = 0): output differs when q toggles
+        uint32_t o = 0;
+#pragma unroll
+        for (int b = 0; b < (1 << KM); ++b)
+            if (!((b >> q) & 1)) o |= cons[b] & tt_leaf(dq, b);
+        O[q] = o & E[q];
     }
-    A = c0 & c1;
+    A = O[0] | O[1] | O[2] | O[3];
 }
 
 // Eq. (4) by nested Horner in FP64 with FMA, outer in x = phi_V(v) from
@@ -372,9 +379,9 @@ __device__ __forceinline__ int phase_a(const SweepParams& p, const Grp& G, int g
             }
         }
     }
-    uint32_t y0, A;
-    if (__any_sync(FULL, K > 2)) eval_masks<4>(tt, X, E, y0, A);
-    else eval_masks<2>(tt, X, E, y0, A);
+    uint32_t y0, A, O[4];
+    if (__any_sync(FULL, K > 2)) eval_masks<4>(tt, X, E, y0, A, O);
+    else eval_masks<2>(tt, X, E, y0, A, O);
     const uint32_t U = (M[0] & REC_NTOT) + (M[1] & REC_NTOT) + (M[2] & REC_NTOT) + (M[3] & REC_NTOT);
     bool pois = on && ((M[0] | M[1] | M[2] | M[3]) & REC_POISON);
     bool own = false, spilled = false;
@@ -444,7 +451,7 @@ __device__ __forceinline__ int phase_a(const SweepParams& p, const Grp& G, int g
         sts_u32x4(qe + 4 * Q_TB, make_uint4((uint32_t)tb, (uint32_t)(tb >> 32), 0u,
                                             (counted ? QF_COUNT : 0u) | (spilled ? QF_SPILL : 0u) | (d1.w << 8)));
         sts_u32x4(qe + 4 * Q_X, make_uint4(X[0], X[1], X[2], X[3]));
-        sts_u32x4(qe + 4 * Q_E, make_uint4(E[0], E[1], E[2], E[3]));
+        sts_u32x4(qe + 4 * Q_E, make_uint4(O[0], O[1], O[2], O[3]));      // observable events
         sts_u32x4(qe + 4 * Q_AQ, make_uint4(AQ[0], AQ[1], AQ[2], AQ[3]));
         sts_u32x4(qe + 4 * Q_LOC, make_uint4(loc[0], loc[1], loc[2], loc[3]));
 #pragma unroll
@@ -595,27 +602,14 @@ __device__ __forceinline__ void phase_b(const SweepParams& p, const Grp& G, int 
         const uint32_t qe = q_s + 4u * QW * e;
         const uint4 w0 = lds_u32x4(qe + 4 * Q_TTK);
         const uint32_t tt = w0.x & 0xffffu, K = (w0.x >> 16) & 0xffu;
-        const uint4 X = lds_u32x4(qe + 4 * Q_X), Ev = lds_u32x4(qe + 4 * Q_E);
-        const uint32_t Xa[4] = {X.x, X.y, X.z, X.w}, Ea[4] = {Ev.x, Ev.y, Ev.z, Ev.w};
+        const uint4 X = lds_u32x4(qe + 4 * Q_X), Ov = lds_u32x4(qe + 4 * Q_E);
         const uint32_t lmask = (1u << l) - 1u;
-        uint32_t bits = 0, evb = 0;
-#pragma unroll
-        for (int q = 0; q < 4; ++q) {
-            bits |= ((Xa[q] >> l) & 1u) << q;
-            evb |= ((Ea[q] >> l) & 1u) << q;
-        }
-        // observable inputs of this slot: with the inputs without events at
-        // their values, the truth table restricted to the remaining minterms
-        // depends on input q
-        constexpr uint32_t POS[4] = {0xAAAAu, 0xCCCCu, 0xF0F0u, 0xFF00u};
-        uint32_t mt = 0xFFFFu >> (16 - (1 << K));
-#pragma unroll
-        for (int q = 0; q < 4; ++q)
-            if ((uint32_t)q < K && !((evb >> q) & 1u)) mt &= ((bits >> q) & 1u) ? POS[q] : ~POS[q];
-        uint32_t use = 0;
-#pragma unroll
-        for (int q = 0; q < 4; ++q)
-            if (((evb >> q) & 1u) && ((((tt >> (1 << q)) ^ tt) & mt & ~POS[q]) != 0)) use |= 1u << q;
+        // the slot's input values and its inputs with observable events
+        // (the bit-parallel phase's masks)
+        const uint32_t bits = ((X.x >> l) & 1u) | (((X.y >> l) & 1u) << 1) | (((X.z >> l) & 1u) << 2) |
+                              (((X.w >> l) & 1u) << 3);
+        uint32_t use = ((Ov.x >> l) & 1u) | (((Ov.y >> l) & 1u) << 1) | (((Ov.z >> l) & 1u) << 2) |
+                       (((Ov.w >> l) & 1u) << 3);
         if (!v) use = 0;
         // entries of the used inputs
         const uint4 AQ = lds_u32x4(qe + 4 * Q_AQ), LOC = lds_u32x4(qe + 4 * Q_LOC);
