@@ -939,8 +939,12 @@ static avfs_status run_round(avfs_ctx* ctx, Round& R, int round_idx, const int32
     DevBuf& pois = ctx->d_pois[round_idx & 1];
     CK(pois.ensure(pois_words * 4));
     CK(cudaMemsetAsync(pois.p, 0, pois_words * 4, ctx->stream));
-    CK(ctx->d_zero.ensure(16));
-    CK(cudaMemsetAsync(ctx->d_zero.p, 0, 16, ctx->stream));
+    if (ctx->d_zero.n < 16 + 128) {                 // 4 zero times, then 32 PI entries {n = 1, offset 0}
+        CK(ctx->d_zero.ensure(16 + 128));
+        uint32_t init[36] = {0u, 0u, 0u, 0u};
+        for (int k = 4; k < 36; ++k) init[k] = 1u;
+        CK(cudaMemcpy(ctx->d_zero.p, init, sizeof init, cudaMemcpyHostToDevice));
+    }
     SweepParams p{};
     p.gates = ctx->d_gates.as<GateDesc>();
     p.level_ptr = ctx->d_level_ptr.as<int32_t>();
@@ -980,6 +984,7 @@ static avfs_status run_round(avfs_ctx* ctx, Round& R, int round_idx, const int32
     p.pois_prev = round_idx == 0 ? nullptr : ctx->d_pois[(round_idx - 1) & 1].as<uint32_t>();
     p.prev_idx = d_prev_idx;
     p.zero = ctx->d_zero.as<float>();
+    p.pi_ents = reinterpret_cast<const uint32_t*>(ctx->d_zero.as<uint8_t>() + 16);
     p.act = ctx->d_act.as<unsigned long long>();
     p.latest = ctx->d_latest.as<unsigned int>();
     p.ovf = ctx->d_ovf.as<int32_t>();

@@ -128,6 +128,7 @@ struct SweepParams {
     const uint32_t* pois_prev;
     const int32_t* prev_idx;                // [n_sw] group's index in the previous round
     const float* zero;                      // 4 words of 0.0f: the time of every PI event (reading C2)
+    const uint32_t* pi_ents;                // 32 entries {n = 1, offset 0}: every PI slot with an event
     // outputs
     unsigned long long* act;                // [n_signals][n_vdd]
     unsigned int* latest;                   // [n_vdd] float bits (non-negative)

@@ -207,15 +207,16 @@ __device__ unsigned long long g_phase_cycles[16];
 #endif
 
 constexpr int QN = 16;                 // gates per batch (Phase A lanes, queue entries)
-constexpr int QW = 44;                 // words per queue entry
+constexpr int QW = 48;                 // words per queue entry
 enum : int {
     Q_TTK = 0, Q_SIG = 1, Q_OUT = 2, Q_Y0 = 3,      // descriptor words, output initial values
     Q_A = 4, Q_EOUT = 5, Q_ACT = 6, Q_CARRY = 7,    // entry mask, accumulated event mask / count, next time offset
     Q_TB = 8,                                       // u64 time base of the output
     Q_LAST = 10, Q_FLAG = 11,                       // latest PO time bits; flags | fanout << 8
-    Q_X = 12, Q_E = 16, Q_AQ = 20, Q_LOC = 24,      // per input: init, observable-event, entry masks; location
-    Q_ITB = 28,                                     // 4 x u64 time bases of the inputs
-    Q_DLY = 36                                      // 8 delays [pin][pol], binary32 ps
+    Q_X = 12, Q_E = 16, Q_AQ = 20,                  // per input: init, observable-event, entry masks
+    Q_ENTB = 24,                                    // 4 x u64 entry bases of the inputs (PIs: the PI entry table)
+    Q_ITB = 32,                                     // 4 x u64 time bases of the inputs
+    Q_DLY = 40                                      // 8 delays [pin][pol], binary32 ps
 };
 constexpr uint32_t QF_POISON = 1u, QF_COUNT = 2u, QF_OWN = 4u, QF_SPILL = 8u;
 constexpr int ITEM_WORDS = QN * 32 / 2;             // u16 items: queue entry << 5 | slot
@@ -453,15 +454,17 @@ __device__ __forceinline__ int phase_a(const SweepParams& p, const Grp& G, int g
         sts_u32x4(qe + 4 * Q_X, make_uint4(X[0], X[1], X[2], X[3]));
         sts_u32x4(qe + 4 * Q_E, make_uint4(O[0], O[1], O[2], O[3]));      // observable events
         sts_u32x4(qe + 4 * Q_AQ, make_uint4(AQ[0], AQ[1], AQ[2], AQ[3]));
-        sts_u32x4(qe + 4 * Q_LOC, make_uint4(loc[0], loc[1], loc[2], loc[3]));
 #pragma unroll
         for (int q = 0; q < 4; ++q) {
             unsigned long long itb = reinterpret_cast<unsigned long long>(p.zero);
+            unsigned long long eb = reinterpret_cast<unsigned long long>(p.pi_ents);
             if ((uint32_t)q < K && (loc[q] & LOC_KIND) != LOC_PI) {
                 const uint8_t* r = G.row + (size_t)(loc[q] & LOC_ID) * G.stride;
+                eb = reinterpret_cast<unsigned long long>(r);
                 itb = (M[q] & REC_SPILL) ? __ldcg(reinterpret_cast<const unsigned long long*>(r + REG_SPILLPTR))
                                          : reinterpret_cast<unsigned long long>(r + times_off(AQ[q]));
             }
+            sts_u64(qe + 4 * Q_ENTB + 8 * q, eb);
             sts_u64(qe + 4 * Q_ITB + 8 * q, itb);
         }
         sts_f32x4(qe + 4 * Q_DLY, dl0);
@@ -611,28 +614,45 @@ __device__ __forceinline__ void phase_b(const SweepParams& p, const Grp& G, int 
         uint32_t use = ((Ov.x >> l) & 1u) | (((Ov.y >> l) & 1u) << 1) | (((Ov.z >> l) & 1u) << 2) |
                        (((Ov.w >> l) & 1u) << 3);
         if (!v) use = 0;
-        // entries of the used inputs
-        const uint4 AQ = lds_u32x4(qe + 4 * Q_AQ), LOC = lds_u32x4(qe + 4 * Q_LOC);
-        const uint32_t AQa[4] = {AQ.x, AQ.y, AQ.z, AQ.w}, LOCa[4] = {LOC.x, LOC.y, LOC.z, LOC.w};
+        // the (at most two) first inputs with observable events, p0 < p1
+        // (list 1 may be empty), and their entries: count, time offset (PI
+        // entries point at the PI table: one event, offset 0 into the zero
+        // time, reading C2)
+        const int p0 = use ? __ffs(use) - 1 : 0;
+        const uint32_t rest = use & (use - 1u);
+        const int p1 = rest ? __ffs(rest) - 1 : p0;
+        const bool many = (rest & (rest - 1u)) != 0u;
+        uint32_t e0 = 0, e1 = 0;
+        if (use) {
+            const uint32_t* eb = reinterpret_cast<const uint32_t*>(lds_u64(qe + 4 * Q_ENTB + 8 * p0));
+            e0 = __ldcg(eb + __popc(lds_u32(qe + 4 * Q_AQ + 4 * p0) & lmask));
+        }
+        if (rest) {
+            const uint32_t* eb = reinterpret_cast<const uint32_t*>(lds_u64(qe + 4 * Q_ENTB + 8 * p1));
+            e1 = __ldcg(eb + __popc(lds_u32(qe + 4 * Q_AQ + 4 * p1) & lmask));
+        }
+        const int n0 = (int)(e0 & ENT_N), n1 = (int)(e1 & ENT_N);
+        const float* a0 = reinterpret_cast<const float*>(lds_u64(qe + 4 * Q_ITB + 8 * p0)) + (e0 >> ENT_OFF_SHIFT);
+        const float* a1 = reinterpret_cast<const float*>(lds_u64(qe + 4 * Q_ITB + 8 * p1)) + (e1 >> ENT_OFF_SHIFT);
+        uint32_t m = (uint32_t)(n0 + n1);
+        // rare: three or four inputs with observable events in this slot
         const float* ap[4];
         int nn[4];
+        const bool any_many = __any_sync(FULL, many);
+        if (any_many) {
 #pragma unroll
-        for (int q = 0; q < 4; ++q) {
-            ap[q] = p.zero;
-            nn[q] = 0;
-            if ((use >> q) & 1u) {
-                const unsigned long long itb = lds_u64(qe + 4 * Q_ITB + 8 * q);
-                if ((LOCa[q] & LOC_KIND) == LOC_PI) {
-                    nn[q] = 1;
-                } else {
-                    const uint32_t* ent = reinterpret_cast<const uint32_t*>(G.row + (size_t)(LOCa[q] & LOC_ID) * G.stride);
-                    const uint32_t w = __ldcg(ent + __popc(AQa[q] & lmask));
+            for (int q = 0; q < 4; ++q) {
+                ap[q] = p.zero;
+                nn[q] = 0;
+                if (many && ((use >> q) & 1u)) {
+                    const uint32_t* eb = reinterpret_cast<const uint32_t*>(lds_u64(qe + 4 * Q_ENTB + 8 * q));
+                    const uint32_t w = __ldcg(eb + __popc(lds_u32(qe + 4 * Q_AQ + 4 * q) & lmask));
                     nn[q] = (int)(w & ENT_N);
-                    ap[q] = reinterpret_cast<const float*>(itb) + (w >> ENT_OFF_SHIFT);
+                    ap[q] = reinterpret_cast<const float*>(lds_u64(qe + 4 * Q_ITB + 8 * q)) + (w >> ENT_OFF_SHIFT);
                 }
             }
+            if (many) m = (uint32_t)(nn[0] + nn[1] + nn[2] + nn[3]);
         }
-        const uint32_t m = (uint32_t)(nn[0] + nn[1] + nn[2] + nn[3]);
         // output offsets: segmented exclusive prefix of m over the entry's
         // items in this pass, after the entry's carry from earlier passes
         const uint32_t prev_seg = __shfl_up_sync(FULL, seg, 1);
@@ -652,27 +672,22 @@ __device__ __forceinline__ void phase_b(const SweepParams& p, const Grp& G, int 
         float* out = reinterpret_cast<float*>(tbo) + off;
         const uint32_t y0 = (w0.w >> l) & 1u;
         uint32_t n_out;
-        if (__any_sync(FULL, __popc(use) > 2)) {
+        if (any_many) {
+            if (!many) {                               // the other lanes' (at most two) lists
+#pragma unroll
+                for (int q = 0; q < 4; ++q) {
+                    ap[q] = (q == p0) ? a0 : ((q == p1 && rest) ? a1 : p.zero);
+                    nn[q] = (q == p0) ? n0 : ((q == p1 && rest) ? n1 : 0);
+                }
+            }
             n_out = merge_four(ap, nn, bits, y0, tt, qe + 4 * Q_DLY, out, steps);
         } else {
-            // the (at most two) used pins in ascending order; list 1 may be empty
-            const int p0 = use ? __ffs(use) - 1 : 0;
-            const uint32_t rest = use & (use - 1u);
-            const int p1 = rest ? __ffs(rest) - 1 : p0;
-            const float* a0 = ap[0];
-            const float* a1 = ap[0];
-            int n0 = 0, n1 = 0;
-#pragma unroll
-            for (int q = 0; q < 4; ++q) {
-                if (q == p0) { a0 = ap[q]; n0 = nn[q]; }
-                if (q == p1 && rest) { a1 = ap[q]; n1 = nn[q]; }
-            }
             float4 dl;
             dl.x = lds_f32(qe + 4 * (Q_DLY + 2 * p0));
             dl.y = lds_f32(qe + 4 * (Q_DLY + 2 * p0 + 1));
             dl.z = lds_f32(qe + 4 * (Q_DLY + 2 * p1));
             dl.w = lds_f32(qe + 4 * (Q_DLY + 2 * p1 + 1));
-            n_out = merge_two(a0, n0, a1, n1, bits, 1u << p0, rest ? 1u << p1 : 0u, y0, tt, dl, out, steps);
+            n_out = merge_two(a0, n0, a1, rest ? n1 : 0, bits, 1u << p0, rest ? 1u << p1 : 0u, y0, tt, dl, out, steps);
         }
         if (v) {
             uint32_t* oent = reinterpret_cast<uint32_t*>(G.row + (size_t)w0.z * G.stride);
