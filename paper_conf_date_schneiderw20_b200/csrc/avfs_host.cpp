@@ -129,7 +129,7 @@ struct avfs_ctx {
 
     // device state
     bool dev_net_valid = false, dev_vdd_valid = false;
-    DevBuf d_gates, d_ddesc, d_dtab, d_coef, d_cload, d_island, d_energy, c_loc, c_tclk, c_slot, c_out, d_level_ptr, d_vdd, d_p1, d_p2, d_p1t, d_p2t, d_act, d_latest, d_ovf,
+    DevBuf d_gates, d_ddesc, d_dtab, d_coef, d_cload, d_island, d_energy, c_loc, c_tclk, c_slot, c_out, d_level_ptr, d_vdd, d_p1, d_p2, d_p1t, d_p2t, d_p1g, d_p2g, d_act, d_latest, d_ovf,
         d_err, d_list[2], d_prev[2], d_pois[2], d_spill_top, d_lvlsync, d_count, d_swround, d_swindex, g_loc, g_init, g_count,
         g_times, g_bad;
     std::vector<DevBuf> arena;        // per round: [buffer][slot group][region]
@@ -154,6 +154,8 @@ struct avfs_ctx {
     std::chrono::steady_clock::time_point pend_t0;
     std::vector<Round> rounds;
     int64_t sim_first = 0, sim_end = 0;
+    SlotBox box{};                   // the last simulate's slot box (pair-major slot groups)
+    int64_t n_grp = 0;
     avfs_stats stats{};
     DelayParams dparams{};            // delay model of the last simulate (the sweep may evaluate it)
 };
@@ -950,15 +952,13 @@ static avfs_status run_round(avfs_ctx* ctx, Round& R, int round_idx, const int32
     p.level_ptr = ctx->d_level_ptr.as<int32_t>();
     p.depth = ctx->depth;
     p.n_gates = ctx->n_gates;
-    p.dtab = ctx->opt.delay_in_sweep ? nullptr : ctx->d_dtab.as<float4>();
+    p.dtab = ctx->opt.delay_in_sweep ? nullptr : ctx->d_dtab.as<float>();
     p.dp = ctx->dparams;
-    p.p1t = ctx->d_p1t.as<uint32_t>();
-    p.p2t = ctx->d_p2t.as<uint32_t>();
-    p.n_pw = (int32_t)((ctx->n_pairs + 31) / 32);
-    p.n_pairs = ctx->n_pairs;
+    p.p1g = ctx->d_p1g.as<uint32_t>();
+    p.p2g = ctx->d_p2g.as<uint32_t>();
+    p.n_grp = ctx->n_grp;
+    p.box = ctx->box;
     p.n_vdd = (int32_t)ctx->vdd.size();
-    p.slot_first = ctx->sim_first;
-    p.slot_end = ctx->sim_end;
     p.sw_list = d_sw_list;
     p.sw_first = R.sw_first;
     p.n_sw = R.n_sw;
@@ -1140,13 +1140,36 @@ avfs_status avfs_simulate(avfs_ctx* ctx, void* cuda_stream) {
     ctx->sim_first = first;
     ctx->sim_end = end;
     const int32_t n_pw = (int32_t)((P + 31) / 32);
-    const int64_t sw_lo = (first / P) * n_pw + (first % P) / 32;
-    const int64_t sw_hi = ((end - 1) / P) * n_pw + ((end - 1) % P) / 32 + 1;
+    // the slot box (SlotBox): the pairs and operating points the range
+    // covers, enumerated pair-major into 32-slot groups
+    {
+        SlotBox& b = ctx->box;
+        b.n_pairs = P;
+        b.k0 = (int32_t)(first / P);
+        b.nk = (int32_t)((end - 1) / P) - b.k0 + 1;
+        const int64_t ja = first % P, jb = (end - 1) % P;
+        if (b.nk == 1) {
+            b.j0 = ja;
+            b.nj = jb - ja + 1;
+        } else if (b.nk == 2 && jb + 1 < ja) {           // two partial rows: pairs ja .. P-1, 0 .. jb
+            b.j0 = ja;
+            b.nj = P - ja + jb + 1;
+        } else {
+            b.j0 = 0;
+            b.nj = P;
+        }
+        b.slot_first = first;
+        b.slot_end = end;
+        ctx->n_grp = (b.nj * b.nk + 31) / 32;
+    }
+    const int64_t sw_lo = 0, sw_hi = ctx->n_grp;
     const int32_t S = ctx->n_pi + ctx->n_gates;
     std::memset(&ctx->stats, 0, sizeof ctx->stats);
 
     CK(ctx->d_p1t.ensure((size_t)std::max(ctx->n_pi, 1) * n_pw * 4));
     CK(ctx->d_p2t.ensure((size_t)std::max(ctx->n_pi, 1) * n_pw * 4));
+    CK(ctx->d_p1g.ensure((size_t)std::max(ctx->n_pi, 1) * ctx->n_grp * 4));
+    CK(ctx->d_p2g.ensure((size_t)std::max(ctx->n_pi, 1) * ctx->n_grp * 4));
     CK(ctx->d_act.ensure((size_t)S * V * sizeof(unsigned long long)));
     CK(ctx->d_latest.ensure((size_t)V * 4));
     CK(ctx->d_err.ensure(16));
@@ -1160,7 +1183,7 @@ avfs_status avfs_simulate(avfs_ctx* ctx, void* cuda_stream) {
     // binary32 table, or (delay_in_sweep) only the d' > 0 check, the sweep
     // then evaluating Eq. (4)/(9) itself for the gates that need delays
     const bool in_sweep = ctx->opt.delay_in_sweep != 0;
-    if (!in_sweep) CK(ctx->d_dtab.ensure((size_t)V * std::max(ctx->n_gates, 1) * 8 * sizeof(float)));
+    if (!in_sweep) CK(ctx->d_dtab.ensure((size_t)ctx->box.nk * std::max(ctx->n_gates, 1) * 8 * sizeof(float)));
     else ctx->d_dtab.release();
     {
         DelayParams& dp = ctx->dparams;
@@ -1172,8 +1195,8 @@ avfs_status avfs_simulate(avfs_ctx* ctx, void* cuda_stream) {
         dp.deg_c = ctx->deg_c;
         dp.vdd = ctx->d_vdd.as<double>();
         dp.n_vdd = V;
-        dp.kv_lo = (int32_t)(first / P);
-        dp.kv_hi = (int32_t)((end - 1) / P + 1);
+        dp.kv_lo = ctx->box.k0;
+        dp.kv_hi = ctx->box.k0 + ctx->box.nk;
         dp.n_isl = ctx->n_isl;
         dp.v_min = ctx->v_min;
         dp.v_max = ctx->v_max;
@@ -1186,9 +1209,11 @@ avfs_status avfs_simulate(avfs_ctx* ctx, void* cuda_stream) {
     // H4: stimulus expansion (transpose to PI-major 32-pair words)
     CK(launch_expand(ctx->d_p1.as<uint32_t>(), ctx->d_p2.as<uint32_t>(), P, ctx->words, ctx->n_pi, n_pw,
                      ctx->d_p1t.as<uint32_t>(), ctx->d_p2t.as<uint32_t>(), ctx->stream));
+    CK(launch_expand_groups(ctx->d_p1.as<uint32_t>(), ctx->d_p2.as<uint32_t>(), ctx->words, ctx->n_pi, ctx->box,
+                            ctx->n_grp, ctx->d_p1g.as<uint32_t>(), ctx->d_p2g.as<uint32_t>(), ctx->stream));
     CK(launch_pi_activity(ctx->d_p1t.as<uint32_t>(), ctx->d_p2t.as<uint32_t>(), ctx->n_pi, n_pw, P, V, first, end,
                           ctx->d_act.as<unsigned long long>(), ctx->stream));
-    ctx->stats.launches += 2;
+    ctx->stats.launches += 3;
 
     ctx->rounds.clear();
     // rerun rounds' arenas and heaps of the previous simulate are kept for
@@ -1329,8 +1354,7 @@ avfs_status avfs_get_latest_arrival(avfs_ctx* ctx, float* out, int32_t out_is_de
 
 // device map slot group -> (round holding its final data, index in that round)
 static avfs_status ensure_round_map(avfs_ctx* ctx) {
-    const int32_t n_pw = (int32_t)((ctx->n_pairs + 31) / 32);
-    const int64_t n_sw_total = (int64_t)n_pw * ctx->vdd.size();
+    const int64_t n_sw_total = std::max<int64_t>(ctx->n_grp, 1);
     if (!ctx->map_valid) {
         std::vector<int32_t> rnd(n_sw_total, -1), idx(n_sw_total, 0);
         for (size_t r = 0; r < ctx->rounds.size(); ++r) {
@@ -1368,7 +1392,6 @@ static avfs_status gather(avfs_ctx* ctx, int32_t n_sig, const int32_t* sig, int6
     }
     if (n_sig == 0 || n_slots == 0) return AVFS_OK;
     const int32_t n_pw = (int32_t)((ctx->n_pairs + 31) / 32);
-    const int64_t n_sw_total = (int64_t)n_pw * ctx->vdd.size();
     {
         avfs_status ms = ensure_round_map(ctx);
         if (ms != AVFS_OK) return ms;
@@ -1386,7 +1409,7 @@ static avfs_status gather(avfs_ctx* ctx, int32_t n_sig, const int32_t* sig, int6
     g.n_sig = n_sig;
     g.slot0 = slot0;
     g.n_slots = n_slots;
-    g.n_pairs = ctx->n_pairs;
+    g.box = ctx->box;
     g.n_pw = n_pw;
     g.p1t = ctx->d_p1t.as<uint32_t>();
     g.p2t = ctx->d_p2t.as<uint32_t>();
@@ -1477,10 +1500,8 @@ avfs_status avfs_capture(avfs_ctx* ctx, const float* t_clk, int32_t n_bins, floa
     p.t_clk = ctx->c_tclk.as<float>();
     p.sw_lo = R0.sw_first;
     p.n_sw = n_sw;
-    p.n_pairs = ctx->n_pairs;
+    p.box = ctx->box;
     p.n_pw = n_pw;
-    p.slot_first = ctx->sim_first;
-    p.slot_end = ctx->sim_end;
     p.p1t = ctx->d_p1t.as<uint32_t>();
     p.p2t = ctx->d_p2t.as<uint32_t>();
     p.sw_round = ctx->d_swround.as<int32_t>();

@@ -73,6 +73,22 @@ struct alignas(16) DelayDesc {
 };
 static_assert(sizeof(DelayDesc) == 96, "DelayDesc layout");
 
+// The slots of a simulate.  Public slot s = k * n_pairs + j (stimulus pair j,
+// operating point k); the simulated range [slot_first, slot_end) lies in the
+// box pairs j0, j0 + 1, ... (nj of them, modulo n_pairs: a range that
+// straddles two rows starts at its first pair and wraps around) x points
+// [k0, k0 + nk).  Internally the box is enumerated pair-major,
+// i = ((j - j0) mod n_pairs) * nk + (k - k0), so that a pair's
+// operating points are adjacent: slot group sw = i / 32, lane i % 32.  A
+// group's slots then share (mostly) one input pair and differ only in Vdd --
+// the same transitions, scaled in time -- so their event counts are alike.
+struct SlotBox {
+    int64_t n_pairs;
+    int64_t j0, nj;
+    int32_t k0, nk;
+    int64_t slot_first, slot_end;
+};
+
 struct DelayParams {
     const DelayDesc* __restrict__ dd;
     int32_t n_gates;
@@ -81,10 +97,10 @@ struct DelayParams {
     const double* __restrict__ vdd;          // [n_vdd][n_isl] volts
     int32_t n_vdd;
     int32_t n_isl;
-    int32_t kv_lo, kv_hi;                    // operating points with simulated slots (delay kernel rows)
+    int32_t kv_lo, kv_hi;                    // operating points with simulated slots (the box's k0, k0 + nk)
     double v_min, v_max;
     double quantum;                          // 0: F mode
-    float* dtab;                             // [n_vdd][n_gates][8] delays (binary32), ps; null: check only
+    float* dtab;                             // [n_gates][8][kv_hi - kv_lo] delays (binary32), ps; null: check only
     int32_t* err;                            // bit 0: non-positive delay
 };
 
@@ -93,14 +109,13 @@ struct SweepParams {
     const int32_t* __restrict__ level_ptr;  // [depth+1] offsets into gates (level 1..depth)
     int32_t depth;
     int32_t n_gates;
-    const float4* __restrict__ dtab;        // [n_vdd][n_gates][2] float4 delays, or null: evaluated in the sweep
+    const float* __restrict__ dtab;         // [n_gates][8][box.nk] delays, or null: evaluated in the sweep
     DelayParams dp;                         // delay model (used when dtab is null)
-    const uint32_t* __restrict__ p1t;       // [n_pi][n_pw] bit-transposed stimuli
-    const uint32_t* __restrict__ p2t;
-    int32_t n_pw;                           // pair-warps (ceil(n_pairs/32))
-    int64_t n_pairs;
+    const uint32_t* __restrict__ p1g;       // [n_pi][n_grp] stimulus words per slot group (bit l: lane l's pair)
+    const uint32_t* __restrict__ p2g;
+    int64_t n_grp;                          // slot groups of the box
+    SlotBox box;
     int32_t n_vdd;
-    int64_t slot_first, slot_end;           // public slot range simulated
     // slot groups of this run: sw = sw_list ? sw_list[i] : sw_first + i, i < n_sw
     const int32_t* __restrict__ sw_list;
     int64_t sw_first;
@@ -144,6 +159,8 @@ cudaError_t launch_delays(const DelayParams& p, cudaStream_t st);
 cudaError_t launch_sweep(const SweepParams& p, bool rerun, int grid, int warps_per_cta, cudaStream_t st);
 cudaError_t launch_expand(const uint32_t* p1, const uint32_t* p2, int64_t n_pairs, int32_t words,
                           int32_t n_pi, int32_t n_pw, uint32_t* p1t, uint32_t* p2t, cudaStream_t st);
+cudaError_t launch_expand_groups(const uint32_t* p1, const uint32_t* p2, int32_t words, int32_t n_pi,
+                                 const SlotBox& box, int64_t n_grp, uint32_t* p1g, uint32_t* p2g, cudaStream_t st);
 cudaError_t launch_pi_activity(const uint32_t* p1t, const uint32_t* p2t, int32_t n_pi, int32_t n_pw,
                                int64_t n_pairs, int32_t n_vdd, int64_t slot_first, int64_t slot_end,
                                unsigned long long* act, cudaStream_t st);
@@ -162,12 +179,12 @@ struct GatherParams {
     const uint32_t* sig_loc;    // [n_sig] location codes (LOC_PI | pi, or LOC_PINNED | arena buffer)
     int32_t n_sig;
     int64_t slot0, n_slots;
-    int64_t n_pairs;
+    SlotBox box;
     int32_t n_pw;
-    const uint32_t* p1t;
+    const uint32_t* p1t;        // [n_pi][n_pw] pair-warp stimulus words (PI waveforms)
     const uint32_t* p2t;
-    const int32_t* sw_round;    // [n_sw_total] round index holding the final data (-1: not simulated)
-    const int32_t* sw_index;    // [n_sw_total] index within that round
+    const int32_t* sw_round;    // [n_grp] round index holding the final data (-1: not simulated)
+    const int32_t* sw_index;    // [n_grp] index within that round
     GatherRound rounds[8];
     int32_t cap;
     uint8_t* init;
@@ -184,9 +201,8 @@ struct CaptureParams {
     int32_t n_vdd;
     const float* t_clk;         // [n_vdd]
     int64_t sw_lo, n_sw;        // simulated slot groups [sw_lo, sw_lo + n_sw)
-    int64_t n_pairs;
+    SlotBox box;
     int32_t n_pw;
-    int64_t slot_first, slot_end;
     const uint32_t* p1t;
     const uint32_t* p2t;
     const int32_t* sw_round;

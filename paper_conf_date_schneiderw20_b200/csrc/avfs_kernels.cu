@@ -216,10 +216,10 @@ enum : int {
     Q_X = 12, Q_E = 16, Q_AQ = 20,                  // per input: init, observable-event, entry masks
     Q_ENTB = 24,                                    // 4 x u64 entry bases of the inputs (PIs: the PI entry table)
     Q_ITB = 32,                                     // 4 x u64 time bases of the inputs
-    Q_DLY = 40                                      // 8 delays [pin][pol], binary32 ps
+    Q_GATE = 40                                     // gate index (sorted; delay table row)
 };
 constexpr uint32_t QF_POISON = 1u, QF_COUNT = 2u, QF_OWN = 4u, QF_SPILL = 8u;
-constexpr int ITEM_WORDS = QN * 32 / 2;             // u16 items: queue entry << 5 | slot
+constexpr int ITEM_WORDS = QN * 32 / 2;             // u16 items: queue entry << 5 | slot, then the item's count
 constexpr int WARP_SMEM_WORDS = QN * QW + ITEM_WORDS;
 constexpr int CTA_HDR_WORDS = 2 * 32 + 4;           // level counters [group][2], pad
 
@@ -229,14 +229,28 @@ struct Grp {
     uint32_t stride;       // bytes between arena buffers (pin_n_sw * region_bytes < 4 GiB, host-checked)
     uint32_t rstride;      // records between buffers (pin_n_sw)
     int64_t gi;            // group index in the round
-    int kv, pw;
+    int64_t sw;            // slot group in the box
+    int krel;              // this lane's operating point - box.k0
     uint32_t vmask;        // slots of the group inside the simulated range
 };
 
+// lane's slot of group sw in the box (SlotBox, avfs_internal.h): pair j,
+// operating point k; false outside the box or the simulated range
+__device__ __forceinline__ bool box_slot(const SlotBox& b, int64_t sw, int lane, int64_t& j, int& k) {
+    const int64_t i = sw * 32 + lane;
+    j = 0;
+    k = b.k0;
+    if (i >= b.nj * b.nk) return false;
+    j = b.j0 + i / b.nk;
+    if (j >= b.n_pairs) j -= b.n_pairs;
+    k = b.k0 + (int)(i % b.nk);
+    const int64_t pub = (int64_t)k * b.n_pairs + j;
+    return pub >= b.slot_first && pub < b.slot_end;
+}
+
 __device__ __forceinline__ void group_setup(const SweepParams& p, int64_t i, int lane, Grp& G) {
     const int64_t sw = p.sw_list ? (int64_t)p.sw_list[i] : p.sw_first + i;
-    G.kv = (int)(sw / p.n_pw);
-    G.pw = (int)(sw % p.n_pw);
+    G.sw = sw;
     G.gi = p.i_base + i;
 #if AVFS_REG_GROUP_MAJOR
     G.row = p.arena + G.gi * p.n_buf * p.region_bytes;
@@ -258,9 +272,10 @@ __device__ __forceinline__ void group_setup(const SweepParams& p, int64_t i, int
 #else
     G.rstride = (uint32_t)p.pin_n_sw;
 #endif
-    const int64_t j = (int64_t)G.pw * 32 + lane;
-    const int64_t pub = (int64_t)G.kv * p.n_pairs + j;
-    G.vmask = __ballot_sync(FULL, j < p.n_pairs && pub >= p.slot_first && pub < p.slot_end);
+    int64_t j;
+    int k;
+    G.vmask = __ballot_sync(FULL, box_slot(p.box, sw, lane, j, k));
+    G.krel = k - p.box.k0;
 }
 
 // all-ones iff truth-table bit b is set
@@ -342,20 +357,14 @@ __device__ __forceinline__ void poison_bit(const SweepParams& p, int64_t gi, uin
 
 // Phase A for gates g0 .. g0 + nb - 1 (nb <= QN); returns the number queued.
 template <bool RERUN>
-__device__ __forceinline__ int phase_a(const SweepParams& p, const Grp& G, int g0, int nb, uint32_t q_s,
-                                       const float4* __restrict__ dt, int lane) {
+__device__ __forceinline__ int phase_a(const SweepParams& p, const Grp& G, int g0, int nb, uint32_t q_s, int lane) {
     const bool on = lane < nb;
     const int g = g0 + (on ? lane : 0);
     const uint4* gd = reinterpret_cast<const uint4*>(p.gates);
     uint4 d0 = make_uint4(0, 0, 0, 0), d1 = make_uint4(0, 0, 0, 0);
-    float4 dl0 = make_float4(0, 0, 0, 0), dl1 = dl0;
     if (on) {
         d0 = __ldg(gd + 2 * g);
         d1 = __ldg(gd + 2 * g + 1);
-        if (dt) {
-            dl0 = __ldg(dt + 2 * g);
-            dl1 = __ldg(dt + 2 * g + 1);
-        }
     }
     const uint32_t tt = d1.z & 0xffffu, K = on ? (d1.z >> 16) & 0xffu : 0u;
     const uint32_t loc[4] = {d0.x, d0.y, d0.z, d0.w};
@@ -366,8 +375,8 @@ __device__ __forceinline__ int phase_a(const SweepParams& p, const Grp& G, int g
         if ((uint32_t)q < K) {
             const uint32_t id = loc[q] & LOC_ID;
             if ((loc[q] & LOC_KIND) == LOC_PI) {       // reading C2: one event at t = 0 iff p1 != p2
-                const int64_t ix = (int64_t)id * p.n_pw + G.pw;
-                const uint32_t w1 = __ldg(p.p1t + ix), w2 = __ldg(p.p2t + ix);
+                const int64_t ix = (int64_t)id * p.n_grp + G.sw;
+                const uint32_t w1 = __ldg(p.p1g + ix), w2 = __ldg(p.p2g + ix);
                 X[q] = w1;
                 E[q] = AQ[q] = (w1 ^ w2) & G.vmask;
                 M[q] = (uint32_t)__popc(E[q]);
@@ -423,27 +432,6 @@ __device__ __forceinline__ int phase_a(const SweepParams& p, const Grp& G, int g
             if (own) p.ovf[G.gi] = 1;
         }
     }
-    if (!dt && active) {                      // Eq. (4)/(9) evaluated here, for the gates that need delays
-        const DelayParams& P = p.dp;
-        const DelayDesc& D = P.dd[g];
-        const double v = __ldg(P.vdd + (size_t)G.kv * P.n_isl + D.island);
-        const double x = (v - P.v_min) / (P.v_max - P.v_min);
-        const int nb = (P.deg_v + 1) * (P.deg_c + 1);
-        float dd[8];
-        bool bad = false;
-#pragma unroll
-        for (int e = 0; e < 8; ++e) {
-            dd[e] = 1.0f;
-            if ((uint32_t)e < 2 * K) {
-                bool b;
-                dd[e] = arc_delay(P.coef + D.coef_off + e * nb, P.deg_v, P.deg_c, x, D.z, D.dnom[e], P.quantum, b);
-                bad |= b;
-            }
-        }
-        if (bad) atomicOr(P.err, 1);
-        dl0 = make_float4(dd[0], dd[1], dd[2], dd[3]);
-        dl1 = make_float4(dd[4], dd[5], dd[6], dd[7]);
-    }
     const uint32_t bal = __ballot_sync(FULL, active);
     if (active) {
         const uint32_t qe = q_s + 4u * QW * (uint32_t)__popc(bal & lanemask_lt());
@@ -467,8 +455,7 @@ __device__ __forceinline__ int phase_a(const SweepParams& p, const Grp& G, int g
             sts_u64(qe + 4 * Q_ENTB + 8 * q, eb);
             sts_u64(qe + 4 * Q_ITB + 8 * q, itb);
         }
-        sts_f32x4(qe + 4 * Q_DLY, dl0);
-        sts_f32x4(qe + 4 * Q_DLY + 16, dl1);
+        sts_u32(qe + 4 * Q_GATE, (uint32_t)g);
     }
     __syncwarp();                             // queue entries -> the item phase's lanes
     return __popc(bal);
@@ -541,10 +528,36 @@ __device__ __forceinline__ uint32_t merge_two(const float* a0, int n0, const flo
     return F.cnt;
 }
 
+// Delay of arc e = 2 pin + pol of sorted gate `gate` at operating point k,
+// evaluated in the sweep (delay_in_sweep: Eq. (4)/(9) as in delay_kernel).
+__device__ __noinline__ float sweep_delay(const DelayDesc* __restrict__ dd, const double* __restrict__ coef,
+                                          const double* __restrict__ vdd, int n_isl, int deg_v, int deg_c,
+                                          double v_min, double v_max, double quantum, int32_t* err, uint32_t gate,
+                                          int k, int e) {
+    const DelayDesc& D = dd[gate];
+    const double v = __ldg(vdd + (size_t)k * n_isl + D.island);
+    const double x = (v - v_min) / (v_max - v_min);
+    const int nb = (deg_v + 1) * (deg_c + 1);
+    bool bad;
+    const float d = arc_delay(coef + D.coef_off + e * nb, deg_v, deg_c, x, D.z, D.dnom[e], quantum, bad);
+    if (bad) atomicOr(err, 1);
+    return d;
+}
+
+// Delay of arc e of a queued gate at slot operating point k0 + krel: the
+// table row [gate][e][krel], or evaluated here.
+__device__ __forceinline__ float item_delay(const SweepParams& p, uint32_t gate, int krel, int e) {
+    if (p.dtab) return __ldg(p.dtab + ((size_t)gate * 8 + e) * (uint32_t)p.box.nk + krel);
+    const DelayParams& P = p.dp;
+    return sweep_delay(P.dd, P.coef, P.vdd, P.n_isl, P.deg_v, P.deg_c, P.v_min, P.v_max, P.quantum, P.err, gate,
+                       p.box.k0 + krel, e);
+}
+
 // Merge of up to four sorted lists (list q = pin q, n[q] = 0 if unused);
-// delays read from the queue entry.
-__device__ __forceinline__ uint32_t merge_four(const float* const (&a_in)[4], const int (&n_in)[4], uint32_t bits,
-                                               uint32_t proj, uint32_t tt, uint32_t dly_s, float* out, uint32_t steps) {
+// delays from the table (or evaluated) per step.
+__device__ __forceinline__ uint32_t merge_four(const SweepParams& p, const float* const (&a_in)[4], const int (&n_in)[4],
+                                               uint32_t bits, uint32_t proj, uint32_t tt, uint32_t gate, int krel,
+                                               float* out, uint32_t steps) {
     float h[4];
     const float* a[4];
     int n[4];
@@ -579,7 +592,7 @@ __device__ __forceinline__ uint32_t merge_four(const float* const (&a_in)[4], co
         const bool live = t < AVFS_INF;
         bits ^= live ? (1u << pm) : 0u;
         const uint32_t y = (tt >> bits) & 1u;
-        F.step(t, live, y, lds_f32(dly_s + 8 * pm + 4 * y), out);
+        F.step(t, live, y, live ? item_delay(p, gate, krel, 2 * pm + (int)y) : 1.0f, out);
     }
     return F.cnt;
 }
@@ -604,7 +617,7 @@ __device__ __forceinline__ void phase_b(const SweepParams& p, const Grp& G, int 
         const uint32_t seg = v ? e : 31u;             // segment id (31: no entry)
         const uint32_t qe = q_s + 4u * QW * e;
         const uint4 w0 = lds_u32x4(qe + 4 * Q_TTK);
-        const uint32_t tt = w0.x & 0xffffu, K = (w0.x >> 16) & 0xffu;
+        const uint32_t tt = w0.x & 0xffffu;
         const uint4 X = lds_u32x4(qe + 4 * Q_X), Ov = lds_u32x4(qe + 4 * Q_E);
         const uint32_t lmask = (1u << l) - 1u;
         // the slot's input values and its inputs with observable events
@@ -632,6 +645,16 @@ __device__ __forceinline__ void phase_b(const SweepParams& p, const Grp& G, int 
             e1 = __ldcg(eb + __popc(lds_u32(qe + 4 * Q_AQ + 4 * p1) & lmask));
         }
         const int n0 = (int)(e0 & ENT_N), n1 = (int)(e1 & ENT_N);
+        // the slot's operating point and the delays of the two pins' arcs
+        const uint32_t gate = lds_u32(qe + 4 * Q_GATE);
+        const int krel = __shfl_sync(FULL, G.krel, (int)l);
+        float4 dl = make_float4(1.0f, 1.0f, 1.0f, 1.0f);
+        if (use && !many) {
+            dl.x = item_delay(p, gate, krel, 2 * p0);
+            dl.y = item_delay(p, gate, krel, 2 * p0 + 1);
+            dl.z = item_delay(p, gate, krel, 2 * p1);
+            dl.w = item_delay(p, gate, krel, 2 * p1 + 1);
+        }
         const float* a0 = reinterpret_cast<const float*>(lds_u64(qe + 4 * Q_ITB + 8 * p0)) + (e0 >> ENT_OFF_SHIFT);
         const float* a1 = reinterpret_cast<const float*>(lds_u64(qe + 4 * Q_ITB + 8 * p1)) + (e1 >> ENT_OFF_SHIFT);
         uint32_t m = (uint32_t)(n0 + n1);
@@ -680,13 +703,8 @@ __device__ __forceinline__ void phase_b(const SweepParams& p, const Grp& G, int 
                     nn[q] = (q == p0) ? n0 : ((q == p1 && rest) ? n1 : 0);
                 }
             }
-            n_out = merge_four(ap, nn, bits, y0, tt, qe + 4 * Q_DLY, out, steps);
+            n_out = merge_four(p, ap, nn, bits, y0, tt, gate, krel, out, steps);
         } else {
-            float4 dl;
-            dl.x = lds_f32(qe + 4 * (Q_DLY + 2 * p0));
-            dl.y = lds_f32(qe + 4 * (Q_DLY + 2 * p0 + 1));
-            dl.z = lds_f32(qe + 4 * (Q_DLY + 2 * p1));
-            dl.w = lds_f32(qe + 4 * (Q_DLY + 2 * p1 + 1));
             n_out = merge_two(a0, n0, a1, rest ? n1 : 0, bits, 1u << p0, rest ? 1u << p1 : 0u, y0, tt, dl, out, steps);
         }
         if (v) {
@@ -694,17 +712,38 @@ __device__ __forceinline__ void phase_b(const SweepParams& p, const Grp& G, int 
             const uint32_t A = lds_u32(qe + 4 * Q_A);
             __stcg(oent + __popc(A & lmask), min(n_out, ENT_N) | (off << ENT_OFF_SHIFT));
             if (m > ENT_N) atoms_or(qe + 4 * Q_FLAG, QF_POISON | QF_OWN);
-            if (n_out) {
-                atoms_or(qe + 4 * Q_EOUT, 1u << l);
-                atoms_add(qe + 4 * Q_ACT, n_out);
-                if (w0.x & (1u << 24)) atoms_max(qe + 4 * Q_LAST, __float_as_uint(__ldcg(out + n_out - 1)));
+            sts_u16(it_s + 2u * it, min(n_out, 0xFFFFu));          // the item's count replaces its code
+            // latest PO arrival at the slot's operating point (a max:
+            // recomputing a group in a rerun round changes nothing)
+            if (n_out && (w0.x & (1u << 24)))
+                atomicMax(p.latest + p.box.k0 + krel, __float_as_uint(__ldcg(out + n_out - 1)));
+        }
+        __syncwarp();
+    }
+    // per gate, lane = slot: event mask, total count, and activity per
+    // (signal, operating point) (reading C15), counted once per slot group
+    // across rerun rounds
+    {
+        uint32_t base = 0;
+        for (int e = 0; e < nq; ++e) {
+            const uint32_t qe = q_s + 4u * QW * (uint32_t)e;
+            const uint32_t A = lds_u32(qe + 4 * Q_A);
+            const uint32_t c = ((A >> lane) & 1u) ? lds_u16(it_s + 2u * (base + (uint32_t)__popc(A & lanemask_lt()))) : 0u;
+            base += (uint32_t)__popc(A);
+            const uint32_t Em = __ballot_sync(FULL, c != 0u);
+            const uint32_t tot = __reduce_add_sync(FULL, c);
+            const uint32_t fl = lds_u32(qe + 4 * Q_FLAG);
+            if (c && (fl & (QF_POISON | QF_COUNT)) == QF_COUNT)
+                atomicAdd(p.act + (size_t)lds_u32(qe + 4 * Q_SIG) * (uint32_t)p.n_vdd + (uint32_t)(p.box.k0 + G.krel),
+                          (unsigned long long)c);
+            if (lane == 0) {
+                sts_u32(qe + 4 * Q_EOUT, Em);
+                sts_u32(qe + 4 * Q_ACT, tot);
             }
         }
         __syncwarp();
     }
-    // records of the queued gates; one global atomic per gate for activity
-    // (reading C15) and the latest PO arrival, counted once per slot
-    // group across rerun rounds
+    // records of the queued gates
     if (lane < nq) {
         const uint32_t qe = q_s + 4u * QW * (uint32_t)lane;
         const uint4 w0 = lds_u32x4(qe + 4 * Q_TTK);     // ttk, sig, out, y0
@@ -719,8 +758,6 @@ __device__ __forceinline__ void phase_b(const SweepParams& p, const Grp& G, int 
             if (!RERUN || counted) poison_bit(p, G.gi, w0.y);
             if (fl & QF_OWN) p.ovf[G.gi] = 1;
         } else {
-            if (counted && w1.z) atomicAdd(p.act + (size_t)w0.y * (uint32_t)p.n_vdd + G.kv, (unsigned long long)w1.z);
-            if (counted && (w0.x & (1u << 24)) && w2.z) atomicMax(p.latest + G.kv, w2.z);
             enc += (unsigned long long)(1u + (fl >> 8)) * (unsigned long long)__popc(w1.y);
         }
     }
@@ -750,7 +787,6 @@ __global__ void __launch_bounds__(AVFS_SWEEP_THREADS, 1) sweep_kernel(const Swee
         const int64_t i = i0 + sg;
         const bool valid = i < p.n_sw;                 // idle warps still meet every level barrier
         group_setup(p, valid ? i : i0, lane, G);
-        const float4* dt = p.dtab ? p.dtab + (int64_t)G.kv * p.n_gates * 2 : nullptr;
         if (wl == 0 && lane == 0) {
             sts_u32(ctr_s, 0u);
             sts_u32(ctr_s + 4, 0u);
@@ -797,7 +833,7 @@ __global__ void __launch_bounds__(AVFS_SWEEP_THREADS, 1) sweep_kernel(const Swee
                     if ((int)gb >= nlv) break;
                     const int nb = min(bsz, nlv - (int)gb);
                     PROF_T0();
-                    const int nq = phase_a<RERUN>(p, G, ls + (int)gb, nb, q_s, dt, lane);
+                    const int nq = phase_a<RERUN>(p, G, ls + (int)gb, nb, q_s, lane);
                     PROF_ACC(1);
                     if (nq) phase_b<RERUN>(p, G, nq, q_s, it_s, lane, enc);
                     PROF_ACC(5);
@@ -902,14 +938,16 @@ cudaError_t launch_sweep(const SweepParams& p, bool rerun, int grid, int warps_p
 // (operating point, gate, pin, polarity); fills the table the sweep reads,
 // or (dtab null) only checks every delay for d' > 0 (reading C14).
 __global__ void delay_kernel(const DelayParams p) {
-    // rows kv_lo .. kv_hi-1 only: the operating points the slot range covers
-    const int64_t t = (int64_t)p.kv_lo * p.n_gates * 8 + (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-    const int64_t total = (int64_t)p.kv_hi * p.n_gates * 8;
-    if (t >= total) return;
-    const int e = (int)(t & 7);
-    const int64_t vg = t >> 3;
-    const int g = (int)(vg % p.n_gates);
-    const int kv = (int)(vg / p.n_gates);
+    // table [gate][arc][k - kv_lo], operating points kv_lo .. kv_hi-1 only
+    // (the ones the slot range covers); a warp covers consecutive points of
+    // one arc, as the sweep's items read them
+    const int nk = p.kv_hi - p.kv_lo;
+    const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (t >= (int64_t)p.n_gates * 8 * nk) return;
+    const int kv = p.kv_lo + (int)(t % nk);
+    const int64_t ge = t / nk;
+    const int e = (int)(ge & 7);
+    const int g = (int)(ge >> 3);
     const DelayDesc& D = p.dd[g];
     float out = 1.0f;
     if (e < 2 * (int)D.k) {
@@ -966,6 +1004,47 @@ cudaError_t launch_expand(const uint32_t* p1, const uint32_t* p2, int64_t n_pair
     const int64_t grid = (threads + bs - 1) / bs;
     if (grid == 0) return cudaSuccess;
     expand_kernel<<<(unsigned)grid, bs, 0, st>>>(p1, p2, n_pairs, words, n_pi, n_pw, p1t, p2t);
+    return cudaGetLastError();
+}
+
+// H4 for the sweep: stimulus words per slot group of the box, bit l of
+// p1g[i][sw] = PI i of lane l's pair (0 outside the box).  One warp per
+// (word b, group sw): 32 ballots transpose a 32x32 bit block.
+__global__ void expand_groups_kernel(const uint32_t* __restrict__ p1, const uint32_t* __restrict__ p2, int32_t words,
+                                     int32_t n_pi, const SlotBox box, int64_t n_grp, uint32_t* __restrict__ p1g,
+                                     uint32_t* __restrict__ p2g) {
+    const int lane = threadIdx.x & 31;
+    const int64_t gw = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    if (gw >= (int64_t)words * n_grp) return;
+    const int b = (int)(gw / n_grp);
+    const int64_t sw = gw % n_grp;
+    const int64_t i = sw * 32 + lane;
+    const bool in = i < box.nj * box.nk;
+    int64_t pair = box.j0 + (in ? i / box.nk : 0);
+    if (pair >= box.n_pairs) pair -= box.n_pairs;
+    const uint32_t w1 = in ? p1[pair * words + b] : 0u;
+    const uint32_t w2 = in ? p2[pair * words + b] : 0u;
+    uint32_t m1 = 0, m2 = 0;
+#pragma unroll 4
+    for (int bit = 0; bit < 32; ++bit) {
+        const uint32_t r1 = __ballot_sync(0xffffffffu, (w1 >> bit) & 1u);
+        const uint32_t r2 = __ballot_sync(0xffffffffu, (w2 >> bit) & 1u);
+        if (lane == bit) { m1 = r1; m2 = r2; }
+    }
+    const int pi = b * 32 + lane;
+    if (pi < n_pi) {
+        p1g[(int64_t)pi * n_grp + sw] = m1;
+        p2g[(int64_t)pi * n_grp + sw] = m2;
+    }
+}
+
+cudaError_t launch_expand_groups(const uint32_t* p1, const uint32_t* p2, int32_t words, int32_t n_pi,
+                                 const SlotBox& box, int64_t n_grp, uint32_t* p1g, uint32_t* p2g, cudaStream_t st) {
+    const int64_t threads = (int64_t)words * n_grp * 32;
+    const int bs = 256;
+    const int64_t grid = (threads + bs - 1) / bs;
+    if (grid == 0) return cudaSuccess;
+    expand_groups_kernel<<<(unsigned)grid, bs, 0, st>>>(p1, p2, words, n_pi, box, n_grp, p1g, p2g);
     return cudaGetLastError();
 }
 
@@ -1067,10 +1146,12 @@ __global__ void gather_kernel(const GatherParams p) {
     if (t >= (int64_t)p.n_sig * p.n_slots) return;
     const int q = (int)(t / p.n_slots);
     const int64_t s = p.slot0 + t % p.n_slots;
-    const int64_t k = s / p.n_pairs, j = s % p.n_pairs;
+    const int64_t k = s / p.box.n_pairs, j = s % p.box.n_pairs;
     const int64_t pw = j / 32;
-    const int lane = (int)(j % 32);
-    const int64_t sw = k * p.n_pw + pw;
+    const int64_t jr = j >= p.box.j0 ? j - p.box.j0 : j - p.box.j0 + p.box.n_pairs;
+    const int64_t i = jr * p.box.nk + (k - p.box.k0);                  // position in the box (SlotBox)
+    const int64_t sw = i >> 5;
+    const int lane = (int)(i & 31);
     const uint32_t loc = p.sig_loc[q];
     uint32_t init = 0;
     int n = 0;
@@ -1078,8 +1159,8 @@ __global__ void gather_kernel(const GatherParams p) {
     if ((loc & LOC_KIND) == LOC_PI) {
         const uint32_t w1 = p.p1t[(int64_t)(loc & LOC_ID) * p.n_pw + pw];
         const uint32_t w2 = p.p2t[(int64_t)(loc & LOC_ID) * p.n_pw + pw];
-        init = (w1 >> lane) & 1u;
-        n = (int)(((w1 ^ w2) >> lane) & 1u);
+        init = (w1 >> (j & 31)) & 1u;
+        n = (int)(((w1 ^ w2) >> (j & 31)) & 1u);
         if (tout) for (int i = 0; i < p.cap; ++i) tout[i] = 0.0f;
     } else {
         const int r = p.sw_round[sw];
@@ -1112,10 +1193,10 @@ __global__ void capture_kernel(const CaptureParams p) {
     const int o = (int)(gw / p.n_sw);
     const int64_t i = gw % p.n_sw;
     const int64_t sw = p.sw_lo + i;
-    const int kv = (int)(sw / p.n_pw), pw = (int)(sw % p.n_pw);
-    const int64_t j = (int64_t)pw * 32 + lane;
-    const int64_t pub = (int64_t)kv * p.n_pairs + j;
-    const bool valid = j < p.n_pairs && pub >= p.slot_first && pub < p.slot_end;
+    int64_t j;
+    int kv;
+    const bool valid = box_slot(p.box, sw, lane, j, kv);
+    const int64_t pw = j / 32;
     const float T = p.t_clk[kv];
     const uint32_t loc = p.po_loc[o];
     uint32_t init = 0, n = 0, c = 0;
@@ -1123,8 +1204,8 @@ __global__ void capture_kernel(const CaptureParams p) {
     if ((loc & LOC_KIND) == LOC_PI) {
         const uint32_t w1 = p.p1t[(int64_t)(loc & LOC_ID) * p.n_pw + pw];
         const uint32_t w2 = p.p2t[(int64_t)(loc & LOC_ID) * p.n_pw + pw];
-        init = (w1 >> lane) & 1u;
-        n = ((w1 ^ w2) >> lane) & 1u;
+        init = (w1 >> (j & 31)) & 1u;
+        n = ((w1 ^ w2) >> (j & 31)) & 1u;
         c = (n && 0.0f <= T) ? 1u : 0u;
     } else {
         const int r = p.sw_round[sw];
@@ -1141,8 +1222,7 @@ __global__ void capture_kernel(const CaptureParams p) {
         }
     }
     const bool fail = valid && (((init ^ c) & 1u) != ((init ^ n) & 1u));
-    const uint32_t fb = __ballot_sync(0xffffffffu, fail);
-    if (lane == 0 && fb) atomicAdd(p.fail_po + (int64_t)o * p.n_vdd + kv, (uint32_t)__popc(fb));
+    if (fail) atomicAdd(p.fail_po + (int64_t)o * p.n_vdd + kv, 1u);
     if (fail) atomicOr(p.slot_fail + i * 32 + lane, 1u);
     if (valid && last > 0.0f) atomicMax(p.slot_last + i * 32 + lane, __float_as_uint(last));
 }
@@ -1154,13 +1234,13 @@ __global__ void capture_finish_kernel(const CaptureParams p) {
     const int64_t i = t >> 5;
     const int lane = (int)(t & 31);
     const int64_t sw = p.sw_lo + i;
-    const int kv = (int)(sw / p.n_pw), pw = (int)(sw % p.n_pw);
-    const int64_t j = (int64_t)pw * 32 + lane;
-    const int64_t pub = (int64_t)kv * p.n_pairs + j;
-    if (!(j < p.n_pairs && pub >= p.slot_first && pub < p.slot_end)) return;
+    int64_t j;
+    int kv;
+    if (!box_slot(p.box, sw, lane, j, kv)) return;
+    const int64_t pub = (int64_t)kv * p.box.n_pairs + j;
     const uint32_t f = p.slot_fail[t];
     if (f) atomicAdd(p.fail_pairs + kv, 1u);
-    if (p.fail_bits) p.fail_bits[pub - p.slot_first] = (uint8_t)f;
+    if (p.fail_bits) p.fail_bits[pub - p.box.slot_first] = (uint8_t)f;
     if (p.hist) {
         const float slack = p.t_clk[kv] - __uint_as_float(p.slot_last[t]);
         int b = (int)floorf((slack - p.lo) / p.width);

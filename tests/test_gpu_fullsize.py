@@ -138,11 +138,12 @@ def test_fullsize_window_activity(cfg, quantum):
 @pytest.mark.slow
 def test_config5_multibatch_window_activity():
     """Whole-config-5 netlist (2M gates) in forced slot batches: a 160-slot
-    window across two Vdd points run as five 32-slot batches on one reused
-    arena; activity of every signal equals the oracle's (Q mode)."""
+    window across two Vdd points (its slot box: 160 pairs x 2 points, 10
+    groups of 32, half of them in range) run as ten one-group batches on one
+    reused arena; activity of every signal equals the oracle's (Q mode)."""
     first = 1024 * 30 - 64                               # straddles Vdd points 29 / 30
     st = _window_activity(5, 2.0 ** -8, first, 160, max_batch_slots=32)
-    assert st["batches"] == 5
+    assert st["batches"] == st["slot_warps"] == 10
 
 
 @pytest.mark.slow

@@ -329,10 +329,14 @@ def test_slot_batching(quantum):
     assert b.stats()["batches"] == 5 and a.stats()["batches"] == 1
     assert np.array_equal(a.activity(), b.activity())
     assert np.array_equal(a.latest_arrival(), b.latest_arrival())
-    last = w.n_slots - 32                                              # slots of the last group (pairs 64..95, Vdd 2)
-    wa, wb = a.waveforms(sig, last, 32, cap=16), b.waveforms(sig, last, 32, cap=16)
-    for x, y in zip(wa, wb):
-        assert np.array_equal(x, y)
+    # the last slot group holds the box's last 32 slots in pair-major order
+    # (internal i = j * n_vdd + k): pairs 85..95 at their Vdd points
+    P, V = w.stimuli.n_pairs, len(w.vdd)
+    last = [(i % V) * P + i // V for i in range(P * V - 32, P * V)]
+    for s in last:
+        wa, wb = a.waveforms(sig, s, 1, cap=16), b.waveforms(sig, s, 1, cap=16)
+        for x, y in zip(wa, wb):
+            assert np.array_equal(x, y)
     with pytest.raises(AvfsError):
         b.waveforms(sig, 0, 32, cap=16)
     with pytest.raises(AvfsError):
