@@ -12,8 +12,9 @@ the measurement through the public API with host buffers (H2D of the stimuli,
 D2H of activity + latest arrival inside the timed region).
 For N > 1 launch with torchrun (one rank per GPU).  Slots are independent
 problems, so they shard with no data-path exchange; by default the
-scaling is strong: BASELINE's config at every N, its slot space split into N
-contiguous shards ("--scaling weak" grows the pairs N-fold instead).  Config 5
+scaling is strong: BASELINE's config at every N, its stimulus pairs split into
+N contiguous ranges, each simulated at every Vdd point (whole operating-point
+sweeps per slot group; "--scaling weak" grows the pairs N-fold instead).  Config 5
 (specified on 8 x B200) runs as one shard of 8 per GPU with --gpus 8, or
 --shard-of 8 on one GPU.
 """
@@ -264,8 +265,8 @@ def config_dict(w, args):
               "mode": "F (FP64 delay polynomials, FP32 times)" if args.quantum == 0 else f"Q (quantum {args.quantum} ps)",
               "delays": "evaluated in the sweep" if getattr(args, "delay_in_sweep", False) else "delay table",
               "l2": "flushed by a 256 MiB write between timed steps; waveform arena >> L2",
-              "parallelism": (f"one slot shard of {args.shard_of} (rank 0), 1 GPU" if args.shard_of > 1 else
-                              f"slot-shard x{args.gpus} ({args.scaling})")})
+              "parallelism": (f"one pair shard of {args.shard_of} (rank 0, all Vdd points), 1 GPU"
+                              if args.shard_of > 1 else f"pair-shard x{args.gpus} ({args.scaling}, all Vdd points per rank)")})
     return d
 
 
@@ -309,7 +310,7 @@ def main():
         return
 
     import torch
-    from paper_conf_date_schneiderw20_b200 import Context, load_workload, shard_range
+    from paper_conf_date_schneiderw20_b200 import Context, load_workload, shard_pairs
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
     stream = torch.cuda.Stream(dev)
@@ -319,12 +320,13 @@ def main():
     ctx.set_options(capacity=cap, quantum_ps=args.quantum, warps_per_cta=args.warps_per_cta, profile=True,
                     delay_in_sweep=args.delay_in_sweep, spill_bytes=args.spill_bytes)
     total_slots = w.n_slots
-    first, n_local = shard_range(total_slots, rank, world)
+    P, V = w.stimuli.n_pairs, len(w.vdd)
+    first, n_local = shard_pairs(P, rank, world)
     if args.shard_of > 1 and world == 1:
-        first, n_local = shard_range(total_slots, 0, args.shard_of)
-        total_slots = n_local
-        args.shard_slots = n_local
-    ctx.set_slot_range(first, n_local)
+        first, n_local = shard_pairs(P, 0, args.shard_of)
+        total_slots = n_local * V
+        args.shard_slots = total_slots
+    ctx.set_pair_range(first, n_local)
     n_sig, V = w.netlist.n_signals, len(w.vdd)
     act_dev = torch.zeros((n_sig, V), dtype=torch.int64, device=dev)
     lat_dev = torch.zeros(V, dtype=torch.float32, device=dev)

@@ -154,6 +154,15 @@ avfs_status avfs_set_stimuli(avfs_ctx *ctx, int64_t n_pairs, const uint32_t *p1,
  * (multi-GPU sharding).  Default / n_slots < 0: all slots.        */
 avfs_status avfs_set_slot_range(avfs_ctx *ctx, int64_t first_slot, int64_t n_slots);
 
+/* Restrict simulation to stimulus pairs [first_pair, first_pair + n_pairs)
+ * at every operating point (multi-GPU sharding by pairs: each
+ * (pattern, Vdd) is independent).  The slot groups then hold whole pairs'
+ * operating-point sweeps, the layout the sweep is fastest on.  Replaces a
+ * slot range (and avfs_set_slot_range replaces this); readback accepts the
+ * public slots of these pairs.  AVFS_ERR_ARG if n_pairs < 1; at simulate,
+ * if the range exceeds the stimulus pairs.                                 */
+avfs_status avfs_set_pair_range(avfs_ctx *ctx, int64_t first_pair, int64_t n_pairs);
+
 typedef struct {
     int32_t capacity;          /* C: in-place event capacity of a 32-slot
                                   region, 32*C binary32 times.  A gate-warp
@@ -245,8 +254,10 @@ avfs_status avfs_get_waveforms(avfs_ctx *ctx, int32_t n_sig, const int32_t *sig,
  *   fail_po[n_po][n_vdd]       failing pairs per PO (PO order of the netlist); may be NULL
  *   slack_hist[n_vdd][n_bins]  slack histogram, bin b = [lo + b w, lo + (b+1) w),
  *                              values outside clamp to the first / last bin; may be NULL
- *   fail_bits[n_slots_sim]     1 byte per simulated public slot (in slot order of the
- *                              simulated range), 1 = fails; may be NULL
+ *   fail_bits[n_slots_sim]     1 byte per simulated public slot (stats.slots of them, in
+ *                              public slot order: slot - first_slot for a slot range,
+ *                              (k - 0) * n_pairs_range + (j - first_pair) for a pair
+ *                              range), 1 = fails; may be NULL
  * Runs on the device over the kept PO waveforms of the last simulate.       */
 avfs_status avfs_capture(avfs_ctx *ctx, const float *t_clk, int32_t n_bins, float lo_ps,
                          float width_ps, uint32_t *fail_pairs, uint32_t *fail_po,

@@ -6,7 +6,7 @@ package holds its thin ctypes binding and the multi-GPU slot sharding.  There
 is no CPU fallback: without the built library, Context() raises.
 """
 from .avfs import (AvfsError, Context, EXPORTS, LIB_PATH, fit_delay_polynomial, load_library, load_workload)
-from .parallel import shard_range, reduce_results
+from .parallel import shard_range, shard_pairs, reduce_results
 
 __all__ = ["AvfsError", "Context", "EXPORTS", "LIB_PATH", "fit_delay_polynomial", "load_library", "load_workload",
-           "shard_range", "reduce_results"]
+           "shard_range", "shard_pairs", "reduce_results"]

@@ -21,7 +21,7 @@ EXPORTS = [
     "avfs_create", "avfs_destroy", "avfs_last_error", "avfs_status_string", "avfs_version",
     "avfs_load_library", "avfs_load_netlist", "avfs_load_bench", "avfs_find_signal",
     "avfs_get_netlist_info", "avfs_get_levels", "avfs_get_buffer_map",
-    "avfs_set_operating_points", "avfs_set_voltage_islands", "avfs_set_stimuli", "avfs_set_slot_range",
+    "avfs_set_operating_points", "avfs_set_voltage_islands", "avfs_set_stimuli", "avfs_set_slot_range", "avfs_set_pair_range",
     "avfs_set_options", "avfs_default_options", "avfs_simulate", "avfs_sync",
     "avfs_get_activity", "avfs_get_latest_arrival", "avfs_get_final_values",
     "avfs_get_waveforms", "avfs_get_stats", "avfs_capture", "avfs_get_switching_energy",
@@ -93,6 +93,7 @@ def load_library(path: str = LIB_PATH):
             "avfs_set_voltage_islands": ([P, I32, P, I32, P], C.c_int),
             "avfs_set_stimuli": ([P, I64, P, P, I32], C.c_int),
             "avfs_set_slot_range": ([P, I64, I64], C.c_int),
+            "avfs_set_pair_range": ([P, I64, I64], C.c_int),
             "avfs_set_options": ([P, P], C.c_int),
             "avfs_default_options": ([P], C.c_int),
             "avfs_simulate": ([P, P], C.c_int),
@@ -248,6 +249,10 @@ class Context:
 
     def set_slot_range(self, first: int, n: int = -1):
         self._ck(self.lib.avfs_set_slot_range(self.h, int(first), int(n)))
+
+    def set_pair_range(self, first: int, n: int):
+        """Simulate pairs [first, first + n) at every operating point."""
+        self._ck(self.lib.avfs_set_pair_range(self.h, int(first), int(n)))
 
     def set_options(self, capacity=8, quantum_ps=0.0, probes=None, keep_all=False,
                     max_rerun_rounds=3, warps_per_cta=0, profile=False, spill_bytes=0, max_batch_slots=0,

@@ -126,6 +126,8 @@ struct avfs_ctx {
     int32_t words = 0;
     bool stim_set = false;
     int64_t slot_first = 0, slot_count = -1;
+    bool pair_mode = false;          // avfs_set_pair_range: pairs [pair_first, + pair_count) at every point
+    int64_t pair_first = 0, pair_count = 0;
 
     // device state
     bool dev_net_valid = false, dev_vdd_valid = false;
@@ -811,6 +813,20 @@ avfs_status avfs_set_slot_range(avfs_ctx* ctx, int64_t first_slot, int64_t n_slo
     if (first_slot < 0) return fail(ctx, AVFS_ERR_ARG, "negative first slot");
     ctx->slot_first = first_slot;
     ctx->slot_count = n_slots;
+    ctx->pair_mode = false;
+    invalidate_sim(ctx);
+    return AVFS_OK;
+}
+
+avfs_status avfs_set_pair_range(avfs_ctx* ctx, int64_t first_pair, int64_t n_pairs) {
+    CHECK_CTX();
+    if (first_pair < 0 || n_pairs < 1) return fail(ctx, AVFS_ERR_ARG, "bad pair range [%lld, +%lld)",
+                                                    (long long)first_pair, (long long)n_pairs);
+    ctx->pair_mode = true;
+    ctx->pair_first = first_pair;
+    ctx->pair_count = n_pairs;
+    ctx->slot_first = 0;
+    ctx->slot_count = -1;
     invalidate_sim(ctx);
     return AVFS_OK;
 }
@@ -1137,6 +1153,9 @@ avfs_status avfs_simulate(avfs_ctx* ctx, void* cuda_stream) {
     const int64_t first = ctx->slot_first;
     const int64_t end = ctx->slot_count < 0 ? total : std::min(total, first + ctx->slot_count);
     if (first >= end) return fail(ctx, AVFS_ERR_ARG, "empty slot range [%lld, %lld)", (long long)first, (long long)end);
+    if (ctx->pair_mode && ctx->pair_first + ctx->pair_count > P)
+        return fail(ctx, AVFS_ERR_ARG, "pair range [%lld, %lld) beyond the %lld stimulus pairs",
+                    (long long)ctx->pair_first, (long long)(ctx->pair_first + ctx->pair_count), (long long)P);
     ctx->sim_first = first;
     ctx->sim_end = end;
     const int32_t n_pw = (int32_t)((P + 31) / 32);
@@ -1148,7 +1167,10 @@ avfs_status avfs_simulate(avfs_ctx* ctx, void* cuda_stream) {
         b.k0 = (int32_t)(first / P);
         b.nk = (int32_t)((end - 1) / P) - b.k0 + 1;
         const int64_t ja = first % P, jb = (end - 1) % P;
-        if (b.nk == 1) {
+        if (ctx->pair_mode) {                            // every operating point of a pair range
+            b.j0 = ctx->pair_first;
+            b.nj = ctx->pair_count;
+        } else if (b.nk == 1) {
             b.j0 = ja;
             b.nj = jb - ja + 1;
         } else if (b.nk == 2 && jb + 1 < ja) {           // two partial rows: pairs ja .. P-1, 0 .. jb
@@ -1211,7 +1233,7 @@ avfs_status avfs_simulate(avfs_ctx* ctx, void* cuda_stream) {
                      ctx->d_p1t.as<uint32_t>(), ctx->d_p2t.as<uint32_t>(), ctx->stream));
     CK(launch_expand_groups(ctx->d_p1.as<uint32_t>(), ctx->d_p2.as<uint32_t>(), ctx->words, ctx->n_pi, ctx->box,
                             ctx->n_grp, ctx->d_p1g.as<uint32_t>(), ctx->d_p2g.as<uint32_t>(), ctx->stream));
-    CK(launch_pi_activity(ctx->d_p1t.as<uint32_t>(), ctx->d_p2t.as<uint32_t>(), ctx->n_pi, n_pw, P, V, first, end,
+    CK(launch_pi_activity(ctx->d_p1t.as<uint32_t>(), ctx->d_p2t.as<uint32_t>(), ctx->n_pi, n_pw, ctx->box, V,
                           ctx->d_act.as<unsigned long long>(), ctx->stream));
     ctx->stats.launches += 3;
 
@@ -1318,9 +1340,10 @@ avfs_status avfs_simulate(avfs_ctx* ctx, void* cuda_stream) {
     }
     }  // batches
     ctx->pend_t0 = t0;
-    ctx->pend_slots = end - first;
-    ctx->stats.slots = end - first;
-    ctx->stats.evals = (int64_t)ctx->n_gates * (end - first);
+    const int64_t n_sim = ctx->pair_mode ? ctx->box.nj * ctx->box.nk : end - first;
+    ctx->pend_slots = n_sim;
+    ctx->stats.slots = n_sim;
+    ctx->stats.evals = (int64_t)ctx->n_gates * n_sim;
     ctx->stats.slot_warps = sw_hi - sw_lo;
     ctx->stats.grid = ctx->rounds[0].grid;
     ctx->stats.n_scratch_buffers = ctx->n_scratch;
@@ -1381,6 +1404,12 @@ static avfs_status gather(avfs_ctx* ctx, int32_t n_sig, const int32_t* sig, int6
     if (slot0 < ctx->sim_first || slot0 + n_slots > ctx->sim_end)
         return fail(ctx, AVFS_ERR_ARG, "slots [%lld, %lld) outside the simulated range [%lld, %lld)",
                     (long long)slot0, (long long)(slot0 + n_slots), (long long)ctx->sim_first, (long long)ctx->sim_end);
+    if (ctx->pair_mode)
+        for (int64_t s = slot0; s < slot0 + n_slots; ++s)
+            if ((s % ctx->n_pairs) - ctx->pair_first < 0 || (s % ctx->n_pairs) - ctx->pair_first >= ctx->pair_count)
+                return fail(ctx, AVFS_ERR_ARG, "slot %lld (pair %lld) outside the simulated pair range [%lld, %lld)",
+                            (long long)s, (long long)(s % ctx->n_pairs), (long long)ctx->pair_first,
+                            (long long)(ctx->pair_first + ctx->pair_count));
     if (ctx->rounds.size() > 8) return fail(ctx, AVFS_ERR_STATE, "too many rounds");
     std::vector<uint32_t> sl(n_sig);
     for (int32_t i = 0; i < n_sig; ++i) {
@@ -1476,7 +1505,7 @@ avfs_status avfs_capture(avfs_ctx* ctx, const float* t_clk, int32_t n_bins, floa
     const int32_t n_po = (int32_t)ctx->po.size();
     const int32_t n_pw = (int32_t)((ctx->n_pairs + 31) / 32);
     const Round& R0 = ctx->rounds[0];
-    const int64_t n_sw = R0.n_sw, n_slots = ctx->sim_end - ctx->sim_first;
+    const int64_t n_sw = R0.n_sw, n_slots = ctx->pair_mode ? ctx->box.nj * ctx->box.nk : ctx->sim_end - ctx->sim_first;
     std::vector<uint32_t> loc(std::max(n_po, 1));
     for (int32_t o = 0; o < n_po; ++o) {
         const uint32_t l = ctx->loc[ctx->po[o]];
@@ -1517,6 +1546,7 @@ avfs_status avfs_capture(avfs_ctx* ctx, const float* t_clk, int32_t n_bins, floa
     p.n_bins = std::max(n_bins, 1);
     p.lo = lo_ps;
     p.width = width_ps > 0 ? width_ps : 1.0f;
+    p.fb_pairs = ctx->pair_mode ? 1 : 0;
     p.fail_bits = fail_bits ? reinterpret_cast<uint8_t*>(p.fail_pairs + V + (size_t)V * nb) : nullptr;
     CK(launch_capture(p, ctx->stream));
     CK(cudaMemcpyAsync(fail_pairs, p.fail_pairs, (size_t)V * 4, cudaMemcpyDeviceToHost, ctx->stream));
@@ -1569,7 +1599,7 @@ avfs_status avfs_get_stats(avfs_ctx* ctx, avfs_stats* st) {
     const int32_t S = ctx->n_pi + ctx->n_gates;
     std::vector<uint64_t> act((size_t)S * V);
     CK(cudaMemcpy(act.data(), ctx->d_act.p, act.size() * 8, cudaMemcpyDeviceToHost));
-    const double slots = (double)(ctx->sim_end - ctx->sim_first);
+    const double slots = (double)ctx->stats.slots;
     double b = 0;
     for (int32_t s = 0; s < S; ++s) {
         uint64_t a = 0;

@@ -100,7 +100,7 @@ struct DelayParams {
     int32_t kv_lo, kv_hi;                    // operating points with simulated slots (the box's k0, k0 + nk)
     double v_min, v_max;
     double quantum;                          // 0: F mode
-    float* dtab;                             // [n_gates][8][kv_hi - kv_lo] delays (binary32), ps; null: check only
+    float* dtab;                             // [n_gates][pin 4][kv_hi - kv_lo][pol 2] delays (binary32), ps; null: check only
     int32_t* err;                            // bit 0: non-positive delay
 };
 
@@ -109,7 +109,7 @@ struct SweepParams {
     const int32_t* __restrict__ level_ptr;  // [depth+1] offsets into gates (level 1..depth)
     int32_t depth;
     int32_t n_gates;
-    const float* __restrict__ dtab;         // [n_gates][8][box.nk] delays, or null: evaluated in the sweep
+    const float* __restrict__ dtab;         // [n_gates][4][box.nk][2] delays, or null: evaluated in the sweep
     DelayParams dp;                         // delay model (used when dtab is null)
     const uint32_t* __restrict__ p1g;       // [n_pi][n_grp] stimulus words per slot group (bit l: lane l's pair)
     const uint32_t* __restrict__ p2g;
@@ -162,8 +162,7 @@ cudaError_t launch_expand(const uint32_t* p1, const uint32_t* p2, int64_t n_pair
 cudaError_t launch_expand_groups(const uint32_t* p1, const uint32_t* p2, int32_t words, int32_t n_pi,
                                  const SlotBox& box, int64_t n_grp, uint32_t* p1g, uint32_t* p2g, cudaStream_t st);
 cudaError_t launch_pi_activity(const uint32_t* p1t, const uint32_t* p2t, int32_t n_pi, int32_t n_pw,
-                               int64_t n_pairs, int32_t n_vdd, int64_t slot_first, int64_t slot_end,
-                               unsigned long long* act, cudaStream_t st);
+                               const SlotBox& box, int32_t n_vdd, unsigned long long* act, cudaStream_t st);
 cudaError_t launch_compact_overflow(const int32_t* ovf, int64_t n_sw, const int32_t* sw_list,
                                     int64_t sw_first, int32_t* out_list, int32_t* out_prev,
                                     int32_t* out_count, cudaStream_t st);
@@ -215,7 +214,8 @@ struct CaptureParams {
     uint32_t* hist;             // [n_vdd][n_bins] or null
     int32_t n_bins;
     float lo, width;
-    uint8_t* fail_bits;         // [slot_end - slot_first] or null
+    uint8_t* fail_bits;         // [simulated slots] in public slot order, or null
+    int32_t fb_pairs;           // pair range: fail_bits[(k - k0) * nj + j - j0], else [slot - slot_first]
 };
 cudaError_t launch_capture(const CaptureParams& p, cudaStream_t st);
 

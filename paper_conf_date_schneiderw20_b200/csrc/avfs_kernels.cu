@@ -404,14 +404,25 @@ __device__ __forceinline__ int phase_a(const SweepParams& p, const Grp& G, int g
     }
     uint8_t* oreg = G.row + (size_t)d1.x * G.stride;
     unsigned long long tb = 0;
+    // spill-heap requests of the warp's gates: one bump allocation per warp
+    const bool want = active && U < OFF_LIMIT && U > (uint32_t)p.W;
+    const uint32_t need = want ? (U + 3u) & ~3u : 0u;
+    const uint32_t wm = __ballot_sync(FULL, want);
+    unsigned long long wb = 0;
+    if (wm) {
+        const uint32_t incl = warp_incl_scan(need, lane);
+        const uint32_t tot = __shfl_sync(FULL, incl, 31);
+        const int lead = __ffs(wm) - 1;
+        unsigned long long base = 0;
+        if (lane == lead) base = atomicAdd(p.spill_top, (unsigned long long)tot);
+        wb = __shfl_sync(FULL, base, lead) + (incl - need);
+    }
     if (active) {
         if (U >= OFF_LIMIT) {
             own = true;
         } else if (U <= (uint32_t)p.W) {
             tb = reinterpret_cast<unsigned long long>(oreg + times_off(A));
         } else {
-            const unsigned long long need = (U + 3u) & ~3u;
-            const unsigned long long wb = atomicAdd(p.spill_top, need);
             if (wb + need > p.spill_words) {
                 own = true;
             } else {
@@ -544,10 +555,10 @@ __device__ __noinline__ float sweep_delay(const DelayDesc* __restrict__ dd, cons
     return d;
 }
 
-// Delay of arc e of a queued gate at slot operating point k0 + krel: the
-// table row [gate][e][krel], or evaluated here.
+// Delay of arc e = 2 pin + pol of a queued gate at slot operating point
+// k0 + krel: the table entry [gate][pin][krel][pol], or evaluated here.
 __device__ __forceinline__ float item_delay(const SweepParams& p, uint32_t gate, int krel, int e) {
-    if (p.dtab) return __ldg(p.dtab + ((size_t)gate * 8 + e) * (uint32_t)p.box.nk + krel);
+    if (p.dtab) return __ldg(p.dtab + (((size_t)gate * 4 + (e >> 1)) * (uint32_t)p.box.nk + krel) * 2 + (e & 1));
     const DelayParams& P = p.dp;
     return sweep_delay(P.dd, P.coef, P.vdd, P.n_isl, P.deg_v, P.deg_c, P.v_min, P.v_max, P.quantum, P.err, gate,
                        p.box.k0 + krel, e);
@@ -650,10 +661,17 @@ __device__ __forceinline__ void phase_b(const SweepParams& p, const Grp& G, int 
         const int krel = __shfl_sync(FULL, G.krel, (int)l);
         float4 dl = make_float4(1.0f, 1.0f, 1.0f, 1.0f);
         if (use && !many) {
-            dl.x = item_delay(p, gate, krel, 2 * p0);
-            dl.y = item_delay(p, gate, krel, 2 * p0 + 1);
-            dl.z = item_delay(p, gate, krel, 2 * p1);
-            dl.w = item_delay(p, gate, krel, 2 * p1 + 1);
+            if (p.dtab) {                              // (fall, rise) of each pin: one 8-B load
+                const float2* db = reinterpret_cast<const float2*>(p.dtab) + (size_t)gate * 4u * (uint32_t)p.box.nk + krel;
+                const float2 d0 = __ldg(db + (uint32_t)p0 * (uint32_t)p.box.nk);
+                const float2 d1 = __ldg(db + (uint32_t)p1 * (uint32_t)p.box.nk);
+                dl = make_float4(d0.x, d0.y, d1.x, d1.y);
+            } else {
+                dl.x = item_delay(p, gate, krel, 2 * p0);
+                dl.y = item_delay(p, gate, krel, 2 * p0 + 1);
+                dl.z = item_delay(p, gate, krel, 2 * p1);
+                dl.w = item_delay(p, gate, krel, 2 * p1 + 1);
+            }
         }
         const float* a0 = reinterpret_cast<const float*>(lds_u64(qe + 4 * Q_ITB + 8 * p0)) + (e0 >> ENT_OFF_SHIFT);
         const float* a1 = reinterpret_cast<const float*>(lds_u64(qe + 4 * Q_ITB + 8 * p1)) + (e1 >> ENT_OFF_SHIFT);
@@ -938,16 +956,19 @@ cudaError_t launch_sweep(const SweepParams& p, bool rerun, int grid, int warps_p
 // (operating point, gate, pin, polarity); fills the table the sweep reads,
 // or (dtab null) only checks every delay for d' > 0 (reading C14).
 __global__ void delay_kernel(const DelayParams p) {
-    // table [gate][arc][k - kv_lo], operating points kv_lo .. kv_hi-1 only
-    // (the ones the slot range covers); a warp covers consecutive points of
-    // one arc, as the sweep's items read them
+    // table [gate][pin][k - kv_lo][pol], operating points kv_lo .. kv_hi-1
+    // only (the ones the slot range covers): a warp of the sweep's items
+    // (consecutive points of one gate) reads a pin's (fall, rise) pairs as
+    // one contiguous 8-B-per-lane load
     const int nk = p.kv_hi - p.kv_lo;
     const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (t >= (int64_t)p.n_gates * 8 * nk) return;
-    const int kv = p.kv_lo + (int)(t % nk);
-    const int64_t ge = t / nk;
-    const int e = (int)(ge & 7);
-    const int g = (int)(ge >> 3);
+    const int pol = (int)(t & 1);
+    const int64_t r = t >> 1;
+    const int kv = p.kv_lo + (int)(r % nk);
+    const int64_t gp = r / nk;
+    const int e = 2 * (int)(gp & 3) + pol;
+    const int g = (int)(gp >> 2);
     const DelayDesc& D = p.dd[g];
     float out = 1.0f;
     if (e < 2 * (int)D.k) {
@@ -1060,17 +1081,24 @@ __device__ __forceinline__ uint32_t pair_mask(int64_t pw, int64_t lo, int64_t hi
     return upto_e & ~upto_s;
 }
 
-// H8 for primary inputs: act[pi][k] = number of simulated pairs with p1 != p2.
+// H8 for primary inputs: act[pi][k] = number of simulated pairs with p1 != p2
+// (pairs of the public range at point k, within the box's pairs).
 __global__ void pi_activity_kernel(const uint32_t* __restrict__ p1t, const uint32_t* __restrict__ p2t,
-                                   int32_t n_pi, int32_t n_pw, int64_t n_pairs, int32_t n_vdd,
-                                   int64_t slot_first, int64_t slot_end, unsigned long long* act) {
+                                   int32_t n_pi, int32_t n_pw, const SlotBox box, int32_t n_vdd,
+                                   unsigned long long* act) {
     const int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (t >= (int64_t)n_pi * n_vdd) return;
     const int pi = (int)(t / n_vdd);
     const int k = (int)(t % n_vdd);
-    int64_t lo = slot_first - (int64_t)k * n_pairs, hi = slot_end - (int64_t)k * n_pairs;
+    const int64_t P = box.n_pairs;
+    int64_t lo = box.slot_first - (int64_t)k * P, hi = box.slot_end - (int64_t)k * P;
     lo = lo < 0 ? 0 : lo;
-    hi = hi > n_pairs ? n_pairs : hi;
+    hi = hi > P ? P : hi;
+    if (box.j0 + box.nj <= P) {                  // a plain pair interval (not wrapped)
+        lo = lo > box.j0 ? lo : box.j0;
+        hi = hi < box.j0 + box.nj ? hi : box.j0 + box.nj;
+    }
+    if (k < box.k0 || k >= box.k0 + box.nk) hi = lo;
     unsigned long long s = 0;
     if (hi > lo) {
         for (int64_t pw = lo / 32; pw <= (hi - 1) / 32; ++pw) {
@@ -1082,12 +1110,10 @@ __global__ void pi_activity_kernel(const uint32_t* __restrict__ p1t, const uint3
 }
 
 cudaError_t launch_pi_activity(const uint32_t* p1t, const uint32_t* p2t, int32_t n_pi, int32_t n_pw,
-                               int64_t n_pairs, int32_t n_vdd, int64_t slot_first, int64_t slot_end,
-                               unsigned long long* act, cudaStream_t st) {
+                               const SlotBox& box, int32_t n_vdd, unsigned long long* act, cudaStream_t st) {
     const int64_t n = (int64_t)n_pi * n_vdd;
     if (n == 0) return cudaSuccess;
-    pi_activity_kernel<<<(unsigned)((n + 255) / 256), 256, 0, st>>>(p1t, p2t, n_pi, n_pw, n_pairs, n_vdd,
-                                                                    slot_first, slot_end, act);
+    pi_activity_kernel<<<(unsigned)((n + 255) / 256), 256, 0, st>>>(p1t, p2t, n_pi, n_pw, box, n_vdd, act);
     return cudaGetLastError();
 }
 
@@ -1240,7 +1266,8 @@ __global__ void capture_finish_kernel(const CaptureParams p) {
     const int64_t pub = (int64_t)kv * p.box.n_pairs + j;
     const uint32_t f = p.slot_fail[t];
     if (f) atomicAdd(p.fail_pairs + kv, 1u);
-    if (p.fail_bits) p.fail_bits[pub - p.box.slot_first] = (uint8_t)f;
+    if (p.fail_bits)
+        p.fail_bits[p.fb_pairs ? (int64_t)(kv - p.box.k0) * p.box.nj + (j - p.box.j0) : pub - p.box.slot_first] = (uint8_t)f;
     if (p.hist) {
         const float slack = p.t_clk[kv] - __uint_as_float(p.slot_last[t]);
         int b = (int)floorf((slack - p.lo) / p.width);

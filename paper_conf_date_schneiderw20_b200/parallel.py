@@ -15,6 +15,13 @@ def shard_range(total_slots: int, rank: int, world: int) -> tuple:
     return first, end - first
 
 
+def shard_pairs(n_pairs: int, rank: int, world: int) -> tuple:
+    """Pairs [first, first + n) of `rank` (balanced), simulated at every
+    operating point (Context.set_pair_range): each shard keeps whole
+    operating-point sweeps of its pairs, the layout the sweep is fastest on."""
+    return shard_range(n_pairs, rank, world)
+
+
 def reduce_results(activity, latest, dst: int = 0, group=None):
     """In-place reduce of rank-local results onto `dst` (torch tensors:
     activity int64 [n_signals][n_vdd] -> SUM, latest float32 [n_vdd] -> MAX)."""

@@ -21,8 +21,8 @@ ctx = Context(0)
 load_workload(ctx, w.netlist, w.library, w.stimuli, w.vdd)
 ctx.set_options(capacity=a.capacity or w.capacity, warps_per_cta=a.warps_per_cta, profile=True)
 if a.shard_of > 1:
-    from paper_conf_date_schneiderw20_b200 import shard_range
-    ctx.set_slot_range(*shard_range(w.n_slots, 0, a.shard_of))
+    from paper_conf_date_schneiderw20_b200 import shard_pairs
+    ctx.set_pair_range(*shard_pairs(w.stimuli.n_pairs, 0, a.shard_of))
 s = torch.cuda.Stream()
 for _ in range(a.runs):
     ctx.simulate(s)

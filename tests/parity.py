@@ -18,7 +18,7 @@ REPORT = []          # per-compare taint summaries, printed by conftest at sessi
 
 def gpu_run(w_or_parts, quantum=0.0, capacity=None, keep_all=True, probes=None, slot_range=None,
             stream=None, warps_per_cta=0, max_rerun_rounds=3, netlist=None, spill_bytes=0, max_batch_slots=0,
-            delay_in_sweep=False):
+            delay_in_sweep=False, pair_range=None):
     from paper_conf_date_schneiderw20_b200 import Context, load_workload
     nl = netlist if netlist is not None else w_or_parts.netlist
     ctx = Context(0)
@@ -29,6 +29,8 @@ def gpu_run(w_or_parts, quantum=0.0, capacity=None, keep_all=True, probes=None, 
                     delay_in_sweep=delay_in_sweep, profile=True)
     if slot_range is not None:
         ctx.set_slot_range(*slot_range)
+    if pair_range is not None:
+        ctx.set_pair_range(*pair_range)
     ctx.simulate(stream)
     return ctx
 

@@ -1,6 +1,7 @@
 """N>1 host logic on CPU (-m "not gpu"): world_size-2 gloo process group.
 
-Each rank takes its shard of the public slot space (shard_range), computes the
+Each rank takes its shard of the stimulus pairs at every operating point
+(shard_pairs, as bench.py does; Context.set_pair_range), computes the
 shard's activity / latest arrival (with the oracle standing in for the GPU),
 and reduce_results() combines them on rank 0 -- exactly the bench.py path
 with NCCL replaced by gloo.  Rank 0 checks the result equals the full run.
@@ -23,11 +24,10 @@ def _free_port():
     return p
 
 
-def _shard_results(w, first, n):
+def _shard_results(w, slots):
     import oracle
     P = w.stimuli.n_pairs
     V = len(w.vdd)
-    slots = np.arange(first, first + n)
     r = oracle.simulate(w.netlist, w.library, w.stimuli, w.vdd, slots % P, slots // P, cap=64)
     act = np.zeros((w.netlist.n_signals, V), np.int64)
     lat = np.zeros(V, np.float32)
@@ -46,15 +46,16 @@ def _worker(rank, world, port, q):
     os.environ["MASTER_ADDR"] = "127.0.0.1"
     os.environ["MASTER_PORT"] = str(port)
     dist.init_process_group("gloo", rank=rank, world_size=world)
-    from paper_conf_date_schneiderw20_b200.parallel import shard_range, reduce_results
+    from paper_conf_date_schneiderw20_b200.parallel import shard_pairs, reduce_results
     from workloads import make_config
     w = make_config(3, n_pairs=40, n_vdd=3, scale=0.02)
-    first, n = shard_range(w.n_slots, rank, world)
-    act, lat = _shard_results(w, first, n)
+    P, V = w.stimuli.n_pairs, len(w.vdd)
+    first, n = shard_pairs(P, rank, world)
+    act, lat = _shard_results(w, np.array([k * P + j for j in range(first, first + n) for k in range(V)]))
     ta, tl = torch.from_numpy(act), torch.from_numpy(lat)
     reduce_results(ta, tl, dst=0)
     if rank == 0:
-        fa, fl = _shard_results(w, 0, w.n_slots)
+        fa, fl = _shard_results(w, np.arange(w.n_slots))
         q.put((bool(np.array_equal(ta.numpy(), fa)), bool(np.array_equal(tl.numpy(), fl)), int(fa.sum())))
     dist.barrier()
     dist.destroy_process_group()

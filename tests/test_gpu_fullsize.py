@@ -17,20 +17,25 @@ from tests.parity import gpu_run, gpu_waveforms, compare, activity_ref
 pytestmark = pytest.mark.gpu
 
 SAMPLES = {2: 256, 3: 128, 4: 96, 5: 12}
-# config 5 is specified on 8 x B200: one GPU simulates one eighth of its slots
+# config 5 is specified on 8 x B200: one GPU simulates one eighth of its
+# pairs at every operating point (bench.py's shard)
 SHARD = {5: (0, 8)}
 
 
-def slot_window(w):
-    from paper_conf_date_schneiderw20_b200 import shard_range
+def shard(w):
+    """bench.py's pair range for the config and the public slots it covers."""
+    from paper_conf_date_schneiderw20_b200 import shard_pairs
+    P, V = w.stimuli.n_pairs, len(w.vdd)
     r, n = SHARD.get(w.cfg, (0, 1))
-    return shard_range(w.n_slots, r, n)
+    first, cnt = shard_pairs(P, r, n)
+    slots = np.array([k * P + j for k in range(V) for j in range(first, first + cnt)], np.int64)
+    return (first, cnt), slots
 
 
 def sample_slots(w, n):
-    first, cnt = slot_window(w)
+    _, slots = shard(w)
     rng = np.random.default_rng(w.cfg)
-    return np.sort(first + rng.choice(cnt, size=n, replace=False))
+    return np.sort(rng.choice(slots, size=n, replace=False))
 
 
 @pytest.mark.parametrize("cfg,quantum", [(2, 0.0), (3, 0.0), (4, 0.0), pytest.param(5, 0.0, marks=pytest.mark.slow),
@@ -39,10 +44,10 @@ def sample_slots(w, n):
 def test_fullsize_sampled_po_parity(cfg, quantum):
     w = make_config(cfg)
     nl = w.netlist
-    first, cnt = slot_window(w)
-    ctx = gpu_run(w, keep_all=False, slot_range=(first, cnt), quantum=quantum)
+    pr, shard_slots = shard(w)
+    ctx = gpu_run(w, keep_all=False, pair_range=pr, quantum=quantum)
     st = ctx.stats()
-    assert st["evals"] == w.netlist.n_gates * cnt
+    assert st["evals"] == w.netlist.n_gates * len(shard_slots)
     slots = sample_slots(w, SAMPLES[cfg])
     P = w.stimuli.n_pairs
     ref = oracle.simulate(nl, w.library, w.stimuli, w.vdd, slots % P, slots // P, quantum=quantum,
@@ -149,10 +154,10 @@ def test_config5_multibatch_window_activity():
 @pytest.mark.slow
 @pytest.mark.parametrize("quantum", [2.0 ** -8, 0.0])
 def test_config5_all_shards(quantum):
-    """Config 5 as its 8 GPU shards, run one after another on this GPU: two
-    sampled slots per shard (all 51 Vdd points 0.60-1.10 V are covered by the
-    shards), PO waveforms vs the oracle."""
-    from paper_conf_date_schneiderw20_b200 import Context, load_workload, shard_range
+    """Config 5 as its 8 GPU shards (bench.py's pair ranges, every Vdd point
+    0.60-1.10 V in each), run one after another on this GPU: two sampled
+    slots per shard, PO waveforms vs the oracle."""
+    from paper_conf_date_schneiderw20_b200 import Context, load_workload, shard_pairs
     w = make_config(5)
     nl = w.netlist
     P = w.stimuli.n_pairs
@@ -161,16 +166,17 @@ def test_config5_all_shards(quantum):
     ctx.set_options(capacity=w.capacity, quantum_ps=quantum, keep_all=False)
     rng = np.random.default_rng(55)
     all_slots, rows = [], []
+    V = len(w.vdd)
     for r in range(8):
-        first, cnt = shard_range(w.n_slots, r, 8)
-        ctx.set_slot_range(first, cnt)
+        first, cnt = shard_pairs(P, r, 8)
+        ctx.set_pair_range(first, cnt)
         ctx.simulate()
-        slots = np.sort(first + rng.choice(cnt, size=2, replace=False))
+        slots = np.sort(rng.integers(0, V, size=2) * P + first + rng.choice(cnt, size=2, replace=False))
         for s in slots:
             rows.append(gpu_waveforms(ctx, nl.po_sig, int(s), 1, 64))
         all_slots.extend(slots.tolist())
     slots = np.array(all_slots)
-    assert len(np.unique(slots // P)) >= 8
+    assert len(np.unique(slots // P)) >= 8 and len(np.unique(slots % P)) == 16
     ref = oracle.simulate(nl, w.library, w.stimuli, w.vdd, slots % P, slots // P, quantum=quantum,
                           cap=64, out_sig=nl.po_sig)
     cap = max(1, min(64, int(ref.count.max())))
@@ -189,20 +195,21 @@ def test_config5_overflow_reruns_at_scale():
     """H7 at full size: config 5's first shard (2M gates, 204 slot groups)
     with the pass-0 spill heap capped so that part of the groups exhaust it
     and rerun.  Activity of every signal, latest arrival and the PO final
-    values of 2048 slots equal the uncapped run bit for bit (Q mode)."""
-    from paper_conf_date_schneiderw20_b200 import Context, load_workload, shard_range
+    values of the shard's slots at one operating point equal the uncapped run
+    bit for bit (Q mode)."""
+    from paper_conf_date_schneiderw20_b200 import Context, load_workload, shard_pairs
     w = make_config(5)
     nl = w.netlist
-    first, cnt = shard_range(w.n_slots, 0, 8)
+    first, cnt = shard_pairs(w.stimuli.n_pairs, 0, 8)
     res = []
     for spill in (0, 20 << 30):
         ctx = Context(0)
         load_workload(ctx, nl, w.library, w.stimuli, w.vdd)
         ctx.set_options(capacity=w.capacity, quantum_ps=2.0 ** -8, keep_all=False, spill_bytes=spill, profile=True)
-        ctx.set_slot_range(first, cnt)
+        ctx.set_pair_range(first, cnt)
         ctx.simulate()
         st = ctx.stats()
-        fv = ctx.final_values(nl.po_sig, first, 2048)
+        fv = ctx.final_values(nl.po_sig, 30 * w.stimuli.n_pairs + first, cnt)
         res.append((ctx.activity(), ctx.latest_arrival(), fv, st))
         ctx.close()
     print(f"[overflow] uncapped spill {res[0][3]['spill_bytes']} B; capped: {res[1][3]['overflow_slot_warps']} "

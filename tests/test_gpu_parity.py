@@ -181,6 +181,53 @@ def test_slot_range_shards_sum_to_full():
     assert np.array_equal(lat, lat_full)
 
 
+def test_pair_range_shards_sum_to_full():
+    """Pair ranges at every operating point (the bench's multi-GPU shards,
+    avfs_set_pair_range) reproduce the full run exactly: activity sums,
+    latest arrival maxima, PO waveforms of the shard's slots; activity equals
+    the oracle's (Q mode); slots of other pairs are refused; capture's fail
+    bits cover exactly the shard's slots."""
+    from paper_conf_date_schneiderw20_b200 import AvfsError, shard_pairs
+    w = make_config(3, n_pairs=150, n_vdd=3, scale=0.05)
+    P, V = w.stimuli.n_pairs, len(w.vdd)
+    po = w.netlist.po_sig
+    full = gpu_run(w, keep_all=False, quantum=Q)
+    act_full, lat_full = full.activity(), full.latest_arrival()
+    wf_full = full.waveforms(po, 0, w.n_slots, cap=16)
+    t_clk = np.full(V, 150.0, np.float32)
+    cap_full = full.capture(t_clk)
+    full.close()
+    acc = np.zeros_like(act_full)
+    lat = np.zeros_like(lat_full)
+    fails = np.zeros(V, np.int64)
+    for r in range(3):
+        first, n = shard_pairs(P, r, 3)
+        ctx = gpu_run(w, keep_all=False, quantum=Q, pair_range=(first, n))
+        st = ctx.stats()
+        assert st["slots"] == n * V and st["evals"] == w.netlist.n_gates * n * V
+        acc += ctx.activity()
+        lat = np.maximum(lat, ctx.latest_arrival())
+        for k in range(V):
+            wf = ctx.waveforms(po, k * P + first, n, cap=16)
+            for a, b in zip(wf, wf_full):
+                assert np.array_equal(a, b[:, k * P + first:k * P + first + n])
+        other = (first + n) % P
+        with pytest.raises(AvfsError):
+            ctx.waveforms(po, other, 1, cap=16)
+        c = ctx.capture(t_clk)
+        fails += c["fail_pairs"]
+        fb = c["fail_bits"].reshape(V, n)                # [k][j - first]
+        assert np.array_equal(fb, cap_full["fail_bits"].reshape(V, P)[:, first:first + n])
+        ctx.close()
+    assert np.array_equal(acc, act_full)
+    assert np.array_equal(lat, lat_full)
+    assert np.array_equal(fails, cap_full["fail_pairs"])
+    j, k = oracle.all_slots(P, V)
+    ref = oracle.simulate(w.netlist, w.library, w.stimuli, w.vdd, j, k, quantum=Q, cap=0)
+    ra, ok = activity_ref(ref, V, w.netlist.n_signals)
+    assert ok.all() and np.array_equal(acc.astype(np.int64), ra)
+
+
 def test_permuted_gate_order_same_results():
     w = make_config(3, n_pairs=64, n_vdd=2, scale=0.05)
     perm = w.netlist.permuted(5)
