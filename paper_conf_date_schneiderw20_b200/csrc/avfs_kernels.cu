@@ -220,7 +220,10 @@ enum : int {
 };
 constexpr uint32_t QF_POISON = 1u, QF_COUNT = 2u, QF_OWN = 4u, QF_SPILL = 8u;
 constexpr int ITEM_WORDS = QN * 32 / 2;             // u16 items: queue entry << 5 | slot, then the item's count
-constexpr int WARP_SMEM_WORDS = QN * QW + ITEM_WORDS;
+#ifndef AVFS_GATE_PASS
+#define AVFS_GATE_PASS 1
+#endif
+constexpr int WARP_SMEM_WORDS = QN * QW + (AVFS_GATE_PASS ? 0 : ITEM_WORDS);
 constexpr int CTA_HDR_WORDS = 2 * 32 + 4;           // level counters [group][2], pad
 
 struct Grp {
@@ -608,6 +611,129 @@ __device__ __forceinline__ uint32_t merge_four(const SweepParams& p, const float
     return F.cnt;
 }
 
+#if AVFS_GATE_PASS
+// Phase B, one queued gate per pass, lane = slot (pair-major groups: a
+// gate's observable slots are mostly all 32 operating points of one pair,
+// with alike event counts): merge, outputs, entries, activity and the
+// gate's record, all in registers.
+template <bool RERUN>
+__device__ __forceinline__ void phase_b(const SweepParams& p, const Grp& G, int nq, uint32_t q_s, uint32_t,
+                                        int lane, unsigned long long& enc) {
+    const uint32_t lmask = (1u << lane) - 1u;
+    const int krel = G.krel;
+    for (int e = 0; e < nq; ++e) {
+        const uint32_t qe = q_s + 4u * QW * (uint32_t)e;
+        const uint4 w0 = lds_u32x4(qe + 4 * Q_TTK);      // ttk, sig, out, y0
+        const uint32_t A = lds_u32(qe + 4 * Q_A);
+        const bool v = (A >> lane) & 1u;
+        const uint32_t tt = w0.x & 0xffffu;
+        const uint4 X = lds_u32x4(qe + 4 * Q_X), Ov = lds_u32x4(qe + 4 * Q_E);
+        // the slot's input values and its inputs with observable events
+        const uint32_t bits = ((X.x >> lane) & 1u) | (((X.y >> lane) & 1u) << 1) | (((X.z >> lane) & 1u) << 2) |
+                              (((X.w >> lane) & 1u) << 3);
+        const uint32_t use = ((Ov.x >> lane) & 1u) | (((Ov.y >> lane) & 1u) << 1) | (((Ov.z >> lane) & 1u) << 2) |
+                             (((Ov.w >> lane) & 1u) << 3);
+        // the (at most two) first inputs with observable events, p0 < p1, and
+        // their entries (PIs: the PI entry table, reading C2)
+        const int p0 = use ? __ffs(use) - 1 : 0;
+        const uint32_t rest = use & (use - 1u);
+        const int p1 = rest ? __ffs(rest) - 1 : p0;
+        const bool many = (rest & (rest - 1u)) != 0u;
+        uint32_t e0 = 0, e1 = 0;
+        if (use) {
+            const uint32_t* eb = reinterpret_cast<const uint32_t*>(lds_u64(qe + 4 * Q_ENTB + 8 * p0));
+            e0 = __ldcg(eb + __popc(lds_u32(qe + 4 * Q_AQ + 4 * p0) & lmask));
+        }
+        if (rest) {
+            const uint32_t* eb = reinterpret_cast<const uint32_t*>(lds_u64(qe + 4 * Q_ENTB + 8 * p1));
+            e1 = __ldcg(eb + __popc(lds_u32(qe + 4 * Q_AQ + 4 * p1) & lmask));
+        }
+        const uint32_t gate = lds_u32(qe + 4 * Q_GATE);
+        float4 dl = make_float4(1.0f, 1.0f, 1.0f, 1.0f);
+        if (use && !many) {
+            if (p.dtab) {                              // (fall, rise) of each pin: one 8-B load
+                const float2* db = reinterpret_cast<const float2*>(p.dtab) + (size_t)gate * 4u * (uint32_t)p.box.nk + krel;
+                const float2 d0 = __ldg(db + (uint32_t)p0 * (uint32_t)p.box.nk);
+                const float2 d1 = __ldg(db + (uint32_t)p1 * (uint32_t)p.box.nk);
+                dl = make_float4(d0.x, d0.y, d1.x, d1.y);
+            } else {
+                dl.x = item_delay(p, gate, krel, 2 * p0);
+                dl.y = item_delay(p, gate, krel, 2 * p0 + 1);
+                dl.z = item_delay(p, gate, krel, 2 * p1);
+                dl.w = item_delay(p, gate, krel, 2 * p1 + 1);
+            }
+        }
+        const int n0 = (int)(e0 & ENT_N), n1 = (int)(e1 & ENT_N);
+        const float* a0 = reinterpret_cast<const float*>(lds_u64(qe + 4 * Q_ITB + 8 * p0)) + (e0 >> ENT_OFF_SHIFT);
+        const float* a1 = reinterpret_cast<const float*>(lds_u64(qe + 4 * Q_ITB + 8 * p1)) + (e1 >> ENT_OFF_SHIFT);
+        uint32_t m = (uint32_t)(n0 + n1);
+        // rare: three or four inputs with observable events in this slot
+        const float* ap[4];
+        int nn[4];
+        const bool any_many = __any_sync(FULL, many);
+        if (any_many) {
+#pragma unroll
+            for (int q = 0; q < 4; ++q) {
+                ap[q] = p.zero;
+                nn[q] = 0;
+                if (many && ((use >> q) & 1u)) {
+                    const uint32_t* eb = reinterpret_cast<const uint32_t*>(lds_u64(qe + 4 * Q_ENTB + 8 * q));
+                    const uint32_t w = __ldcg(eb + __popc(lds_u32(qe + 4 * Q_AQ + 4 * q) & lmask));
+                    nn[q] = (int)(w & ENT_N);
+                    ap[q] = reinterpret_cast<const float*>(lds_u64(qe + 4 * Q_ITB + 8 * q)) + (w >> ENT_OFF_SHIFT);
+                }
+            }
+            if (many) m = (uint32_t)(nn[0] + nn[1] + nn[2] + nn[3]);
+        }
+        // output offsets: exclusive prefix of the slots' input counts
+        const uint32_t off = warp_incl_scan(m, lane) - m;
+        const uint32_t steps = __reduce_max_sync(FULL, m);
+        float* out = reinterpret_cast<float*>(lds_u64(qe + 4 * Q_TB)) + off;
+        const uint32_t y0 = (w0.w >> lane) & 1u;
+        uint32_t n_out;
+        if (any_many) {
+            if (!many) {                               // the other lanes' (at most two) lists
+#pragma unroll
+                for (int q = 0; q < 4; ++q) {
+                    ap[q] = (q == p0) ? a0 : ((q == p1 && rest) ? a1 : p.zero);
+                    nn[q] = (q == p0) ? n0 : ((q == p1 && rest) ? n1 : 0);
+                }
+            }
+            n_out = merge_four(p, ap, nn, bits, y0, tt, gate, krel, out, steps);
+        } else {
+            n_out = merge_two(a0, n0, a1, rest ? n1 : 0, bits, 1u << p0, rest ? 1u << p1 : 0u, y0, tt, dl, out, steps);
+        }
+        if (!v) n_out = 0;
+        // the gate's output: entries, record, activity per (signal, point)
+        // (reading C15, counted once per slot group across rerun rounds),
+        // latest PO arrival
+        if (v) {
+            uint32_t* oent = reinterpret_cast<uint32_t*>(G.row + (size_t)w0.z * G.stride);
+            __stcg(oent + __popc(A & lmask), min(n_out, ENT_N) | (off << ENT_OFF_SHIFT));
+            if (n_out && (w0.x & (1u << 24)))
+                atomicMax(p.latest + p.box.k0 + krel, __float_as_uint(__ldcg(out + n_out - 1)));
+        }
+        const bool big = __any_sync(FULL, v && m > ENT_N);
+        const uint32_t Eo = __ballot_sync(FULL, n_out != 0u);
+        const uint32_t tot = __reduce_add_sync(FULL, n_out);
+        const uint32_t fl = lds_u32(qe + 4 * Q_FLAG) | (big ? (QF_POISON | QF_OWN) : 0u);
+        const bool pois = fl & QF_POISON, counted = fl & QF_COUNT;
+        if (n_out && counted && !pois)
+            atomicAdd(p.act + (size_t)w0.y * (uint32_t)p.n_vdd + (uint32_t)(p.box.k0 + krel), (unsigned long long)n_out);
+        if (lane == 0) {
+            const uint32_t meta = pois ? REC_POISON : (tot | ((fl & QF_SPILL) ? REC_SPILL : 0u));
+            __stcg(G.rec + (size_t)w0.z * G.rstride, make_uint4(w0.w, pois ? 0u : Eo, pois ? 0u : A, meta));
+            if (pois) {
+                if (!RERUN || counted) poison_bit(p, G.gi, w0.y);
+                if (fl & QF_OWN) p.ovf[G.gi] = 1;
+            } else {
+                enc += (unsigned long long)(1u + (fl >> 8)) * (unsigned long long)__popc(Eo);
+            }
+        }
+    }
+    __syncwarp();
+}
+#else
 // Phase B over the nq queued gates, then their records.
 template <bool RERUN>
 __device__ __forceinline__ void phase_b(const SweepParams& p, const Grp& G, int nq, uint32_t q_s, uint32_t it_s,
@@ -781,6 +907,8 @@ __device__ __forceinline__ void phase_b(const SweepParams& p, const Grp& G, int 
     }
     __syncwarp();
 }
+
+#endif  // AVFS_GATE_PASS
 
 template <bool SPLIT, bool RERUN>
 __global__ void __launch_bounds__(AVFS_SWEEP_THREADS, 1) sweep_kernel(const SweepParams p) {
