@@ -876,9 +876,10 @@ static avfs_status run_round(avfs_ctx* ctx, Round& R, int round_idx, const int32
     // slot groups per sweep CTA: two by default (each group has its own
     // level barrier, so one group's wait overlaps the other's work); more
     // for narrow netlists (few gates per level), up to 8, until every warp
-    // has >= 4 gates of a level; one if the groups would not fill the SMs
+    // has two batches (2 x 32 gates) of a level; one if the groups would not
+    // fill the SMs
     int grp = wpc >= 2 ? 2 : 1;
-    while (grp < std::min(wpc, 8) && per_level / (double)(wpc / grp) < 4.0) grp *= 2;
+    while (grp < std::min(wpc, 8) && per_level / (double)(wpc / grp) < 64.0) grp *= 2;
     const int smem = sweep_smem_bytes(wpc, grp);
     int bps = 0;
     CK(sweep_occupancy(wpc, smem, &bps));

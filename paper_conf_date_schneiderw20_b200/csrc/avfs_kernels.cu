@@ -206,24 +206,21 @@ __device__ unsigned long long g_phase_cycles[16];
 #define PROF_ACC(k) do {} while (0)
 #endif
 
-constexpr int QN = 16;                 // gates per batch (Phase A lanes, queue entries)
-constexpr int QW = 48;                 // words per queue entry
+#ifndef AVFS_QN
+#define AVFS_QN 32
+#endif
+constexpr int QN = AVFS_QN;            // gates per batch (Phase A lanes, queue entries)
+constexpr int QW = 40;                 // words per queue entry
 enum : int {
     Q_TTK = 0, Q_SIG = 1, Q_OUT = 2, Q_Y0 = 3,      // descriptor words, output initial values
-    Q_A = 4, Q_EOUT = 5, Q_ACT = 6, Q_CARRY = 7,    // entry mask, accumulated event mask / count, next time offset
+    Q_A = 4, Q_GATE = 5, Q_FLAG = 6,                // entry mask, gate index (delay table row), flags | fanout << 8
     Q_TB = 8,                                       // u64 time base of the output
-    Q_LAST = 10, Q_FLAG = 11,                       // latest PO time bits; flags | fanout << 8
     Q_X = 12, Q_E = 16, Q_AQ = 20,                  // per input: init, observable-event, entry masks
     Q_ENTB = 24,                                    // 4 x u64 entry bases of the inputs (PIs: the PI entry table)
-    Q_ITB = 32,                                     // 4 x u64 time bases of the inputs
-    Q_GATE = 40                                     // gate index (sorted; delay table row)
+    Q_ITB = 32                                      // 4 x u64 time bases of the inputs
 };
 constexpr uint32_t QF_POISON = 1u, QF_COUNT = 2u, QF_OWN = 4u, QF_SPILL = 8u;
-constexpr int ITEM_WORDS = QN * 32 / 2;             // u16 items: queue entry << 5 | slot, then the item's count
-#ifndef AVFS_GATE_PASS
-#define AVFS_GATE_PASS 1
-#endif
-constexpr int WARP_SMEM_WORDS = QN * QW + (AVFS_GATE_PASS ? 0 : ITEM_WORDS);
+constexpr int WARP_SMEM_WORDS = QN * QW;
 constexpr int CTA_HDR_WORDS = 2 * 32 + 4;           // level counters [group][2], pad
 
 struct Grp {
@@ -450,9 +447,9 @@ __device__ __forceinline__ int phase_a(const SweepParams& p, const Grp& G, int g
     if (active) {
         const uint32_t qe = q_s + 4u * QW * (uint32_t)__popc(bal & lanemask_lt());
         sts_u32x4(qe + 4 * Q_TTK, make_uint4(d1.z, sig, d1.x, y0));
-        sts_u32x4(qe + 4 * Q_A, make_uint4(A, 0u, 0u, 0u));
-        sts_u32x4(qe + 4 * Q_TB, make_uint4((uint32_t)tb, (uint32_t)(tb >> 32), 0u,
-                                            (counted ? QF_COUNT : 0u) | (spilled ? QF_SPILL : 0u) | (d1.w << 8)));
+        sts_u32x4(qe + 4 * Q_A, make_uint4(A, (uint32_t)g,
+                                           (counted ? QF_COUNT : 0u) | (spilled ? QF_SPILL : 0u) | (d1.w << 8), 0u));
+        sts_u64(qe + 4 * Q_TB, tb);
         sts_u32x4(qe + 4 * Q_X, make_uint4(X[0], X[1], X[2], X[3]));
         sts_u32x4(qe + 4 * Q_E, make_uint4(O[0], O[1], O[2], O[3]));      // observable events
         sts_u32x4(qe + 4 * Q_AQ, make_uint4(AQ[0], AQ[1], AQ[2], AQ[3]));
@@ -469,7 +466,6 @@ __device__ __forceinline__ int phase_a(const SweepParams& p, const Grp& G, int g
             sts_u64(qe + 4 * Q_ENTB + 8 * q, eb);
             sts_u64(qe + 4 * Q_ITB + 8 * q, itb);
         }
-        sts_u32(qe + 4 * Q_GATE, (uint32_t)g);
     }
     __syncwarp();                             // queue entries -> the item phase's lanes
     return __popc(bal);
@@ -611,14 +607,13 @@ __device__ __forceinline__ uint32_t merge_four(const SweepParams& p, const float
     return F.cnt;
 }
 
-#if AVFS_GATE_PASS
 // Phase B, one queued gate per pass, lane = slot (pair-major groups: a
 // gate's observable slots are mostly all 32 operating points of one pair,
 // with alike event counts): merge, outputs, entries, activity and the
 // gate's record, all in registers.
 template <bool RERUN>
-__device__ __forceinline__ void phase_b(const SweepParams& p, const Grp& G, int nq, uint32_t q_s, uint32_t,
-                                        int lane, unsigned long long& enc) {
+__device__ __forceinline__ void phase_b(const SweepParams& p, const Grp& G, int nq, uint32_t q_s, int lane,
+                                        unsigned long long& enc) {
     const uint32_t lmask = (1u << lane) - 1u;
     const int krel = G.krel;
     for (int e = 0; e < nq; ++e) {
@@ -733,182 +728,7 @@ __device__ __forceinline__ void phase_b(const SweepParams& p, const Grp& G, int 
     }
     __syncwarp();
 }
-#else
-// Phase B over the nq queued gates, then their records.
-template <bool RERUN>
-__device__ __forceinline__ void phase_b(const SweepParams& p, const Grp& G, int nq, uint32_t q_s, uint32_t it_s,
-                                        int lane, unsigned long long& enc) {
-    // item list: entry e's slots in ascending order, entries in queue order
-    uint32_t T = 0;
-    for (int e = 0; e < nq; ++e) {
-        const uint32_t A = lds_u32(q_s + 4u * (QW * e + Q_A));
-        if ((A >> lane) & 1u) sts_u16(it_s + 2u * (T + (uint32_t)__popc(A & lanemask_lt())), ((uint32_t)e << 5) | lane);
-        T += (uint32_t)__popc(A);
-    }
-    __syncwarp();
-    for (uint32_t b0 = 0; b0 < T; b0 += 32) {
-        const uint32_t it = b0 + lane;
-        const bool v = it < T;
-        const uint32_t code = v ? lds_u16(it_s + 2u * it) : 0u;
-        const uint32_t e = code >> 5, l = code & 31u;
-        const uint32_t seg = v ? e : 31u;             // segment id (31: no entry)
-        const uint32_t qe = q_s + 4u * QW * e;
-        const uint4 w0 = lds_u32x4(qe + 4 * Q_TTK);
-        const uint32_t tt = w0.x & 0xffffu;
-        const uint4 X = lds_u32x4(qe + 4 * Q_X), Ov = lds_u32x4(qe + 4 * Q_E);
-        const uint32_t lmask = (1u << l) - 1u;
-        // the slot's input values and its inputs with observable events
-        // (the bit-parallel phase's masks)
-        const uint32_t bits = ((X.x >> l) & 1u) | (((X.y >> l) & 1u) << 1) | (((X.z >> l) & 1u) << 2) |
-                              (((X.w >> l) & 1u) << 3);
-        uint32_t use = ((Ov.x >> l) & 1u) | (((Ov.y >> l) & 1u) << 1) | (((Ov.z >> l) & 1u) << 2) |
-                       (((Ov.w >> l) & 1u) << 3);
-        if (!v) use = 0;
-        // the (at most two) first inputs with observable events, p0 < p1
-        // (list 1 may be empty), and their entries: count, time offset (PI
-        // entries point at the PI table: one event, offset 0 into the zero
-        // time, reading C2)
-        const int p0 = use ? __ffs(use) - 1 : 0;
-        const uint32_t rest = use & (use - 1u);
-        const int p1 = rest ? __ffs(rest) - 1 : p0;
-        const bool many = (rest & (rest - 1u)) != 0u;
-        uint32_t e0 = 0, e1 = 0;
-        if (use) {
-            const uint32_t* eb = reinterpret_cast<const uint32_t*>(lds_u64(qe + 4 * Q_ENTB + 8 * p0));
-            e0 = __ldcg(eb + __popc(lds_u32(qe + 4 * Q_AQ + 4 * p0) & lmask));
-        }
-        if (rest) {
-            const uint32_t* eb = reinterpret_cast<const uint32_t*>(lds_u64(qe + 4 * Q_ENTB + 8 * p1));
-            e1 = __ldcg(eb + __popc(lds_u32(qe + 4 * Q_AQ + 4 * p1) & lmask));
-        }
-        const int n0 = (int)(e0 & ENT_N), n1 = (int)(e1 & ENT_N);
-        // the slot's operating point and the delays of the two pins' arcs
-        const uint32_t gate = lds_u32(qe + 4 * Q_GATE);
-        const int krel = __shfl_sync(FULL, G.krel, (int)l);
-        float4 dl = make_float4(1.0f, 1.0f, 1.0f, 1.0f);
-        if (use && !many) {
-            if (p.dtab) {                              // (fall, rise) of each pin: one 8-B load
-                const float2* db = reinterpret_cast<const float2*>(p.dtab) + (size_t)gate * 4u * (uint32_t)p.box.nk + krel;
-                const float2 d0 = __ldg(db + (uint32_t)p0 * (uint32_t)p.box.nk);
-                const float2 d1 = __ldg(db + (uint32_t)p1 * (uint32_t)p.box.nk);
-                dl = make_float4(d0.x, d0.y, d1.x, d1.y);
-            } else {
-                dl.x = item_delay(p, gate, krel, 2 * p0);
-                dl.y = item_delay(p, gate, krel, 2 * p0 + 1);
-                dl.z = item_delay(p, gate, krel, 2 * p1);
-                dl.w = item_delay(p, gate, krel, 2 * p1 + 1);
-            }
-        }
-        const float* a0 = reinterpret_cast<const float*>(lds_u64(qe + 4 * Q_ITB + 8 * p0)) + (e0 >> ENT_OFF_SHIFT);
-        const float* a1 = reinterpret_cast<const float*>(lds_u64(qe + 4 * Q_ITB + 8 * p1)) + (e1 >> ENT_OFF_SHIFT);
-        uint32_t m = (uint32_t)(n0 + n1);
-        // rare: three or four inputs with observable events in this slot
-        const float* ap[4];
-        int nn[4];
-        const bool any_many = __any_sync(FULL, many);
-        if (any_many) {
-#pragma unroll
-            for (int q = 0; q < 4; ++q) {
-                ap[q] = p.zero;
-                nn[q] = 0;
-                if (many && ((use >> q) & 1u)) {
-                    const uint32_t* eb = reinterpret_cast<const uint32_t*>(lds_u64(qe + 4 * Q_ENTB + 8 * q));
-                    const uint32_t w = __ldcg(eb + __popc(lds_u32(qe + 4 * Q_AQ + 4 * q) & lmask));
-                    nn[q] = (int)(w & ENT_N);
-                    ap[q] = reinterpret_cast<const float*>(lds_u64(qe + 4 * Q_ITB + 8 * q)) + (w >> ENT_OFF_SHIFT);
-                }
-            }
-            if (many) m = (uint32_t)(nn[0] + nn[1] + nn[2] + nn[3]);
-        }
-        // output offsets: segmented exclusive prefix of m over the entry's
-        // items in this pass, after the entry's carry from earlier passes
-        const uint32_t prev_seg = __shfl_up_sync(FULL, seg, 1);
-        const bool head = lane == 0 || prev_seg != seg;
-        const uint32_t heads = __ballot_sync(FULL, head);
-        const int sl = 31 - __clz(heads & lanemask_le());
-        const uint32_t incl = warp_incl_scan(m, lane);
-        const uint32_t excl = incl - m;
-        const uint32_t seg_excl = __shfl_sync(FULL, excl, sl);
-        const uint32_t carry = lds_u32(qe + 4 * Q_CARRY);
-        const uint32_t off = carry + (excl - seg_excl);
-        const bool seg_last = (lane == 31) || ((heads >> (lane + 1)) & 1u);
-        __syncwarp();
-        if (v && seg_last) sts_u32(qe + 4 * Q_CARRY, off + m);
-        const uint32_t steps = __reduce_max_sync(FULL, m);
-        const unsigned long long tbo = lds_u64(qe + 4 * Q_TB);
-        float* out = reinterpret_cast<float*>(tbo) + off;
-        const uint32_t y0 = (w0.w >> l) & 1u;
-        uint32_t n_out;
-        if (any_many) {
-            if (!many) {                               // the other lanes' (at most two) lists
-#pragma unroll
-                for (int q = 0; q < 4; ++q) {
-                    ap[q] = (q == p0) ? a0 : ((q == p1 && rest) ? a1 : p.zero);
-                    nn[q] = (q == p0) ? n0 : ((q == p1 && rest) ? n1 : 0);
-                }
-            }
-            n_out = merge_four(p, ap, nn, bits, y0, tt, gate, krel, out, steps);
-        } else {
-            n_out = merge_two(a0, n0, a1, rest ? n1 : 0, bits, 1u << p0, rest ? 1u << p1 : 0u, y0, tt, dl, out, steps);
-        }
-        if (v) {
-            uint32_t* oent = reinterpret_cast<uint32_t*>(G.row + (size_t)w0.z * G.stride);
-            const uint32_t A = lds_u32(qe + 4 * Q_A);
-            __stcg(oent + __popc(A & lmask), min(n_out, ENT_N) | (off << ENT_OFF_SHIFT));
-            if (m > ENT_N) atoms_or(qe + 4 * Q_FLAG, QF_POISON | QF_OWN);
-            sts_u16(it_s + 2u * it, min(n_out, 0xFFFFu));          // the item's count replaces its code
-            // latest PO arrival at the slot's operating point (a max:
-            // recomputing a group in a rerun round changes nothing)
-            if (n_out && (w0.x & (1u << 24)))
-                atomicMax(p.latest + p.box.k0 + krel, __float_as_uint(__ldcg(out + n_out - 1)));
-        }
-        __syncwarp();
-    }
-    // per gate, lane = slot: event mask, total count, and activity per
-    // (signal, operating point) (reading C15), counted once per slot group
-    // across rerun rounds
-    {
-        uint32_t base = 0;
-        for (int e = 0; e < nq; ++e) {
-            const uint32_t qe = q_s + 4u * QW * (uint32_t)e;
-            const uint32_t A = lds_u32(qe + 4 * Q_A);
-            const uint32_t c = ((A >> lane) & 1u) ? lds_u16(it_s + 2u * (base + (uint32_t)__popc(A & lanemask_lt()))) : 0u;
-            base += (uint32_t)__popc(A);
-            const uint32_t Em = __ballot_sync(FULL, c != 0u);
-            const uint32_t tot = __reduce_add_sync(FULL, c);
-            const uint32_t fl = lds_u32(qe + 4 * Q_FLAG);
-            if (c && (fl & (QF_POISON | QF_COUNT)) == QF_COUNT)
-                atomicAdd(p.act + (size_t)lds_u32(qe + 4 * Q_SIG) * (uint32_t)p.n_vdd + (uint32_t)(p.box.k0 + G.krel),
-                          (unsigned long long)c);
-            if (lane == 0) {
-                sts_u32(qe + 4 * Q_EOUT, Em);
-                sts_u32(qe + 4 * Q_ACT, tot);
-            }
-        }
-        __syncwarp();
-    }
-    // records of the queued gates
-    if (lane < nq) {
-        const uint32_t qe = q_s + 4u * QW * (uint32_t)lane;
-        const uint4 w0 = lds_u32x4(qe + 4 * Q_TTK);     // ttk, sig, out, y0
-        const uint4 w1 = lds_u32x4(qe + 4 * Q_A);       // A, E, count, carry
-        const uint4 w2 = lds_u32x4(qe + 4 * Q_TB);      // time base, latest, flags
-        const uint32_t fl = w2.w;
-        const bool pois = fl & QF_POISON;
-        const uint32_t meta = pois ? REC_POISON : (w1.z | ((fl & QF_SPILL) ? REC_SPILL : 0u));
-        __stcg(G.rec + (size_t)w0.z * G.rstride, make_uint4(w0.w, pois ? 0u : w1.y, pois ? 0u : w1.x, meta));
-        const bool counted = fl & QF_COUNT;
-        if (pois) {
-            if (!RERUN || counted) poison_bit(p, G.gi, w0.y);
-            if (fl & QF_OWN) p.ovf[G.gi] = 1;
-        } else {
-            enc += (unsigned long long)(1u + (fl >> 8)) * (unsigned long long)__popc(w1.y);
-        }
-    }
-    __syncwarp();
-}
 
-#endif  // AVFS_GATE_PASS
 
 template <bool SPLIT, bool RERUN>
 __global__ void __launch_bounds__(AVFS_SWEEP_THREADS, 1) sweep_kernel(const SweepParams p) {
@@ -916,7 +736,6 @@ __global__ void __launch_bounds__(AVFS_SWEEP_THREADS, 1) sweep_kernel(const Swee
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nw = blockDim.x >> 5;
     const uint32_t base_s = smem_u32(smem_w);
     const uint32_t q_s = base_s + 4u * (uint32_t)(CTA_HDR_WORDS + warp * WARP_SMEM_WORDS);
-    const uint32_t it_s = q_s + 4u * QN * QW;
     // narrow netlists: the CTA walks GP slot groups at once, nw / GP warps
     // each; few slot groups: S co-resident CTAs (consecutive blocks, grid a
     // multiple of S) share one group, each taking 1/S of every level
@@ -981,7 +800,7 @@ __global__ void __launch_bounds__(AVFS_SWEEP_THREADS, 1) sweep_kernel(const Swee
                     PROF_T0();
                     const int nq = phase_a<RERUN>(p, G, ls + (int)gb, nb, q_s, lane);
                     PROF_ACC(1);
-                    if (nq) phase_b<RERUN>(p, G, nq, q_s, it_s, lane, enc);
+                    if (nq) phase_b<RERUN>(p, G, nq, q_s, lane, enc);
                     PROF_ACC(5);
                 }
             }
