@@ -246,8 +246,13 @@ avfs_status levelize(avfs_ctx* ctx) {
     for (int32_t g = 0; g < G; ++g) ctx->depth = std::max(ctx->depth, ctx->level[ctx->n_pi + g]);
     ctx->order.resize(G);
     for (int32_t g = 0; g < G; ++g) ctx->order[g] = g;
+    // by level; within a level, gates with <= 2 inputs first, so that most
+    // 32-gate batches evaluate the 2-input masks only (sweep phase A)
     std::stable_sort(ctx->order.begin(), ctx->order.end(), [&](int32_t a, int32_t b) {
-        return ctx->level[ctx->n_pi + a] < ctx->level[ctx->n_pi + b];
+        const int32_t la = ctx->level[ctx->n_pi + a], lb = ctx->level[ctx->n_pi + b];
+        if (la != lb) return la < lb;
+        const bool wa = ctx->fanin_ptr[a + 1] - ctx->fanin_ptr[a] > 2, wb = ctx->fanin_ptr[b + 1] - ctx->fanin_ptr[b] > 2;
+        return !wa && wb;
     });
     ctx->level_ptr.assign(ctx->depth + 1, 0);
     for (int32_t g = 0; g < G; ++g) ctx->level_ptr[ctx->level[ctx->n_pi + g]]++;

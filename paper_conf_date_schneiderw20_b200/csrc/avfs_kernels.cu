@@ -617,6 +617,7 @@ __device__ __forceinline__ void phase_b(const SweepParams& p, const Grp& G, int 
     const uint32_t lmask = (1u << lane) - 1u;
     const int krel = G.krel;
     for (int e = 0; e < nq; ++e) {
+        PROF_T0();
         const uint32_t qe = q_s + 4u * QW * (uint32_t)e;
         const uint4 w0 = lds_u32x4(qe + 4 * Q_TTK);      // ttk, sig, out, y0
         const uint32_t A = lds_u32(qe + 4 * Q_A);
@@ -683,6 +684,7 @@ __device__ __forceinline__ void phase_b(const SweepParams& p, const Grp& G, int 
         // output offsets: exclusive prefix of the slots' input counts
         const uint32_t off = warp_incl_scan(m, lane) - m;
         const uint32_t steps = __reduce_max_sync(FULL, m);
+        PROF_ACC(2);
         float* out = reinterpret_cast<float*>(lds_u64(qe + 4 * Q_TB)) + off;
         const uint32_t y0 = (w0.w >> lane) & 1u;
         uint32_t n_out;
@@ -699,6 +701,7 @@ __device__ __forceinline__ void phase_b(const SweepParams& p, const Grp& G, int 
             n_out = merge_two(a0, n0, a1, rest ? n1 : 0, bits, 1u << p0, rest ? 1u << p1 : 0u, y0, tt, dl, out, steps);
         }
         if (!v) n_out = 0;
+        PROF_ACC(3);
         // the gate's output: entries, record, activity per (signal, point)
         // (reading C15, counted once per slot group across rerun rounds),
         // latest PO arrival
@@ -725,6 +728,7 @@ __device__ __forceinline__ void phase_b(const SweepParams& p, const Grp& G, int 
                 enc += (unsigned long long)(1u + (fl >> 8)) * (unsigned long long)__popc(Eo);
             }
         }
+        PROF_ACC(4);
     }
     __syncwarp();
 }
