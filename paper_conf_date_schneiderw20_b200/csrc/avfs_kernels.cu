@@ -221,11 +221,14 @@ enum : int {
 };
 constexpr uint32_t QF_POISON = 1u, QF_COUNT = 2u, QF_OWN = 4u, QF_SPILL = 8u;
 constexpr int WARP_SMEM_WORDS = QN * QW;
-constexpr int CTA_HDR_WORDS = 2 * 32 + 4;           // level counters [group][2], pad
+constexpr int WARP_INFO_WORDS = 8;                   // per warp: enc u64, group's region row u64, record row u64
+constexpr int CTA_HDR_WORDS = 2 * 32 + 4 + 32 * WARP_INFO_WORDS;   // level counters [group][2], pad, warp info
 
+// A warp's slot group.  Its region and record rows (64-bit pointers) are
+// kept in the warp's shared info block and loaded where used (ws), not held
+// in registers through the sweep's loops.
 struct Grp {
-    uint8_t* row;          // arena + gi * region_bytes
-    uint4* rec;            // recs + gi
+    uint32_t ws;           // shared address of the warp info: +0 enc, +8 region row, +16 record row
     uint32_t stride;       // bytes between arena buffers (pin_n_sw * region_bytes < 4 GiB, host-checked)
     uint32_t rstride;      // records between buffers (pin_n_sw)
     int64_t gi;            // group index in the round
@@ -233,6 +236,9 @@ struct Grp {
     int krel;              // this lane's operating point - box.k0
     uint32_t vmask;        // slots of the group inside the simulated range
 };
+
+__device__ __forceinline__ uint8_t* grp_row(const Grp& G) { return reinterpret_cast<uint8_t*>(lds_u64(G.ws + 8)); }
+__device__ __forceinline__ uint4* grp_rec(const Grp& G) { return reinterpret_cast<uint4*>(lds_u64(G.ws + 16)); }
 
 // lane's slot of group sw in the box (SlotBox, avfs_internal.h): pair j,
 // operating point k; false outside the box or the simulated range
@@ -253,15 +259,20 @@ __device__ __forceinline__ void group_setup(const SweepParams& p, int64_t i, int
     G.sw = sw;
     G.gi = p.i_base + i;
 #if AVFS_REG_GROUP_MAJOR
-    G.row = p.arena + G.gi * p.n_buf * p.region_bytes;
+    uint8_t* row = p.arena + G.gi * p.n_buf * p.region_bytes;
 #else
-    G.row = p.arena + G.gi * p.region_bytes;
+    uint8_t* row = p.arena + G.gi * p.region_bytes;
 #endif
 #if AVFS_REC_GROUP_MAJOR
-    G.rec = p.recs + G.gi * (int64_t)p.n_buf;
+    uint4* rec = p.recs + G.gi * (int64_t)p.n_buf;
 #else
-    G.rec = p.recs + G.gi;
+    uint4* rec = p.recs + G.gi;
 #endif
+    if (lane == 0) {
+        sts_u64(G.ws + 8, reinterpret_cast<unsigned long long>(row));
+        sts_u64(G.ws + 16, reinterpret_cast<unsigned long long>(rec));
+    }
+    __syncwarp();
 #if AVFS_REG_GROUP_MAJOR
     G.stride = (uint32_t)p.region_bytes;
 #else
@@ -381,7 +392,7 @@ __device__ __forceinline__ int phase_a(const SweepParams& p, const Grp& G, int g
                 E[q] = AQ[q] = (w1 ^ w2) & G.vmask;
                 M[q] = (uint32_t)__popc(E[q]);
             } else {
-                const uint4 r = __ldcg(G.rec + (size_t)id * G.rstride);
+                const uint4 r = __ldcg(grp_rec(G) + (size_t)id * G.rstride);
                 X[q] = r.x;
                 E[q] = r.y;
                 AQ[q] = r.z;
@@ -402,7 +413,7 @@ __device__ __forceinline__ int phase_a(const SweepParams& p, const Grp& G, int g
         const uint64_t b = (uint64_t)__ldg(p.prev_idx + (G.gi - 0)) * (uint32_t)p.n_gates + (sig - (uint32_t)p.n_pi);
         counted = (__ldg(p.pois_prev + (b >> 5)) >> (b & 31u)) & 1u;
     }
-    uint8_t* oreg = G.row + (size_t)d1.x * G.stride;
+    uint8_t* oreg = grp_row(G) + (size_t)d1.x * G.stride;
     unsigned long long tb = 0;
     // spill-heap requests of the warp's gates: one bump allocation per warp
     const bool want = active && U < OFF_LIMIT && U > (uint32_t)p.W;
@@ -437,7 +448,7 @@ __device__ __forceinline__ int phase_a(const SweepParams& p, const Grp& G, int g
         }
     }
     if (on && !active) {                      // finished here: constant output, or poisoned
-        __stcg(G.rec + (size_t)d1.x * G.rstride, make_uint4(y0, 0u, 0u, pois ? REC_POISON : 0u));
+        __stcg(grp_rec(G) + (size_t)d1.x * G.rstride, make_uint4(y0, 0u, 0u, pois ? REC_POISON : 0u));
         if (pois) {
             if (!RERUN || counted) poison_bit(p, G.gi, sig);
             if (own) p.ovf[G.gi] = 1;
@@ -458,7 +469,7 @@ __device__ __forceinline__ int phase_a(const SweepParams& p, const Grp& G, int g
             unsigned long long itb = reinterpret_cast<unsigned long long>(p.zero);
             unsigned long long eb = reinterpret_cast<unsigned long long>(p.pi_ents);
             if ((uint32_t)q < K && (loc[q] & LOC_KIND) != LOC_PI) {
-                const uint8_t* r = G.row + (size_t)(loc[q] & LOC_ID) * G.stride;
+                const uint8_t* r = grp_row(G) + (size_t)(loc[q] & LOC_ID) * G.stride;
                 eb = reinterpret_cast<unsigned long long>(r);
                 itb = (M[q] & REC_SPILL) ? __ldcg(reinterpret_cast<const unsigned long long*>(r + REG_SPILLPTR))
                                          : reinterpret_cast<unsigned long long>(r + times_off(AQ[q]));
@@ -612,8 +623,7 @@ __device__ __forceinline__ uint32_t merge_four(const SweepParams& p, const float
 // with alike event counts): merge, outputs, entries, activity and the
 // gate's record, all in registers.
 template <bool RERUN>
-__device__ __forceinline__ void phase_b(const SweepParams& p, const Grp& G, int nq, uint32_t q_s, int lane,
-                                        unsigned long long& enc) {
+__device__ __forceinline__ void phase_b(const SweepParams& p, const Grp& G, int nq, uint32_t q_s, int lane) {
     const uint32_t lmask = (1u << lane) - 1u;
     const int krel = G.krel;
     for (int e = 0; e < nq; ++e) {
@@ -706,7 +716,7 @@ __device__ __forceinline__ void phase_b(const SweepParams& p, const Grp& G, int 
         // (reading C15, counted once per slot group across rerun rounds),
         // latest PO arrival
         if (v) {
-            uint32_t* oent = reinterpret_cast<uint32_t*>(G.row + (size_t)w0.z * G.stride);
+            uint32_t* oent = reinterpret_cast<uint32_t*>(grp_row(G) + (size_t)w0.z * G.stride);
             __stcg(oent + __popc(A & lmask), min(n_out, ENT_N) | (off << ENT_OFF_SHIFT));
             if (n_out && (w0.x & (1u << 24)))
                 atomicMax(p.latest + p.box.k0 + krel, __float_as_uint(__ldcg(out + n_out - 1)));
@@ -720,12 +730,12 @@ __device__ __forceinline__ void phase_b(const SweepParams& p, const Grp& G, int 
             atomicAdd(p.act + (size_t)w0.y * (uint32_t)p.n_vdd + (uint32_t)(p.box.k0 + krel), (unsigned long long)n_out);
         if (lane == 0) {
             const uint32_t meta = pois ? REC_POISON : (tot | ((fl & QF_SPILL) ? REC_SPILL : 0u));
-            __stcg(G.rec + (size_t)w0.z * G.rstride, make_uint4(w0.w, pois ? 0u : Eo, pois ? 0u : A, meta));
+            __stcg(grp_rec(G) + (size_t)w0.z * G.rstride, make_uint4(w0.w, pois ? 0u : Eo, pois ? 0u : A, meta));
             if (pois) {
                 if (!RERUN || counted) poison_bit(p, G.gi, w0.y);
                 if (fl & QF_OWN) p.ovf[G.gi] = 1;
             } else {
-                enc += (unsigned long long)(1u + (fl >> 8)) * (unsigned long long)__popc(Eo);
+                sts_u64(G.ws, lds_u64(G.ws) + (unsigned long long)(1u + (fl >> 8)) * (unsigned long long)__popc(Eo));
             }
         }
         PROF_ACC(4);
@@ -746,8 +756,9 @@ __global__ void __launch_bounds__(AVFS_SWEEP_THREADS, 1) sweep_kernel(const Swee
     const int GP = SPLIT ? 1 : p.grp_per_cta, wpg = nw / GP, S = SPLIT ? p.split : 1;
     const int sg = warp / wpg, wl = warp % wpg;
     const uint32_t ctr_s = base_s + 8u * (uint32_t)sg;        // this group's level counters
-    unsigned long long enc = 0;
     Grp G;
+    G.ws = base_s + 4u * (uint32_t)(2 * 32 + 4 + warp * WARP_INFO_WORDS);
+    if (lane == 0) sts_u64(G.ws, 0ull);                  // encoding units of this warp
     const int64_t u_end = SPLIT ? p.n_sw * S : p.n_sw;
     const int64_t u_step = SPLIT ? (int64_t)gridDim.x : (int64_t)gridDim.x * GP;
     for (int64_t u = SPLIT ? (int64_t)blockIdx.x : (int64_t)blockIdx.x * GP; u < u_end; u += u_step) {
@@ -804,7 +815,7 @@ __global__ void __launch_bounds__(AVFS_SWEEP_THREADS, 1) sweep_kernel(const Swee
                     PROF_T0();
                     const int nq = phase_a<RERUN>(p, G, ls + (int)gb, nb, q_s, lane);
                     PROF_ACC(1);
-                    if (nq) phase_b<RERUN>(p, G, nq, q_s, lane, enc);
+                    if (nq) phase_b<RERUN>(p, G, nq, q_s, lane);
                     PROF_ACC(5);
                 }
             }
@@ -832,7 +843,10 @@ __global__ void __launch_bounds__(AVFS_SWEEP_THREADS, 1) sweep_kernel(const Swee
             PROF_ACC(6);
         }
     }
-    if (enc) atomicAdd(p.enc_units, enc);
+    if (lane == 0) {
+        const unsigned long long enc = lds_u64(G.ws);
+        if (enc) atomicAdd(p.enc_units, enc);
+    }
 }
 
 int debug_phase_cycles(unsigned long long* out, int reset) {
