@@ -221,24 +221,34 @@ enum : int {
 };
 constexpr uint32_t QF_POISON = 1u, QF_COUNT = 2u, QF_OWN = 4u, QF_SPILL = 8u;
 constexpr int WARP_SMEM_WORDS = QN * QW;
-constexpr int WARP_INFO_WORDS = 8;                   // per warp: enc u64, group's region row u64, record row u64
+constexpr int WARP_INFO_WORDS = 16;  // per warp: enc, region row, record row, gi, sw (u64 each), vmask
 constexpr int CTA_HDR_WORDS = 2 * 32 + 4 + 32 * WARP_INFO_WORDS;   // level counters [group][2], pad, warp info
 
 // A warp's slot group.  Its region and record rows (64-bit pointers) are
 // kept in the warp's shared info block and loaded where used (ws), not held
 // in registers through the sweep's loops.
 struct Grp {
-    uint32_t ws;           // shared address of the warp info: +0 enc, +8 region row, +16 record row
-    uint32_t stride;       // bytes between arena buffers (pin_n_sw * region_bytes < 4 GiB, host-checked)
-    uint32_t rstride;      // records between buffers (pin_n_sw)
-    int64_t gi;            // group index in the round
-    int64_t sw;            // slot group in the box
+    uint32_t ws;           // shared address of the warp info: +0 enc, +8 region row, +16 record row,
+                           // +24 group index in the round, +32 slot group in the box, +40 vmask
     int krel;              // this lane's operating point - box.k0
-    uint32_t vmask;        // slots of the group inside the simulated range
 };
 
 __device__ __forceinline__ uint8_t* grp_row(const Grp& G) { return reinterpret_cast<uint8_t*>(lds_u64(G.ws + 8)); }
 __device__ __forceinline__ uint4* grp_rec(const Grp& G) { return reinterpret_cast<uint4*>(lds_u64(G.ws + 16)); }
+__device__ __forceinline__ int64_t grp_gi(const Grp& G) { return (int64_t)lds_u64(G.ws + 24); }
+__device__ __forceinline__ int64_t grp_sw(const Grp& G) { return (int64_t)lds_u64(G.ws + 32); }
+__device__ __forceinline__ uint32_t grp_vmask(const Grp& G) { return lds_u32(G.ws + 40); }
+// bytes between a group's arena buffers / records between its buffers
+#if AVFS_REG_GROUP_MAJOR
+#define GRP_STRIDE(p) ((uint32_t)(p).region_bytes)
+#else
+#define GRP_STRIDE(p) ((uint32_t)((p).pin_n_sw * (p).region_bytes))
+#endif
+#if AVFS_REC_GROUP_MAJOR
+#define GRP_RSTRIDE(p) 1u
+#else
+#define GRP_RSTRIDE(p) ((uint32_t)(p).pin_n_sw)
+#endif
 
 // lane's slot of group sw in the box (SlotBox, avfs_internal.h): pair j,
 // operating point k; false outside the box or the simulated range
@@ -256,37 +266,29 @@ __device__ __forceinline__ bool box_slot(const SlotBox& b, int64_t sw, int lane,
 
 __device__ __forceinline__ void group_setup(const SweepParams& p, int64_t i, int lane, Grp& G) {
     const int64_t sw = p.sw_list ? (int64_t)p.sw_list[i] : p.sw_first + i;
-    G.sw = sw;
-    G.gi = p.i_base + i;
+    const int64_t gi = p.i_base + i;
 #if AVFS_REG_GROUP_MAJOR
-    uint8_t* row = p.arena + G.gi * p.n_buf * p.region_bytes;
+    uint8_t* row = p.arena + gi * p.n_buf * p.region_bytes;
 #else
-    uint8_t* row = p.arena + G.gi * p.region_bytes;
+    uint8_t* row = p.arena + gi * p.region_bytes;
 #endif
 #if AVFS_REC_GROUP_MAJOR
-    uint4* rec = p.recs + G.gi * (int64_t)p.n_buf;
+    uint4* rec = p.recs + gi * (int64_t)p.n_buf;
 #else
-    uint4* rec = p.recs + G.gi;
-#endif
-    if (lane == 0) {
-        sts_u64(G.ws + 8, reinterpret_cast<unsigned long long>(row));
-        sts_u64(G.ws + 16, reinterpret_cast<unsigned long long>(rec));
-    }
-    __syncwarp();
-#if AVFS_REG_GROUP_MAJOR
-    G.stride = (uint32_t)p.region_bytes;
-#else
-    G.stride = (uint32_t)(p.pin_n_sw * p.region_bytes);
-#endif
-#if AVFS_REC_GROUP_MAJOR
-    G.rstride = 1u;
-#else
-    G.rstride = (uint32_t)p.pin_n_sw;
+    uint4* rec = p.recs + gi;
 #endif
     int64_t j;
     int k;
-    G.vmask = __ballot_sync(FULL, box_slot(p.box, sw, lane, j, k));
+    const uint32_t vmask = __ballot_sync(FULL, box_slot(p.box, sw, lane, j, k));
     G.krel = k - p.box.k0;
+    if (lane == 0) {
+        sts_u64(G.ws + 8, reinterpret_cast<unsigned long long>(row));
+        sts_u64(G.ws + 16, reinterpret_cast<unsigned long long>(rec));
+        sts_u64(G.ws + 24, (unsigned long long)gi);
+        sts_u64(G.ws + 32, (unsigned long long)sw);
+        sts_u32(G.ws + 40, vmask);
+    }
+    __syncwarp();
 }
 
 // all-ones iff truth-table bit b is set
@@ -386,13 +388,13 @@ __device__ __forceinline__ int phase_a(const SweepParams& p, const Grp& G, int g
         if ((uint32_t)q < K) {
             const uint32_t id = loc[q] & LOC_ID;
             if ((loc[q] & LOC_KIND) == LOC_PI) {       // reading C2: one event at t = 0 iff p1 != p2
-                const int64_t ix = (int64_t)id * p.n_grp + G.sw;
+                const int64_t ix = (int64_t)id * p.n_grp + grp_sw(G);
                 const uint32_t w1 = __ldg(p.p1g + ix), w2 = __ldg(p.p2g + ix);
                 X[q] = w1;
-                E[q] = AQ[q] = (w1 ^ w2) & G.vmask;
+                E[q] = AQ[q] = (w1 ^ w2) & grp_vmask(G);
                 M[q] = (uint32_t)__popc(E[q]);
             } else {
-                const uint4 r = __ldcg(grp_rec(G) + (size_t)id * G.rstride);
+                const uint4 r = __ldcg(grp_rec(G) + (size_t)id * GRP_RSTRIDE(p));
                 X[q] = r.x;
                 E[q] = r.y;
                 AQ[q] = r.z;
@@ -410,10 +412,10 @@ __device__ __forceinline__ int phase_a(const SweepParams& p, const Grp& G, int g
     bool counted = true;                      // activity of this (group, gate) not yet counted
     const uint32_t sig = d1.y;
     if (RERUN && on) {
-        const uint64_t b = (uint64_t)__ldg(p.prev_idx + (G.gi - 0)) * (uint32_t)p.n_gates + (sig - (uint32_t)p.n_pi);
+        const uint64_t b = (uint64_t)__ldg(p.prev_idx + grp_gi(G)) * (uint32_t)p.n_gates + (sig - (uint32_t)p.n_pi);
         counted = (__ldg(p.pois_prev + (b >> 5)) >> (b & 31u)) & 1u;
     }
-    uint8_t* oreg = grp_row(G) + (size_t)d1.x * G.stride;
+    uint8_t* oreg = grp_row(G) + (size_t)d1.x * GRP_STRIDE(p);
     unsigned long long tb = 0;
     // spill-heap requests of the warp's gates: one bump allocation per warp
     const bool want = active && U < OFF_LIMIT && U > (uint32_t)p.W;
@@ -448,10 +450,10 @@ __device__ __forceinline__ int phase_a(const SweepParams& p, const Grp& G, int g
         }
     }
     if (on && !active) {                      // finished here: constant output, or poisoned
-        __stcg(grp_rec(G) + (size_t)d1.x * G.rstride, make_uint4(y0, 0u, 0u, pois ? REC_POISON : 0u));
+        __stcg(grp_rec(G) + (size_t)d1.x * GRP_RSTRIDE(p), make_uint4(y0, 0u, 0u, pois ? REC_POISON : 0u));
         if (pois) {
-            if (!RERUN || counted) poison_bit(p, G.gi, sig);
-            if (own) p.ovf[G.gi] = 1;
+            if (!RERUN || counted) poison_bit(p, grp_gi(G), sig);
+            if (own) p.ovf[grp_gi(G)] = 1;
         }
     }
     const uint32_t bal = __ballot_sync(FULL, active);
@@ -469,7 +471,7 @@ __device__ __forceinline__ int phase_a(const SweepParams& p, const Grp& G, int g
             unsigned long long itb = reinterpret_cast<unsigned long long>(p.zero);
             unsigned long long eb = reinterpret_cast<unsigned long long>(p.pi_ents);
             if ((uint32_t)q < K && (loc[q] & LOC_KIND) != LOC_PI) {
-                const uint8_t* r = grp_row(G) + (size_t)(loc[q] & LOC_ID) * G.stride;
+                const uint8_t* r = grp_row(G) + (size_t)(loc[q] & LOC_ID) * GRP_STRIDE(p);
                 eb = reinterpret_cast<unsigned long long>(r);
                 itb = (M[q] & REC_SPILL) ? __ldcg(reinterpret_cast<const unsigned long long*>(r + REG_SPILLPTR))
                                          : reinterpret_cast<unsigned long long>(r + times_off(AQ[q]));
@@ -716,7 +718,7 @@ __device__ __forceinline__ void phase_b(const SweepParams& p, const Grp& G, int 
         // (reading C15, counted once per slot group across rerun rounds),
         // latest PO arrival
         if (v) {
-            uint32_t* oent = reinterpret_cast<uint32_t*>(grp_row(G) + (size_t)w0.z * G.stride);
+            uint32_t* oent = reinterpret_cast<uint32_t*>(grp_row(G) + (size_t)w0.z * GRP_STRIDE(p));
             __stcg(oent + __popc(A & lmask), min(n_out, ENT_N) | (off << ENT_OFF_SHIFT));
             if (n_out && (w0.x & (1u << 24)))
                 atomicMax(p.latest + p.box.k0 + krel, __float_as_uint(__ldcg(out + n_out - 1)));
@@ -730,10 +732,10 @@ __device__ __forceinline__ void phase_b(const SweepParams& p, const Grp& G, int 
             atomicAdd(p.act + (size_t)w0.y * (uint32_t)p.n_vdd + (uint32_t)(p.box.k0 + krel), (unsigned long long)n_out);
         if (lane == 0) {
             const uint32_t meta = pois ? REC_POISON : (tot | ((fl & QF_SPILL) ? REC_SPILL : 0u));
-            __stcg(grp_rec(G) + (size_t)w0.z * G.rstride, make_uint4(w0.w, pois ? 0u : Eo, pois ? 0u : A, meta));
+            __stcg(grp_rec(G) + (size_t)w0.z * GRP_RSTRIDE(p), make_uint4(w0.w, pois ? 0u : Eo, pois ? 0u : A, meta));
             if (pois) {
-                if (!RERUN || counted) poison_bit(p, G.gi, w0.y);
-                if (fl & QF_OWN) p.ovf[G.gi] = 1;
+                if (!RERUN || counted) poison_bit(p, grp_gi(G), w0.y);
+                if (fl & QF_OWN) p.ovf[grp_gi(G)] = 1;
             } else {
                 sts_u64(G.ws, lds_u64(G.ws) + (unsigned long long)(1u + (fl >> 8)) * (unsigned long long)__popc(Eo));
             }
