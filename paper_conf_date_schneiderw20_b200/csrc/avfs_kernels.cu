@@ -747,7 +747,7 @@ __device__ __forceinline__ void phase_b(const SweepParams& p, const Grp& G, int 
 
 
 template <bool SPLIT, bool RERUN>
-__global__ void __launch_bounds__(AVFS_SWEEP_THREADS, 1) sweep_kernel(const SweepParams p) {
+__global__ void __launch_bounds__(AVFS_SWEEP_THREADS, AVFS_SWEEP_MINB) sweep_kernel(const SweepParams p) {
     extern __shared__ __align__(16) uint32_t smem_w[];
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nw = blockDim.x >> 5;
     const uint32_t base_s = smem_u32(smem_w);
