@@ -209,6 +209,9 @@ __device__ unsigned long long g_phase_cycles[16];
 #ifndef AVFS_QN
 #define AVFS_QN 32
 #endif
+#ifndef AVFS_TAIL_SPLIT
+#define AVFS_TAIL_SPLIT 1
+#endif
 constexpr int QN = AVFS_QN;            // gates per batch (Phase A lanes, queue entries)
 constexpr int QW = 40;                 // words per queue entry
 enum : int {
@@ -809,8 +812,22 @@ __global__ void __launch_bounds__(AVFS_SWEEP_THREADS, AVFS_SWEEP_MINB) sweep_ker
                         bsz = (int)(gb >> 24);
                         gb &= 0xFFFFFFu;
                     } else {
+#if AVFS_TAIL_SPLIT
+                        // wide levels: full batches, except that the last
+                        // round (fewer than a batch per warp left) is split
+                        // evenly over the group's warps
+                        if (lane == 0) {
+                            const int rem = nlv - (int)lds_u32(cs);
+                            const int bs = rem >= QN * wpg ? QN : max(1, (rem + wpg - 1) / wpg);
+                            gb = atoms_add(cs, (uint32_t)bs) | ((uint32_t)bs << 24);
+                        }
+                        gb = __shfl_sync(FULL, gb, 0);
+                        bsz = (int)(gb >> 24);
+                        gb &= 0xFFFFFFu;
+#else
                         if (lane == 0) gb = atoms_add(cs, QN);
                         gb = __shfl_sync(FULL, gb, 0);
+#endif
                     }
                     if ((int)gb >= nlv) break;
                     const int nb = min(bsz, nlv - (int)gb);
