@@ -223,24 +223,27 @@ enum : int {
     Q_ITB = 32                                      // 4 x u64 time bases of the inputs
 };
 constexpr uint32_t QF_POISON = 1u, QF_COUNT = 2u, QF_OWN = 4u, QF_SPILL = 8u;
-constexpr int WARP_SMEM_WORDS = QN * QW;
-constexpr int WARP_INFO_WORDS = 16;  // per warp: enc, region row, record row, gi, sw (u64 each), vmask
-constexpr int CTA_HDR_WORDS = 2 * 32 + 4 + 32 * WARP_INFO_WORDS;   // level counters [group][2], pad, warp info
+constexpr int WARP_INFO_WORDS = 16;  // per warp, after its queue: enc, region row, record row, gi, sw (u64 each), vmask
+constexpr int WARP_SMEM_WORDS = QN * QW + WARP_INFO_WORDS;
+constexpr uint32_t WS_OFF = 4u * QN * QW;          // byte offset of the warp info block from the warp's queue
+constexpr int CTA_HDR_WORDS = 2 * 32 + 4;                          // level counters [group][2], pad
 
 // A warp's slot group.  Its region and record rows (64-bit pointers) are
 // kept in the warp's shared info block and loaded where used (ws), not held
 // in registers through the sweep's loops.
+// (warp info block at q_s + WS_OFF: +0 enc, +8 region row, +16 record row,
+// +24 group index in the round, +32 slot group in the box, +40 vmask; at a
+// constant offset from the warp's queue, so its loads need no address math)
 struct Grp {
-    uint32_t ws;           // shared address of the warp info: +0 enc, +8 region row, +16 record row,
-                           // +24 group index in the round, +32 slot group in the box, +40 vmask
+    uint32_t q;            // the warp's queue (shared address)
     int krel;              // this lane's operating point - box.k0
 };
 
-__device__ __forceinline__ uint8_t* grp_row(const Grp& G) { return reinterpret_cast<uint8_t*>(lds_u64(G.ws + 8)); }
-__device__ __forceinline__ uint4* grp_rec(const Grp& G) { return reinterpret_cast<uint4*>(lds_u64(G.ws + 16)); }
-__device__ __forceinline__ int64_t grp_gi(const Grp& G) { return (int64_t)lds_u64(G.ws + 24); }
-__device__ __forceinline__ int64_t grp_sw(const Grp& G) { return (int64_t)lds_u64(G.ws + 32); }
-__device__ __forceinline__ uint32_t grp_vmask(const Grp& G) { return lds_u32(G.ws + 40); }
+__device__ __forceinline__ uint8_t* grp_row(const Grp& G) { return reinterpret_cast<uint8_t*>(lds_u64(G.q + WS_OFF + 8)); }
+__device__ __forceinline__ uint4* grp_rec(const Grp& G) { return reinterpret_cast<uint4*>(lds_u64(G.q + WS_OFF + 16)); }
+__device__ __forceinline__ int64_t grp_gi(const Grp& G) { return (int64_t)lds_u64(G.q + WS_OFF + 24); }
+__device__ __forceinline__ int64_t grp_sw(const Grp& G) { return (int64_t)lds_u64(G.q + WS_OFF + 32); }
+__device__ __forceinline__ uint32_t grp_vmask(const Grp& G) { return lds_u32(G.q + WS_OFF + 40); }
 // bytes between a group's arena buffers / records between its buffers
 #if AVFS_REG_GROUP_MAJOR
 #define GRP_STRIDE(p) ((uint32_t)(p).region_bytes)
@@ -285,11 +288,11 @@ __device__ __forceinline__ void group_setup(const SweepParams& p, int64_t i, int
     const uint32_t vmask = __ballot_sync(FULL, box_slot(p.box, sw, lane, j, k));
     G.krel = k - p.box.k0;
     if (lane == 0) {
-        sts_u64(G.ws + 8, reinterpret_cast<unsigned long long>(row));
-        sts_u64(G.ws + 16, reinterpret_cast<unsigned long long>(rec));
-        sts_u64(G.ws + 24, (unsigned long long)gi);
-        sts_u64(G.ws + 32, (unsigned long long)sw);
-        sts_u32(G.ws + 40, vmask);
+        sts_u64(G.q + WS_OFF + 8, reinterpret_cast<unsigned long long>(row));
+        sts_u64(G.q + WS_OFF + 16, reinterpret_cast<unsigned long long>(rec));
+        sts_u64(G.q + WS_OFF + 24, (unsigned long long)gi);
+        sts_u64(G.q + WS_OFF + 32, (unsigned long long)sw);
+        sts_u32(G.q + WS_OFF + 40, vmask);
     }
     __syncwarp();
 }
@@ -571,9 +574,10 @@ __device__ __noinline__ float sweep_delay(const DelayDesc* __restrict__ dd, cons
 }
 
 // Delay of arc e = 2 pin + pol of a queued gate at slot operating point
-// k0 + krel: the table entry [gate][pin][krel][pol], or evaluated here.
+// k0 + krel: the table entry [gate][pin][krel][pol] (DT), or evaluated here.
+template <bool DT>
 __device__ __forceinline__ float item_delay(const SweepParams& p, uint32_t gate, int krel, int e) {
-    if (p.dtab) return __ldg(p.dtab + (((size_t)gate * 4 + (e >> 1)) * (uint32_t)p.box.nk + krel) * 2 + (e & 1));
+    if (DT) return __ldg(p.dtab + (((size_t)gate * 4 + (e >> 1)) * (uint32_t)p.box.nk + krel) * 2 + (e & 1));
     const DelayParams& P = p.dp;
     return sweep_delay(P.dd, P.coef, P.vdd, P.n_isl, P.deg_v, P.deg_c, P.v_min, P.v_max, P.quantum, P.err, gate,
                        p.box.k0 + krel, e);
@@ -581,6 +585,7 @@ __device__ __forceinline__ float item_delay(const SweepParams& p, uint32_t gate,
 
 // Merge of up to four sorted lists (list q = pin q, n[q] = 0 if unused);
 // delays from the table (or evaluated) per step.
+template <bool DT>
 __device__ __forceinline__ uint32_t merge_four(const SweepParams& p, const float* const (&a_in)[4], const int (&n_in)[4],
                                                uint32_t bits, uint32_t proj, uint32_t tt, uint32_t gate, int krel,
                                                float* out, uint32_t steps) {
@@ -618,7 +623,7 @@ __device__ __forceinline__ uint32_t merge_four(const SweepParams& p, const float
         const bool live = t < AVFS_INF;
         bits ^= live ? (1u << pm) : 0u;
         const uint32_t y = (tt >> bits) & 1u;
-        F.step(t, live, y, live ? item_delay(p, gate, krel, 2 * pm + (int)y) : 1.0f, out);
+        F.step(t, live, y, live ? item_delay<DT>(p, gate, krel, 2 * pm + (int)y) : 1.0f, out);
     }
     return F.cnt;
 }
@@ -627,7 +632,7 @@ __device__ __forceinline__ uint32_t merge_four(const SweepParams& p, const float
 // gate's observable slots are mostly all 32 operating points of one pair,
 // with alike event counts): merge, outputs, entries, activity and the
 // gate's record, all in registers.
-template <bool RERUN>
+template <bool RERUN, bool DT>
 __device__ __forceinline__ void phase_b(const SweepParams& p, const Grp& G, int nq, uint32_t q_s, int lane) {
     const uint32_t lmask = (1u << lane) - 1u;
     const int krel = G.krel;
@@ -662,16 +667,16 @@ __device__ __forceinline__ void phase_b(const SweepParams& p, const Grp& G, int 
         const uint32_t gate = lds_u32(qe + 4 * Q_GATE);
         float4 dl = make_float4(1.0f, 1.0f, 1.0f, 1.0f);
         if (use && !many) {
-            if (p.dtab) {                              // (fall, rise) of each pin: one 8-B load
+            if (DT) {                                  // (fall, rise) of each pin: one 8-B load
                 const float2* db = reinterpret_cast<const float2*>(p.dtab) + (size_t)gate * 4u * (uint32_t)p.box.nk + krel;
                 const float2 d0 = __ldg(db + (uint32_t)p0 * (uint32_t)p.box.nk);
                 const float2 d1 = __ldg(db + (uint32_t)p1 * (uint32_t)p.box.nk);
                 dl = make_float4(d0.x, d0.y, d1.x, d1.y);
             } else {
-                dl.x = item_delay(p, gate, krel, 2 * p0);
-                dl.y = item_delay(p, gate, krel, 2 * p0 + 1);
-                dl.z = item_delay(p, gate, krel, 2 * p1);
-                dl.w = item_delay(p, gate, krel, 2 * p1 + 1);
+                dl.x = item_delay<DT>(p, gate, krel, 2 * p0);
+                dl.y = item_delay<DT>(p, gate, krel, 2 * p0 + 1);
+                dl.z = item_delay<DT>(p, gate, krel, 2 * p1);
+                dl.w = item_delay<DT>(p, gate, krel, 2 * p1 + 1);
             }
         }
         const int n0 = (int)(e0 & ENT_N), n1 = (int)(e1 & ENT_N);
@@ -711,7 +716,7 @@ __device__ __forceinline__ void phase_b(const SweepParams& p, const Grp& G, int 
                     nn[q] = (q == p0) ? n0 : ((q == p1 && rest) ? n1 : 0);
                 }
             }
-            n_out = merge_four(p, ap, nn, bits, y0, tt, gate, krel, out, steps);
+            n_out = merge_four<DT>(p, ap, nn, bits, y0, tt, gate, krel, out, steps);
         } else {
             n_out = merge_two(a0, n0, a1, rest ? n1 : 0, bits, 1u << p0, rest ? 1u << p1 : 0u, y0, tt, dl, out, steps);
         }
@@ -740,7 +745,7 @@ __device__ __forceinline__ void phase_b(const SweepParams& p, const Grp& G, int 
                 if (!RERUN || counted) poison_bit(p, grp_gi(G), w0.y);
                 if (fl & QF_OWN) p.ovf[grp_gi(G)] = 1;
             } else {
-                sts_u64(G.ws, lds_u64(G.ws) + (unsigned long long)(1u + (fl >> 8)) * (unsigned long long)__popc(Eo));
+                sts_u64(G.q + WS_OFF, lds_u64(G.q + WS_OFF) + (unsigned long long)(1u + (fl >> 8)) * (unsigned long long)__popc(Eo));
             }
         }
         PROF_ACC(4);
@@ -749,7 +754,7 @@ __device__ __forceinline__ void phase_b(const SweepParams& p, const Grp& G, int 
 }
 
 
-template <bool SPLIT, bool RERUN>
+template <bool SPLIT, bool RERUN, bool DT>
 __global__ void __launch_bounds__(AVFS_SWEEP_THREADS, AVFS_SWEEP_MINB) sweep_kernel(const SweepParams p) {
     extern __shared__ __align__(16) uint32_t smem_w[];
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nw = blockDim.x >> 5;
@@ -762,8 +767,8 @@ __global__ void __launch_bounds__(AVFS_SWEEP_THREADS, AVFS_SWEEP_MINB) sweep_ker
     const int sg = warp / wpg, wl = warp % wpg;
     const uint32_t ctr_s = base_s + 8u * (uint32_t)sg;        // this group's level counters
     Grp G;
-    G.ws = base_s + 4u * (uint32_t)(2 * 32 + 4 + warp * WARP_INFO_WORDS);
-    if (lane == 0) sts_u64(G.ws, 0ull);                  // encoding units of this warp
+    G.q = q_s;
+    if (lane == 0) sts_u64(q_s + WS_OFF, 0ull);           // encoding units of this warp
     const int64_t u_end = SPLIT ? p.n_sw * S : p.n_sw;
     const int64_t u_step = SPLIT ? (int64_t)gridDim.x : (int64_t)gridDim.x * GP;
     for (int64_t u = SPLIT ? (int64_t)blockIdx.x : (int64_t)blockIdx.x * GP; u < u_end; u += u_step) {
@@ -834,7 +839,7 @@ __global__ void __launch_bounds__(AVFS_SWEEP_THREADS, AVFS_SWEEP_MINB) sweep_ker
                     PROF_T0();
                     const int nq = phase_a<RERUN>(p, G, ls + (int)gb, nb, q_s, lane);
                     PROF_ACC(1);
-                    if (nq) phase_b<RERUN>(p, G, nq, q_s, lane);
+                    if (nq) phase_b<RERUN, DT>(p, G, nq, q_s, lane);
                     PROF_ACC(5);
                 }
             }
@@ -863,7 +868,7 @@ __global__ void __launch_bounds__(AVFS_SWEEP_THREADS, AVFS_SWEEP_MINB) sweep_ker
         }
     }
     if (lane == 0) {
-        const unsigned long long enc = lds_u64(G.ws);
+        const unsigned long long enc = lds_u64(q_s + WS_OFF);
         if (enc) atomicAdd(p.enc_units, enc);
     }
 }
@@ -885,11 +890,15 @@ int debug_phase_cycles(unsigned long long* out, int reset) {
 
 int sweep_smem_bytes(int warps_per_cta, int) { return 4 * (CTA_HDR_WORDS + warps_per_cta * WARP_SMEM_WORDS); }
 
+// the sweep instantiations: (split group, rerun round, delay table)
 template <bool SPLIT, bool RERUN>
-static cudaError_t occ_one(int warps_per_cta, int smem, int* b) {
-    cudaError_t e = cudaFuncSetAttribute(sweep_kernel<SPLIT, RERUN>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
-    if (e == cudaSuccess) e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(b, sweep_kernel<SPLIT, RERUN>, warps_per_cta * 32, smem);
-    return e;
+static const void* sweep_fn(bool dt) {
+    return dt ? reinterpret_cast<const void*>(sweep_kernel<SPLIT, RERUN, true>)
+              : reinterpret_cast<const void*>(sweep_kernel<SPLIT, RERUN, false>);
+}
+static const void* sweep_fn(bool split, bool rerun, bool dt) {
+    return split ? (rerun ? sweep_fn<true, true>(dt) : sweep_fn<true, false>(dt))
+                 : (rerun ? sweep_fn<false, true>(dt) : sweep_fn<false, false>(dt));
 }
 
 cudaError_t sweep_occupancy(int warps_per_cta, int smem, int* blocks_per_sm) {
@@ -902,13 +911,15 @@ cudaError_t sweep_occupancy(int warps_per_cta, int smem, int* blocks_per_sm) {
         *blocks_per_sm = c_bps;
         return cudaSuccess;
     }
-    int b[4] = {0, 0, 0, 0};
-    cudaError_t e = occ_one<false, false>(warps_per_cta, smem, b + 0);
-    if (e == cudaSuccess) e = occ_one<true, false>(warps_per_cta, smem, b + 1);
-    if (e == cudaSuccess) e = occ_one<false, true>(warps_per_cta, smem, b + 2);
-    if (e == cudaSuccess) e = occ_one<true, true>(warps_per_cta, smem, b + 3);
-    int m = b[0];
-    for (int k = 1; k < 4; ++k) m = b[k] < m ? b[k] : m;    // split groups need every CTA resident
+    int m = 1 << 30;
+    cudaError_t e = cudaSuccess;
+    for (int v = 0; v < 8 && e == cudaSuccess; ++v) {          // split groups need every CTA resident
+        const void* f = sweep_fn(v & 1, (v >> 1) & 1, (v >> 2) & 1);
+        int b = 0;
+        e = cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+        if (e == cudaSuccess) e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, f, warps_per_cta * 32, smem);
+        m = b < m ? b : m;
+    }
     *blocks_per_sm = m;
     if (e == cudaSuccess) {
         c_dev = dev;
@@ -921,18 +932,13 @@ cudaError_t sweep_occupancy(int warps_per_cta, int smem, int* blocks_per_sm) {
 
 cudaError_t launch_sweep(const SweepParams& p, bool rerun, int grid, int warps_per_cta, cudaStream_t st) {
     const int smem = sweep_smem_bytes(warps_per_cta, p.grp_per_cta);
-    if (p.split > 1) {
-        // the parts of a slot group wait for each other: a cooperative launch
-        // guarantees that every CTA of the grid is resident (or fails)
-        SweepParams q = p;
-        void* args[] = {&q};
-        const void* f = rerun ? reinterpret_cast<const void*>(sweep_kernel<true, true>)
-                              : reinterpret_cast<const void*>(sweep_kernel<true, false>);
-        return cudaLaunchCooperativeKernel(f, dim3(grid), dim3(warps_per_cta * 32), args, (size_t)smem, st);
-    }
-    if (rerun) sweep_kernel<false, true><<<grid, warps_per_cta * 32, smem, st>>>(p);
-    else sweep_kernel<false, false><<<grid, warps_per_cta * 32, smem, st>>>(p);
-    return cudaGetLastError();
+    SweepParams q = p;
+    void* args[] = {&q};
+    const void* f = sweep_fn(p.split > 1, rerun, p.dtab != nullptr);
+    // the parts of a split slot group wait for each other: a cooperative
+    // launch guarantees that every CTA of the grid is resident (or fails)
+    if (p.split > 1) return cudaLaunchCooperativeKernel(f, dim3(grid), dim3(warps_per_cta * 32), args, (size_t)smem, st);
+    return cudaLaunchKernel(f, dim3(grid), dim3(warps_per_cta * 32), args, (size_t)smem, st);
 }
 
 // ---------------------------------------------------------------------------
