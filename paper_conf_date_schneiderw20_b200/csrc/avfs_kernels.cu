@@ -513,6 +513,9 @@ struct Filt {
 #ifndef AVFS_LOOKAHEAD
 #define AVFS_LOOKAHEAD 3
 #endif
+#ifndef AVFS_MERGE_IDX
+#define AVFS_MERGE_IDX 1
+#endif
 __device__ __forceinline__ uint32_t merge_two(const float* a0, int n0, const float* a1, int n1, uint32_t bits,
                                               uint32_t tm0, uint32_t tm1, uint32_t proj, uint32_t tt, float4 dl,
                                               float* out, uint32_t steps) {
@@ -527,6 +530,34 @@ __device__ __forceinline__ uint32_t merge_two(const float* a0, int n0, const flo
         w0[i] = n0 > i ? ld_f32(a0 + i) : AVFS_INF;
         w1[i] = n1 > i ? ld_f32(a1 + i) : AVFS_INF;
     }
+#if AVFS_MERGE_IDX
+    // list positions as 32-bit indices (next element to load) against fixed
+    // bases and counts: one address multiply-add per refill, no 64-bit
+    // pointer updates
+    uint32_t i0 = D, i1 = D;
+    Filt F{proj, 0u, -AVFS_INF};
+#pragma unroll 1
+    for (uint32_t it = 0; it < steps; ++it) {
+        const bool p = w1[0] < w0[0];                 // ties: the lower pin first (reading C5)
+        const float t = fminf(w0[0], w1[0]);
+        const uint32_t ix = p ? i1 : i0;
+        const float nx = (int)ix < (p ? n1 : n0) ? ld_f32((p ? a1 : a0) + ix) : AVFS_INF;
+#pragma unroll
+        for (int i = 0; i + 1 < D; ++i) {
+            w1[i] = p ? w1[i + 1] : w1[i];
+            w0[i] = p ? w0[i] : w0[i + 1];
+        }
+        w1[D - 1] = p ? nx : w1[D - 1];
+        w0[D - 1] = p ? w0[D - 1] : nx;
+        i1 += p ? 1u : 0u;
+        i0 += p ? 0u : 1u;
+        const bool live = t < AVFS_INF;
+        bits ^= live ? (p ? tm1 : tm0) : 0u;
+        const uint32_t y = (tt >> bits) & 1u;
+        F.step(t, live, y, p ? (y ? dl.w : dl.z) : (y ? dl.y : dl.x), out);
+    }
+    return F.cnt;
+#else
     a0 += D;
     a1 += D;
     n0 -= D;
@@ -555,6 +586,7 @@ __device__ __forceinline__ uint32_t merge_two(const float* a0, int n0, const flo
         F.step(t, live, y, p ? (y ? dl.w : dl.z) : (y ? dl.y : dl.x), out);
     }
     return F.cnt;
+#endif
 }
 
 // Delay of arc e = 2 pin + pol of sorted gate `gate` at operating point k,
