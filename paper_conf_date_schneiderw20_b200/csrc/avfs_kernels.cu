@@ -736,6 +736,7 @@ __device__ __forceinline__ void phase_b(const SweepParams& p, const Grp& G, int 
         // output offsets: exclusive prefix of the slots' input counts
         const uint32_t off = warp_incl_scan(m, lane) - m;
         const uint32_t steps = __reduce_max_sync(FULL, m);
+        const bool big = __any_sync(FULL, v && m > ENT_N);
         PROF_ACC(2);
         float* out = reinterpret_cast<float*>(lds_u64(qe + 4 * Q_TB)) + off;
         const uint32_t y0 = (w0.w >> lane) & 1u;
@@ -752,32 +753,39 @@ __device__ __forceinline__ void phase_b(const SweepParams& p, const Grp& G, int 
         } else {
             n_out = merge_two(a0, n0, a1, rest ? n1 : 0, bits, 1u << p0, rest ? 1u << p1 : 0u, y0, tt, dl, out, steps);
         }
-        if (!v) n_out = 0;
         PROF_ACC(3);
         // the gate's output: entries, record, activity per (signal, point)
         // (reading C15, counted once per slot group across rerun rounds),
-        // latest PO arrival
-        if (v) {
-            uint32_t* oent = reinterpret_cast<uint32_t*>(grp_row(G) + (size_t)w0.z * GRP_STRIDE(p));
-            __stcg(oent + __popc(A & lmask), min(n_out, ENT_N) | (off << ENT_OFF_SHIFT));
-            if (n_out && (w0.x & (1u << 24)))
-                atomicMax(p.latest + p.box.k0 + krel, __float_as_uint(__ldcg(out + n_out - 1)));
-        }
-        const bool big = __any_sync(FULL, v && m > ENT_N);
-        const uint32_t Eo = __ballot_sync(FULL, n_out != 0u);
-        const uint32_t tot = __reduce_add_sync(FULL, n_out);
-        const uint32_t fl = lds_u32(qe + 4 * Q_FLAG) | (big ? (QF_POISON | QF_OWN) : 0u);
-        const bool pois = fl & QF_POISON, counted = fl & QF_COUNT;
-        if (n_out && counted && !pois)
-            atomicAdd(p.act + (size_t)w0.y * (uint32_t)p.n_vdd + (uint32_t)(p.box.k0 + krel), (unsigned long long)n_out);
-        if (lane == 0) {
-            const uint32_t meta = pois ? REC_POISON : (tot | ((fl & QF_SPILL) ? REC_SPILL : 0u));
-            __stcg(grp_rec(G) + (size_t)w0.z * GRP_RSTRIDE(p), make_uint4(w0.w, pois ? 0u : Eo, pois ? 0u : A, meta));
-            if (pois) {
-                if (!RERUN || counted) poison_bit(p, grp_gi(G), w0.y);
-                if (fl & QF_OWN) p.ovf[grp_gi(G)] = 1;
-            } else {
-                sts_u64(G.q + WS_OFF, lds_u64(G.q + WS_OFF) + (unsigned long long)(1u + (fl >> 8)) * (unsigned long long)__popc(Eo));
+        // latest PO arrival.  The queue words are read again here
+        // rather than held in registers through the merge.
+        {
+            const uint4 w0 = lds_u32x4(qe + 4 * Q_TTK);
+            const uint32_t A = lds_u32(qe + 4 * Q_A);
+            const bool v = (A >> lane) & 1u;
+            if (!v) n_out = 0;
+            if (v) {
+                uint32_t* oent = reinterpret_cast<uint32_t*>(grp_row(G) + (size_t)w0.z * GRP_STRIDE(p));
+                __stcg(oent + __popc(A & lmask), min(n_out, ENT_N) | (off << ENT_OFF_SHIFT));
+                if (n_out && (w0.x & (1u << 24))) {
+                    const float* o = reinterpret_cast<const float*>(lds_u64(qe + 4 * Q_TB)) + off;
+                    atomicMax(p.latest + p.box.k0 + krel, __float_as_uint(__ldcg(o + n_out - 1)));
+                }
+            }
+            const uint32_t Eo = __ballot_sync(FULL, n_out != 0u);
+            const uint32_t tot = __reduce_add_sync(FULL, n_out);
+            const uint32_t fl = lds_u32(qe + 4 * Q_FLAG) | (big ? (QF_POISON | QF_OWN) : 0u);
+            const bool pois = fl & QF_POISON, counted = fl & QF_COUNT;
+            if (n_out && counted && !pois)
+                atomicAdd(p.act + (size_t)w0.y * (uint32_t)p.n_vdd + (uint32_t)(p.box.k0 + krel), (unsigned long long)n_out);
+            if (lane == 0) {
+                const uint32_t meta = pois ? REC_POISON : (tot | ((fl & QF_SPILL) ? REC_SPILL : 0u));
+                __stcg(grp_rec(G) + (size_t)w0.z * GRP_RSTRIDE(p), make_uint4(w0.w, pois ? 0u : Eo, pois ? 0u : A, meta));
+                if (pois) {
+                    if (!RERUN || counted) poison_bit(p, grp_gi(G), w0.y);
+                    if (fl & QF_OWN) p.ovf[grp_gi(G)] = 1;
+                } else {
+                    sts_u64(G.q + WS_OFF, lds_u64(G.q + WS_OFF) + (unsigned long long)(1u + (fl >> 8)) * (unsigned long long)__popc(Eo));
+                }
             }
         }
         PROF_ACC(4);
