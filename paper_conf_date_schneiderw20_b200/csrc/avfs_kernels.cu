@@ -516,6 +516,9 @@ struct Filt {
 #ifndef AVFS_MERGE_IDX
 #define AVFS_MERGE_IDX 1
 #endif
+#ifndef AVFS_UNIFORM_OFF
+#define AVFS_UNIFORM_OFF 1
+#endif
 __device__ __forceinline__ uint32_t merge_two(const float* a0, int n0, const float* a1, int n1, uint32_t bits,
                                               uint32_t tm0, uint32_t tm1, uint32_t proj, uint32_t tt, float4 dl,
                                               float* out, uint32_t steps) {
@@ -733,9 +736,14 @@ __device__ __forceinline__ void phase_b(const SweepParams& p, const Grp& G, int 
             }
             if (many) m = (uint32_t)(nn[0] + nn[1] + nn[2] + nn[3]);
         }
-        // output offsets: exclusive prefix of the slots' input counts
-        const uint32_t off = warp_incl_scan(m, lane) - m;
+        // output offsets: exclusive prefix of the slots' input counts (all
+        // slots alike, the common pair-major case: lane x count)
         const uint32_t steps = __reduce_max_sync(FULL, m);
+#if AVFS_UNIFORM_OFF
+        const uint32_t off = __reduce_min_sync(FULL, m) == steps ? (uint32_t)lane * m : warp_incl_scan(m, lane) - m;
+#else
+        const uint32_t off = warp_incl_scan(m, lane) - m;
+#endif
         const bool big = __any_sync(FULL, v && m > ENT_N);
         PROF_ACC(2);
         float* out = reinterpret_cast<float*>(lds_u64(qe + 4 * Q_TB)) + off;
