@@ -671,6 +671,7 @@ template <bool RERUN, bool DT>
 __device__ __forceinline__ void phase_b(const SweepParams& p, const Grp& G, int nq, uint32_t q_s, int lane) {
     const uint32_t lmask = (1u << lane) - 1u;
     const int krel = G.krel;
+    uint32_t encb = 0;                                 // this batch's encoding units (lane 0)
     for (int e = 0; e < nq; ++e) {
         PROF_T0();
         const uint32_t qe = q_s + 4u * QW * (uint32_t)e;
@@ -792,12 +793,13 @@ __device__ __forceinline__ void phase_b(const SweepParams& p, const Grp& G, int 
                     if (!RERUN || counted) poison_bit(p, grp_gi(G), w0.y);
                     if (fl & QF_OWN) p.ovf[grp_gi(G)] = 1;
                 } else {
-                    sts_u64(G.q + WS_OFF, lds_u64(G.q + WS_OFF) + (unsigned long long)(1u + (fl >> 8)) * (unsigned long long)__popc(Eo));
+                    encb += (1u + (fl >> 8)) * (uint32_t)__popc(Eo);
                 }
             }
         }
         PROF_ACC(4);
     }
+    if (lane == 0) sts_u64(G.q + WS_OFF, lds_u64(G.q + WS_OFF) + encb);
     __syncwarp();
 }
 
