@@ -181,6 +181,33 @@ def test_slot_range_shards_sum_to_full():
     assert np.array_equal(lat, lat_full)
 
 
+@pytest.mark.parametrize("first,n", [(130, 40), (100, 160), (10, 430), (149, 2)])
+def test_slot_range_boxes(first, n):
+    """Slot ranges whose slot box wraps around the pairs (two partial rows),
+    spans whole rows, or is a single row: every kept waveform and the
+    activity restricted to the range equal the full run's (Q mode)."""
+    w = make_config(3, n_pairs=150, n_vdd=3, scale=0.05)
+    P, V = w.stimuli.n_pairs, len(w.vdd)
+    po = w.netlist.po_sig
+    full = gpu_run(w, keep_all=True, quantum=Q)
+    sig = np.arange(w.netlist.n_signals, dtype=np.int32)
+    wf_full = full.waveforms(sig, 0, w.n_slots, cap=16)
+    full.close()
+    ctx = gpu_run(w, keep_all=True, quantum=Q, slot_range=(first, n))
+    assert ctx.stats()["slots"] == n
+    wf = ctx.waveforms(sig, first, n, cap=16)
+    for a, b in zip(wf, wf_full):
+        assert np.array_equal(a, b[:, first:first + n])
+    # activity per (signal, Vdd) = the full run's counts summed over the range
+    cnt = wf_full[1][:, first:first + n].astype(np.int64)
+    k = np.arange(first, first + n) // P
+    want = np.zeros((w.netlist.n_signals, V), np.int64)
+    for kv in range(V):
+        want[:, kv] = cnt[:, k == kv].sum(1)
+    assert np.array_equal(ctx.activity().astype(np.int64), want)
+    ctx.close()
+
+
 def test_pair_range_shards_sum_to_full():
     """Pair ranges at every operating point (the bench's multi-GPU shards,
     avfs_set_pair_range) reproduce the full run exactly: activity sums,
