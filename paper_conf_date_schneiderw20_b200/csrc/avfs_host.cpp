@@ -1139,6 +1139,11 @@ avfs_status avfs_simulate(avfs_ctx* ctx, void* cuda_stream) {
     if (!has_dev(ctx)) return fail(ctx, AVFS_ERR_STATE, "host-only context");
     if (!ctx->net_loaded || !ctx->stim_set || ctx->vdd.empty())
         return fail(ctx, AVFS_ERR_STATE, "netlist, stimuli and operating points must be set");
+    // the sweep forms activity rows (signal x points) and delay-table rows
+    // (gate x 4 pins x points) as 32-bit element offsets
+    if ((int64_t)(ctx->n_pi + ctx->n_gates) * (int64_t)ctx->vdd.size() >= (int64_t(1) << 32) ||
+        (int64_t)ctx->n_gates * 4 * (int64_t)ctx->vdd.size() >= (int64_t(1) << 32))
+        return fail(ctx, AVFS_ERR_ARG, "signals x operating points too large for 32-bit row offsets");
     SETTLE();                                          // a previous simulate's reruns (same stream)
     const auto t0 = std::chrono::steady_clock::now();
     CK(cudaSetDevice(ctx->dev));

@@ -213,15 +213,21 @@ __device__ unsigned long long g_phase_cycles[16];
 #define AVFS_TAIL_SPLIT 1
 #endif
 constexpr int QN = AVFS_QN;            // gates per batch (Phase A lanes, queue entries)
-constexpr int QW = 40;                 // words per queue entry
+constexpr int QW = 44;                 // words per queue entry
 enum : int {
     Q_TTK = 0, Q_SIG = 1, Q_OUT = 2, Q_Y0 = 3,      // descriptor words, output initial values
-    Q_A = 4, Q_GATE = 5, Q_FLAG = 6,                // entry mask, gate index (delay table row), flags | fanout << 8
+    Q_A = 4, Q_GATE = 5, Q_FLAG = 6,                // entry mask, gate index, flags | fanout << 8
+    Q_DROW = 7,                                     // the gate's delay-table row: gate x 4 x box.nk (float2 units)
     Q_TB = 8,                                       // u64 time base of the output
+    Q_AROW = 10,                                    // the output's activity row: signal x n_vdd + box.k0
+    Q_UNI = 11,                                     // every slot of A alike: UNI_ALIKE | fields below, else 0
     Q_X = 12, Q_E = 16, Q_AQ = 20,                  // per input: init, observable-event, entry masks
     Q_ENTB = 24,                                    // 4 x u64 entry bases of the inputs (PIs: the PI entry table)
-    Q_ITB = 32                                      // 4 x u64 time bases of the inputs
+    Q_ITB = 32,                                     // 4 x u64 time bases of the inputs
+    Q_OREG = 40                                     // u64 output region (its entries)
 };
+// Q_UNI: bits 0-3 the slots' input values, 4-7 their inputs with observable events
+constexpr uint32_t UNI_ALIKE = 0x100u;
 constexpr uint32_t QF_POISON = 1u, QF_COUNT = 2u, QF_OWN = 4u, QF_SPILL = 8u;
 constexpr int WARP_INFO_WORDS = 16;  // per warp, after its queue: enc, region row, record row, gi, sw (u64 each), vmask
 constexpr int WARP_SMEM_WORDS = QN * QW + WARP_INFO_WORDS;
@@ -466,9 +472,27 @@ __device__ __forceinline__ int phase_a(const SweepParams& p, const Grp& G, int g
     if (active) {
         const uint32_t qe = q_s + 4u * QW * (uint32_t)__popc(bal & lanemask_lt());
         sts_u32x4(qe + 4 * Q_TTK, make_uint4(d1.z, sig, d1.x, y0));
+        // the per-gate pass's addresses are formed here, where a lane is a
+        // gate (1/32 of the cost of forming them in the pass)
         sts_u32x4(qe + 4 * Q_A, make_uint4(A, (uint32_t)g,
-                                           (counted ? QF_COUNT : 0u) | (spilled ? QF_SPILL : 0u) | (d1.w << 8), 0u));
+                                           (counted ? QF_COUNT : 0u) | (spilled ? QF_SPILL : 0u) | (d1.w << 8),
+                                           (uint32_t)g * 4u * (uint32_t)p.box.nk));
         sts_u64(qe + 4 * Q_TB, tb);
+        sts_u32(qe + 4 * Q_AROW, sig * (uint32_t)p.n_vdd + (uint32_t)p.box.k0);
+        // the slots of A alike in every input value and observable-event bit
+        // (pair-major groups of one pair: the common case): the per-gate pass
+        // takes its per-slot bits from this word instead of extracting them
+        {
+            uint32_t ub = UNI_ALIKE;
+#pragma unroll
+            for (int q = 0; q < 4; ++q) {
+                const uint32_t xa = X[q] & A, oa = O[q] & A;
+                if ((xa != 0u && xa != A) || (oa != 0u && oa != A)) ub = 0u;
+                ub |= (xa ? 1u << q : 0u) | (oa ? 16u << q : 0u);
+            }
+            sts_u32(qe + 4 * Q_UNI, ub & UNI_ALIKE ? ub : 0u);
+        }
+        sts_u64(qe + 4 * Q_OREG, reinterpret_cast<unsigned long long>(oreg));
         sts_u32x4(qe + 4 * Q_X, make_uint4(X[0], X[1], X[2], X[3]));
         sts_u32x4(qe + 4 * Q_E, make_uint4(O[0], O[1], O[2], O[3]));      // observable events
         sts_u32x4(qe + 4 * Q_AQ, make_uint4(AQ[0], AQ[1], AQ[2], AQ[3]));
@@ -513,9 +537,6 @@ struct Filt {
 #ifndef AVFS_LOOKAHEAD
 #define AVFS_LOOKAHEAD 3
 #endif
-#ifndef AVFS_MERGE_IDX
-#define AVFS_MERGE_IDX 1
-#endif
 #ifndef AVFS_UNIFORM_OFF
 #define AVFS_UNIFORM_OFF 1
 #endif
@@ -533,7 +554,6 @@ __device__ __forceinline__ uint32_t merge_two(const float* a0, int n0, const flo
         w0[i] = n0 > i ? ld_f32(a0 + i) : AVFS_INF;
         w1[i] = n1 > i ? ld_f32(a1 + i) : AVFS_INF;
     }
-#if AVFS_MERGE_IDX
     // list positions as 32-bit indices (next element to load) against fixed
     // bases and counts: one address multiply-add per refill, no 64-bit
     // pointer updates
@@ -560,36 +580,6 @@ __device__ __forceinline__ uint32_t merge_two(const float* a0, int n0, const flo
         F.step(t, live, y, p ? (y ? dl.w : dl.z) : (y ? dl.y : dl.x), out);
     }
     return F.cnt;
-#else
-    a0 += D;
-    a1 += D;
-    n0 -= D;
-    n1 -= D;
-    Filt F{proj, 0u, -AVFS_INF};
-#pragma unroll 1
-    for (uint32_t it = 0; it < steps; ++it) {
-        const bool p = w1[0] < w0[0];                 // ties: the lower pin first (reading C5)
-        const float t = fminf(w0[0], w1[0]);
-        const float* a = p ? a1 : a0;
-        const float nx = (p ? n1 : n0) > 0 ? ld_f32(a) : AVFS_INF;
-#pragma unroll
-        for (int i = 0; i + 1 < D; ++i) {
-            w1[i] = p ? w1[i + 1] : w1[i];
-            w0[i] = p ? w0[i] : w0[i + 1];
-        }
-        w1[D - 1] = p ? nx : w1[D - 1];
-        w0[D - 1] = p ? w0[D - 1] : nx;
-        a1 += p ? 1 : 0;
-        n1 -= p ? 1 : 0;
-        a0 += p ? 0 : 1;
-        n0 -= p ? 0 : 1;
-        const bool live = t < AVFS_INF;
-        bits ^= live ? (p ? tm1 : tm0) : 0u;
-        const uint32_t y = (tt >> bits) & 1u;
-        F.step(t, live, y, p ? (y ? dl.w : dl.z) : (y ? dl.y : dl.x), out);
-    }
-    return F.cnt;
-#endif
 }
 
 // Delay of arc e = 2 pin + pol of sorted gate `gate` at operating point k,
@@ -679,18 +669,26 @@ __device__ __forceinline__ void phase_b(const SweepParams& p, const Grp& G, int 
         const uint32_t A = lds_u32(qe + 4 * Q_A);
         const bool v = (A >> lane) & 1u;
         const uint32_t tt = w0.x & 0xffffu;
-        const uint4 X = lds_u32x4(qe + 4 * Q_X), Ov = lds_u32x4(qe + 4 * Q_E);
         // the slot's input values and its inputs with observable events
-        const uint32_t bits = ((X.x >> lane) & 1u) | (((X.y >> lane) & 1u) << 1) | (((X.z >> lane) & 1u) << 2) |
-                              (((X.w >> lane) & 1u) << 3);
-        const uint32_t use = ((Ov.x >> lane) & 1u) | (((Ov.y >> lane) & 1u) << 1) | (((Ov.z >> lane) & 1u) << 2) |
-                             (((Ov.w >> lane) & 1u) << 3);
-        // the (at most two) first inputs with observable events, p0 < p1, and
-        // their entries (PIs: the PI entry table, reading C2)
+        // and the (at most two) first inputs with observable events, p0 < p1
+        uint32_t bits, use;
+        const uint32_t ub = lds_u32(qe + 4 * Q_UNI);
+        if (ub) {                                      // warp-uniform: every slot of A alike (phase A)
+            bits = ub & 15u;
+            use = v ? (ub >> 4) & 15u : 0u;
+        } else {
+            const uint4 X = lds_u32x4(qe + 4 * Q_X), Ov = lds_u32x4(qe + 4 * Q_E);
+            bits = ((X.x >> lane) & 1u) | (((X.y >> lane) & 1u) << 1) | (((X.z >> lane) & 1u) << 2) |
+                   (((X.w >> lane) & 1u) << 3);
+            use = ((Ov.x >> lane) & 1u) | (((Ov.y >> lane) & 1u) << 1) | (((Ov.z >> lane) & 1u) << 2) |
+                  (((Ov.w >> lane) & 1u) << 3);
+        }
+        // (taking p0, p1 from phase A as well measured slower: 74.6 vs 71.2 ms)
         const int p0 = use ? __ffs(use) - 1 : 0;
         const uint32_t rest = use & (use - 1u);
         const int p1 = rest ? __ffs(rest) - 1 : p0;
         const bool many = (rest & (rest - 1u)) != 0u;
+        // their entries (PIs: the PI entry table, reading C2)
         uint32_t e0 = 0, e1 = 0;
         if (use) {
             const uint32_t* eb = reinterpret_cast<const uint32_t*>(lds_u64(qe + 4 * Q_ENTB + 8 * p0));
@@ -704,9 +702,10 @@ __device__ __forceinline__ void phase_b(const SweepParams& p, const Grp& G, int 
         float4 dl = make_float4(1.0f, 1.0f, 1.0f, 1.0f);
         if (use && !many) {
             if (DT) {                                  // (fall, rise) of each pin: one 8-B load
-                const float2* db = reinterpret_cast<const float2*>(p.dtab) + (size_t)gate * 4u * (uint32_t)p.box.nk + krel;
-                const float2 d0 = __ldg(db + (uint32_t)p0 * (uint32_t)p.box.nk);
-                const float2 d1 = __ldg(db + (uint32_t)p1 * (uint32_t)p.box.nk);
+                const uint32_t dr = lds_u32(qe + 4 * Q_DROW) + (uint32_t)krel;
+                const float2* db = reinterpret_cast<const float2*>(p.dtab);
+                const float2 d0 = __ldg(db + (dr + (uint32_t)p0 * (uint32_t)p.box.nk));
+                const float2 d1 = __ldg(db + (dr + (uint32_t)p1 * (uint32_t)p.box.nk));
                 dl = make_float4(d0.x, d0.y, d1.x, d1.y);
             } else {
                 dl.x = item_delay<DT>(p, gate, krel, 2 * p0);
@@ -773,7 +772,7 @@ __device__ __forceinline__ void phase_b(const SweepParams& p, const Grp& G, int 
             const bool v = (A >> lane) & 1u;
             if (!v) n_out = 0;
             if (v) {
-                uint32_t* oent = reinterpret_cast<uint32_t*>(grp_row(G) + (size_t)w0.z * GRP_STRIDE(p));
+                uint32_t* oent = reinterpret_cast<uint32_t*>(lds_u64(qe + 4 * Q_OREG));
                 __stcg(oent + __popc(A & lmask), min(n_out, ENT_N) | (off << ENT_OFF_SHIFT));
                 if (n_out && (w0.x & (1u << 24))) {
                     const float* o = reinterpret_cast<const float*>(lds_u64(qe + 4 * Q_TB)) + off;
@@ -785,7 +784,7 @@ __device__ __forceinline__ void phase_b(const SweepParams& p, const Grp& G, int 
             const uint32_t fl = lds_u32(qe + 4 * Q_FLAG) | (big ? (QF_POISON | QF_OWN) : 0u);
             const bool pois = fl & QF_POISON, counted = fl & QF_COUNT;
             if (n_out && counted && !pois)
-                atomicAdd(p.act + (size_t)w0.y * (uint32_t)p.n_vdd + (uint32_t)(p.box.k0 + krel), (unsigned long long)n_out);
+                atomicAdd(p.act + (lds_u32(qe + 4 * Q_AROW) + (uint32_t)krel), (unsigned long long)n_out);
             if (lane == 0) {
                 const uint32_t meta = pois ? REC_POISON : (tot | ((fl & QF_SPILL) ? REC_SPILL : 0u));
                 __stcg(grp_rec(G) + (size_t)w0.z * GRP_RSTRIDE(p), make_uint4(w0.w, pois ? 0u : Eo, pois ? 0u : A, meta));
@@ -807,9 +806,14 @@ __device__ __forceinline__ void phase_b(const SweepParams& p, const Grp& G, int 
 template <bool SPLIT, bool RERUN, bool DT>
 __global__ void __launch_bounds__(AVFS_SWEEP_THREADS, AVFS_SWEEP_MINB) sweep_kernel(const SweepParams p) {
     extern __shared__ __align__(16) uint32_t smem_w[];
-    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nw = blockDim.x >> 5;
+    // lane and queue address as opaque values: kept in registers instead of
+    // being rematerialised (S2R + address arithmetic) in every per-gate pass
+    int lane = threadIdx.x & 31;
+    asm volatile("" : "+r"(lane));
+    const int warp = threadIdx.x >> 5, nw = blockDim.x >> 5;
     const uint32_t base_s = smem_u32(smem_w);
-    const uint32_t q_s = base_s + 4u * (uint32_t)(CTA_HDR_WORDS + warp * WARP_SMEM_WORDS);
+    uint32_t q_s = base_s + 4u * (uint32_t)(CTA_HDR_WORDS + warp * WARP_SMEM_WORDS);
+    asm volatile("" : "+r"(q_s));
     // narrow netlists: the CTA walks GP slot groups at once, nw / GP warps
     // each; few slot groups: S co-resident CTAs (consecutive blocks, grid a
     // multiple of S) share one group, each taking 1/S of every level
