@@ -8,19 +8,19 @@
 //                           its PI waveforms with one broadcast load
 //                           (P:L141 step 3).
 //   pi_activity_kernel  H8  PI switching activity per operating point.
-//   sweep_kernel        H6+H7 persistent level sweep.  One CTA owns one
-//                           32-slot group (same Vdd, 32 stimulus pairs) at a
-//                           time and walks every level of the netlist with a
-//                           barrier between levels (P:L166 level-wise
-//                           processing).  Warps grab batches of a level's
-//                           gates; per batch a bit-parallel phase (lane =
-//                           gate, 32 slots per word) evaluates the initial
-//                           values and finds the slots with observable input
-//                           events, and an item phase (lane = (gate, slot))
-//                           merges those slots' input lists with the
-//                           inertial filter (readings C3-C6).
-//                           Delays from the FP64 delay table (Eq. 9).
-//                           Reruns (H7) use the same kernel on the
+//   expand_groups_kernel H4 the same per (PI, pair-major slot group): the PI
+//                           waveforms the sweep reads (no PI storage).
+//   sweep_kernel        H6+H7 persistent level sweep over slot groups
+//                           (pair-major: a group's lanes are one stimulus
+//                           pair's operating points), a barrier per group
+//                           between levels.  Per batch of gates a
+//                           bit-parallel phase (lane = gate, 32 slots per
+//                           word: initial values, observable-event masks)
+//                           and a per-gate pass (lane = slot: merge of the
+//                           input lists with the inertial filter, P:L148,
+//                           readings C3-C6).  Delays from the FP64 delay
+//                           table (Eq. 9) or evaluated in the
+//                           sweep.  Reruns (H7) use the same kernel on the
 //                           overflowed slot groups.
 //   delay_kernel        H2/H3 Eq. (4)/(9) in FP64 per (Vdd, gate, arc).
 //   compact_kernel      H7  list of overflowed slot groups for the rerun.
@@ -94,40 +94,42 @@ __device__ __forceinline__ uint32_t warp_incl_scan(uint32_t v, int) {
 // ---------------------------------------------------------------------------
 // Persistent level sweep (H6 + H7).
 //
-// One CTA owns one 32-slot group (one operating point, 32 stimulus pairs) at
-// a time and walks every level of the netlist with a barrier between levels
-// (P:L166 level-wise processing).  A warp repeatedly grabs a batch of QN
-// gates of the current level and evaluates it in two phases:
+// A CTA walks one or more 32-slot groups at a time (pair-major: a group's
+// lanes are mostly one stimulus pair at 32 operating points)
+// through every level of the netlist, with a (named) barrier per group
+// between levels (P:L166 level-wise processing).  A warp repeatedly grabs a
+// batch of up to QN gates of the current level and evaluates it in two
+// phases:
 //
 //  Phase A (lane = gate; bit-parallel over the 32 slots).  Each lane reads
 //  its gate's descriptor and the records of the gate's inputs (init, event
 //  and entry masks, counts), evaluates the truth table on the 32 initial
-//  values at once (Shannon expansion, y0 = TT(inputs), reading C1) and the
-//  mask A of slots where some input event is observable: the output is not
-//  constant over the input values the slot can take (an input without events
-//  is fixed at its value, one with events is free) -- an event the gate
-//  cannot observe never changes the evaluated output (reading C4) and is not
-//  merged.  Gates with A = 0 (no observable event in any slot) are finished
-//  here: their record {y0, no events} is written and nothing else is read.
-//  The others are queued with their masks, input time bases, and Eq. (9)
-//  delays.  Time storage: a gate whose inputs carry U events in total (an
+//  values at once (Shannon expansion, y0 = TT(inputs), reading C1) and, per
+//  input q, the mask O_q of slots where q's events are observable: the
+//  output is not constant over the input values the slot can take (an input
+//  without events is fixed at its value, one with events is free) -- an
+//  event the gate cannot observe never changes the evaluated output
+//  (reading C4) and is not merged.  A = the union of the O_q.  Gates with
+//  A = 0 are finished here: their record {y0, no events} is written and
+//  nothing else is read.  The others are queued (shared memory) with their
+//  masks, input entry / time bases and the addresses the per-gate pass
+//  needs.  Time storage: a gate whose inputs carry U events in total (an
 //  upper bound of its outputs, reading C17) stores its times in place if
-//  U <= W, else in the round's spill heap; heap exhausted -> poisoned and
-//  the slot group rerun (H7).
+//  U <= W, else in the round's spill heap (one bump allocation per warp);
+//  heap exhausted -> poisoned and the slot group rerun (H7).
 //
-//  Phase B (lane = item = (queued gate, slot in A); items packed 32 per
-//  pass).  Per item: the observable inputs (the per-slot pruning rule
-//  above), their entries (count, offset), output offsets as a segmented
-//  prefix sum of the items' input event counts, then the lane-serial merge
-//  of the sorted input lists by (time, pin) (ties: ascending pin, reading
-//  C5) with the inertial filter (reading C3: a change whose time
-//  precedes the pending output cancels it, equality kept; C4: no reschedule
-//  on confirming events).  Surviving outputs t + d(pin, polarity) are
-//  stored as they are pushed -- only the last one can later be cancelled.
-//  Counts, event masks, activity (reading C15) and the latest PO arrival
-//   are accumulated per queued gate in shared memory; a final step
-//  (lane = queued gate) writes the output records and does one global
-//  atomic per gate and operating point.
+//  Phase B (one queued gate per pass, lane = slot).  Per lane: the slot's
+//  input values and observable inputs, the entries (count, offset) of the
+//  first two observable inputs, the two pins' delays at the lane's operating
+//  point (delay table, or Eq. (4)/(9) evaluated here), the output offset,
+//  then the lane-serial merge of the sorted input lists by (time, pin)
+//  (ties: ascending pin, reading C5) with the inertial filter (
+//  reading C3: a change whose time precedes the pending output cancels it,
+//  equality kept; C4: no reschedule on confirming events).  Surviving
+//  outputs t + d(pin, polarity) are stored as they are pushed -- only the
+//  last one can later be cancelled.  Then the slot's entry, its activity
+//  (reading C15, one u64 reduction per lane), a PO's latest time
+//  and -- lane 0 -- the gate's record.
 // ---------------------------------------------------------------------------
 
 __device__ __forceinline__ uint32_t smem_u32(const void* p) {
@@ -653,6 +655,44 @@ __device__ __forceinline__ uint32_t merge_four(const SweepParams& p, const float
     return F.cnt;
 }
 
+// The end of a queued gate's pass: its entries, record, activity per
+// (signal, point) (reading C15, counted once per slot group across rerun
+// rounds), latest PO arrival.  The queue words are read again here
+// rather than held in registers through the merge.
+template <bool RERUN>
+__device__ __forceinline__ void gate_output(const SweepParams& p, const Grp& G, uint32_t qe, uint32_t n_out,
+                                            uint32_t off, bool big, int lane, uint32_t lmask, int krel,
+                                            uint32_t& encb) {
+    const uint4 w0 = lds_u32x4(qe + 4 * Q_TTK);
+    const uint32_t A = lds_u32(qe + 4 * Q_A);
+    const bool v = (A >> lane) & 1u;
+    if (!v) n_out = 0;
+    if (v) {
+        uint32_t* oent = reinterpret_cast<uint32_t*>(lds_u64(qe + 4 * Q_OREG));
+        __stcg(oent + __popc(A & lmask), min(n_out, ENT_N) | (off << ENT_OFF_SHIFT));
+        if (n_out && (w0.x & (1u << 24))) {
+            const float* o = reinterpret_cast<const float*>(lds_u64(qe + 4 * Q_TB)) + off;
+            atomicMax(p.latest + p.box.k0 + krel, __float_as_uint(__ldcg(o + n_out - 1)));
+        }
+    }
+    const uint32_t Eo = __ballot_sync(FULL, n_out != 0u);
+    const uint32_t tot = __reduce_add_sync(FULL, n_out);
+    const uint32_t fl = lds_u32(qe + 4 * Q_FLAG) | (big ? (QF_POISON | QF_OWN) : 0u);
+    const bool pois = fl & QF_POISON, counted = fl & QF_COUNT;
+    if (n_out && counted && !pois)
+        atomicAdd(p.act + (lds_u32(qe + 4 * Q_AROW) + (uint32_t)krel), (unsigned long long)n_out);
+    if (lane == 0) {
+        const uint32_t meta = pois ? REC_POISON : (tot | ((fl & QF_SPILL) ? REC_SPILL : 0u));
+        __stcg(grp_rec(G) + (size_t)w0.z * GRP_RSTRIDE(p), make_uint4(w0.w, pois ? 0u : Eo, pois ? 0u : A, meta));
+        if (pois) {
+            if (!RERUN || counted) poison_bit(p, grp_gi(G), w0.y);
+            if (fl & QF_OWN) p.ovf[grp_gi(G)] = 1;
+        } else {
+            encb += (1u + (fl >> 8)) * (uint32_t)__popc(Eo);
+        }
+    }
+}
+
 // Phase B, one queued gate per pass, lane = slot (pair-major groups: a
 // gate's observable slots are mostly all 32 operating points of one pair,
 // with alike event counts): merge, outputs, entries, activity and the
@@ -762,40 +802,7 @@ __device__ __forceinline__ void phase_b(const SweepParams& p, const Grp& G, int 
             n_out = merge_two(a0, n0, a1, rest ? n1 : 0, bits, 1u << p0, rest ? 1u << p1 : 0u, y0, tt, dl, out, steps);
         }
         PROF_ACC(3);
-        // the gate's output: entries, record, activity per (signal, point)
-        // (reading C15, counted once per slot group across rerun rounds),
-        // latest PO arrival.  The queue words are read again here
-        // rather than held in registers through the merge.
-        {
-            const uint4 w0 = lds_u32x4(qe + 4 * Q_TTK);
-            const uint32_t A = lds_u32(qe + 4 * Q_A);
-            const bool v = (A >> lane) & 1u;
-            if (!v) n_out = 0;
-            if (v) {
-                uint32_t* oent = reinterpret_cast<uint32_t*>(lds_u64(qe + 4 * Q_OREG));
-                __stcg(oent + __popc(A & lmask), min(n_out, ENT_N) | (off << ENT_OFF_SHIFT));
-                if (n_out && (w0.x & (1u << 24))) {
-                    const float* o = reinterpret_cast<const float*>(lds_u64(qe + 4 * Q_TB)) + off;
-                    atomicMax(p.latest + p.box.k0 + krel, __float_as_uint(__ldcg(o + n_out - 1)));
-                }
-            }
-            const uint32_t Eo = __ballot_sync(FULL, n_out != 0u);
-            const uint32_t tot = __reduce_add_sync(FULL, n_out);
-            const uint32_t fl = lds_u32(qe + 4 * Q_FLAG) | (big ? (QF_POISON | QF_OWN) : 0u);
-            const bool pois = fl & QF_POISON, counted = fl & QF_COUNT;
-            if (n_out && counted && !pois)
-                atomicAdd(p.act + (lds_u32(qe + 4 * Q_AROW) + (uint32_t)krel), (unsigned long long)n_out);
-            if (lane == 0) {
-                const uint32_t meta = pois ? REC_POISON : (tot | ((fl & QF_SPILL) ? REC_SPILL : 0u));
-                __stcg(grp_rec(G) + (size_t)w0.z * GRP_RSTRIDE(p), make_uint4(w0.w, pois ? 0u : Eo, pois ? 0u : A, meta));
-                if (pois) {
-                    if (!RERUN || counted) poison_bit(p, grp_gi(G), w0.y);
-                    if (fl & QF_OWN) p.ovf[grp_gi(G)] = 1;
-                } else {
-                    encb += (1u + (fl >> 8)) * (uint32_t)__popc(Eo);
-                }
-            }
-        }
+        gate_output<RERUN>(p, G, qe, n_out, off, big, lane, lmask, krel, encb);
         PROF_ACC(4);
     }
     if (lane == 0) sts_u64(G.q + WS_OFF, lds_u64(G.q + WS_OFF) + encb);
