@@ -7,7 +7,11 @@ timeout 900 ncu --set full --clock-control none --import-source on -k regex:swee
 # lines of the same run (roofline.traffic)
 python scripts/ncu_summary.py gpurun_out/${TAG:-prof_r02}.ncu-rep --config ${CFG:-4} --tag ${R:-r02} > gpurun_out/ncu_summary.log 2>&1; echo summary rc=$?
 cp profiles/ncu_sweep_traffic.json gpurun_out/ 2>/dev/null
+# compute-sanitizer (memcheck / racecheck / synccheck via scripts/sanitize_run.py) only when
+# AVFS_SANITIZE=1: the GPU pool closed it late in round 2
+if [ "${AVFS_SANITIZE:-0}" = 1 ]; then
 for tool in memcheck racecheck synccheck; do
 timeout 1200 compute-sanitizer --tool $tool --num-cuda-barriers 64 --error-exitcode 9 python scripts/sanitize_run.py > gpurun_out/sanitize_$tool.log 2>&1; echo $tool rc=$?
 tail -3 gpurun_out/sanitize_$tool.log
 done
+fi

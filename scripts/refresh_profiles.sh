@@ -14,5 +14,8 @@ for c in 2 3; do tail -1 gpurun_out/bench_cfg$c.log > profiles/${R}_bench_cfg$c.
 tail -1 gpurun_out/bench_cfg5.log > profiles/${R}_bench_cfg5_shard1of8.json
 tail -1 gpurun_out/bench_cfg5_full.log > profiles/${R}_bench_cfg5_full_1gpu.json
 cp gpurun_out/host.txt profiles/${R}_gpu_box_host.txt
+# (compute-sanitizer was closed on the GPU pool late in round 2: keep the last real run's file)
+if [ -f gpurun_out/sanitize_memcheck.log ] && ! grep -q "compute-sanitizer is closed" gpurun_out/sanitize_memcheck.log; then
 { for t in memcheck racecheck synccheck; do echo "== compute-sanitizer --tool $t (scripts/sanitize_run.py)"; tail -4 gpurun_out/sanitize_$t.log; done; } > profiles/${R}_compute_sanitizer.txt
+fi
 tail -3 gpurun_out/pytest_gpu_all.log > profiles/${R}_pytest_gpu_tail.txt
