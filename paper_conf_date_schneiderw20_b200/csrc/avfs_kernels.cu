@@ -539,23 +539,20 @@ struct Filt {
 #ifndef AVFS_LOOKAHEAD
 #define AVFS_LOOKAHEAD 3
 #endif
+#ifndef AVFS_NOREFILL_LOOP
+#define AVFS_NOREFILL_LOOP 1
+#endif
 #ifndef AVFS_UNIFORM_OFF
 #define AVFS_UNIFORM_OFF 1
 #endif
-__device__ __forceinline__ uint32_t merge_two(const float* a0, int n0, const float* a1, int n1, uint32_t bits,
-                                              uint32_t tm0, uint32_t tm1, uint32_t proj, uint32_t tt, float4 dl,
-                                              float* out, uint32_t steps) {
-    // a window of the next AVFS_LOOKAHEAD elements of each list lives in
-    // registers: their loads are issued together up front, and a refill load
-    // is consumed AVFS_LOOKAHEAD advances of its list later (lists of at most
-    // that many events need no load inside the loop)
+// The merge loop proper; REFILL = false when every lane's lists fit the
+// window (no loads inside the loop).
+template <bool REFILL>
+__device__ __forceinline__ uint32_t merge_two_loop(float (&w0)[AVFS_LOOKAHEAD], float (&w1)[AVFS_LOOKAHEAD],
+                                                   const float* a0, int n0, const float* a1, int n1, uint32_t bits,
+                                                   uint32_t tm0, uint32_t tm1, uint32_t proj, uint32_t tt, float4 dl,
+                                                   float* out, uint32_t steps) {
     constexpr int D = AVFS_LOOKAHEAD;
-    float w0[D], w1[D];
-#pragma unroll
-    for (int i = 0; i < D; ++i) {
-        w0[i] = n0 > i ? ld_f32(a0 + i) : AVFS_INF;
-        w1[i] = n1 > i ? ld_f32(a1 + i) : AVFS_INF;
-    }
     // list positions as 32-bit indices (next element to load) against fixed
     // bases and counts: one address multiply-add per refill, no 64-bit
     // pointer updates
@@ -565,8 +562,13 @@ __device__ __forceinline__ uint32_t merge_two(const float* a0, int n0, const flo
     for (uint32_t it = 0; it < steps; ++it) {
         const bool p = w1[0] < w0[0];                 // ties: the lower pin first (reading C5)
         const float t = fminf(w0[0], w1[0]);
-        const uint32_t ix = p ? i1 : i0;
-        const float nx = (int)ix < (p ? n1 : n0) ? ld_f32((p ? a1 : a0) + ix) : AVFS_INF;
+        float nx = AVFS_INF;
+        if (REFILL) {
+            const uint32_t ix = p ? i1 : i0;
+            nx = (int)ix < (p ? n1 : n0) ? ld_f32((p ? a1 : a0) + ix) : AVFS_INF;
+            i1 += p ? 1u : 0u;
+            i0 += p ? 0u : 1u;
+        }
 #pragma unroll
         for (int i = 0; i + 1 < D; ++i) {
             w1[i] = p ? w1[i + 1] : w1[i];
@@ -574,14 +576,34 @@ __device__ __forceinline__ uint32_t merge_two(const float* a0, int n0, const flo
         }
         w1[D - 1] = p ? nx : w1[D - 1];
         w0[D - 1] = p ? w0[D - 1] : nx;
-        i1 += p ? 1u : 0u;
-        i0 += p ? 0u : 1u;
         const bool live = t < AVFS_INF;
         bits ^= live ? (p ? tm1 : tm0) : 0u;
         const uint32_t y = (tt >> bits) & 1u;
         F.step(t, live, y, p ? (y ? dl.w : dl.z) : (y ? dl.y : dl.x), out);
     }
     return F.cnt;
+}
+
+__device__ __forceinline__ uint32_t merge_two(const float* a0, int n0, const float* a1, int n1, uint32_t bits,
+                                              uint32_t tm0, uint32_t tm1, uint32_t proj, uint32_t tt, float4 dl,
+                                              float* out, uint32_t steps) {
+    // a window of the next AVFS_LOOKAHEAD elements of each list lives in
+    // registers: their loads are issued together up front, and a refill load
+    // is consumed AVFS_LOOKAHEAD advances of its list later; when no lane's
+    // lists are longer than the window (the common case) the loop has no
+    // loads at all
+    constexpr int D = AVFS_LOOKAHEAD;
+    float w0[D], w1[D];
+#pragma unroll
+    for (int i = 0; i < D; ++i) {
+        w0[i] = n0 > i ? ld_f32(a0 + i) : AVFS_INF;
+        w1[i] = n1 > i ? ld_f32(a1 + i) : AVFS_INF;
+    }
+#if AVFS_NOREFILL_LOOP
+    if (__all_sync(FULL, n0 <= D && n1 <= D))
+        return merge_two_loop<false>(w0, w1, a0, n0, a1, n1, bits, tm0, tm1, proj, tt, dl, out, steps);
+#endif
+    return merge_two_loop<true>(w0, w1, a0, n0, a1, n1, bits, tm0, tm1, proj, tt, dl, out, steps);
 }
 
 // Delay of arc e = 2 pin + pol of sorted gate `gate` at operating point k,
