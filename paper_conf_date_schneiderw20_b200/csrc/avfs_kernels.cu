@@ -539,6 +539,10 @@ struct Filt {
 #ifndef AVFS_LOOKAHEAD
 #define AVFS_LOOKAHEAD 3
 #endif
+#ifndef AVFS_MERGE_UNROLL
+#define AVFS_MERGE_UNROLL 2        // merge loop unrolled twice: no loop-carried register copies
+#endif
+constexpr int MERGE_UNROLL = AVFS_MERGE_UNROLL;
 #ifndef AVFS_NOREFILL_LOOP
 #define AVFS_NOREFILL_LOOP 1
 #endif
@@ -558,7 +562,7 @@ __device__ __forceinline__ uint32_t merge_two_loop(float (&w0)[AVFS_LOOKAHEAD], 
     // pointer updates
     uint32_t i0 = D, i1 = D;
     Filt F{proj, 0u, -AVFS_INF};
-#pragma unroll 1
+#pragma unroll MERGE_UNROLL
     for (uint32_t it = 0; it < steps; ++it) {
         const bool p = w1[0] < w0[0];                 // ties: the lower pin first (reading C5)
         const float t = fminf(w0[0], w1[0]);
