@@ -884,15 +884,24 @@ __global__ void __launch_bounds__(AVFS_SWEEP_THREADS, AVFS_SWEEP_MINB) sweep_ker
             const uint32_t cs = ctr_s + 4u * (uint32_t)(L & 1);
             if (wl == 0 && lane == 0) sts_u32(ctr_s + 4u * (uint32_t)((L + 1) & 1), 0u);
             const int nlv = le - ls;
-            // narrow levels (fewer than two full batches per warp): guided
-            // batch sizes, a share of the level's remaining gates, so that
-            // the warps finish together
+            // levels of at most one round of batches (narrow netlists): one
+            // batch per warp, the level split evenly (batch index from the
+            // counter); fewer than two rounds: guided batch sizes, a share of
+            // the level's remaining gates, so that the warps finish together;
+            // wider: full batches and a split last round
+            const bool even = nlv <= QN * wpg;
+            const int esz = (nlv + wpg - 1) / wpg;
             const bool guided = nlv < 2 * QN * wpg;
             if (valid) {
                 while (true) {
                     uint32_t gb = 0;
                     int bsz = QN;
-                    if (guided) {
+                    if (even) {
+                        uint32_t b = 0;
+                        if (lane == 0) b = atoms_add(cs, 1u);
+                        gb = __shfl_sync(FULL, b, 0) * (uint32_t)esz;
+                        bsz = esz;
+                    } else if (guided) {
                         // guided batches: a share of what is left, at most QN
                         // gates, so that the level's last batches are small
                         if (lane == 0) {
