@@ -382,6 +382,19 @@ __device__ __forceinline__ void poison_bit(const SweepParams& p, int64_t gi, uin
     atomicOr(p.pois + (gbit >> 5), 1u << (gbit & 31u));
 }
 
+#ifndef AVFS_PF_L2
+#define AVFS_PF_L2 1
+#endif
+// bulk L2 prefetch of [p, p + bytes) (16-B granules, at most AVFS_PF_MAX bytes)
+#ifndef AVFS_PF_MAX
+#define AVFS_PF_MAX 1024u
+#endif
+__device__ __forceinline__ void l2_prefetch(const void* p, uint32_t bytes) {
+    const uintptr_t a = reinterpret_cast<uintptr_t>(p) & ~uintptr_t(15);
+    const uint32_t n = min((bytes + 15u + (uint32_t)(reinterpret_cast<uintptr_t>(p) & 15u)) & ~15u, AVFS_PF_MAX);
+    if (n) asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(a), "r"(n) : "memory");
+}
+
 // Phase A for gates g0 .. g0 + nb - 1 (nb <= QN); returns the number queued.
 template <bool RERUN>
 __device__ __forceinline__ int phase_a(const SweepParams& p, const Grp& G, int g0, int nb, uint32_t q_s, int lane) {
@@ -507,6 +520,21 @@ __device__ __forceinline__ int phase_a(const SweepParams& p, const Grp& G, int g
                 eb = reinterpret_cast<unsigned long long>(r);
                 itb = (M[q] & REC_SPILL) ? __ldcg(reinterpret_cast<const unsigned long long*>(r + REG_SPILLPTR))
                                          : reinterpret_cast<unsigned long long>(r + times_off(AQ[q]));
+#if AVFS_PF_L2
+                // the observable input's entries and times -> L2 now (one bulk
+                // prefetch of its extent, at most 1 KB), so the per-gate
+                // pass's dependent loads of them hit L2 (prefetching the
+                // pins' delay-table rows as well measured slower: spills)
+                if (O[q]) {
+                    const uint32_t ne = 4u * (uint32_t)__popc(AQ[q]), nt = 4u * (M[q] & REC_NTOT);
+                    if (M[q] & REC_SPILL) {
+                        l2_prefetch(r, ne);
+                        l2_prefetch(reinterpret_cast<const void*>(itb), nt);
+                    } else {
+                        l2_prefetch(r, ne + nt);
+                    }
+                }
+#endif
             }
             sts_u64(qe + 4 * Q_ENTB + 8 * q, eb);
             sts_u64(qe + 4 * Q_ITB + 8 * q, itb);
