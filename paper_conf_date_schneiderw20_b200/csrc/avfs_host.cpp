@@ -1201,7 +1201,7 @@ avfs_status avfs_simulate(avfs_ctx* ctx, void* cuda_stream) {
 
     CK(ctx->d_p1t.ensure((size_t)std::max(ctx->n_pi, 1) * n_pw * 4));
     CK(ctx->d_p2t.ensure((size_t)std::max(ctx->n_pi, 1) * n_pw * 4));
-    CK(ctx->d_p1g.ensure((size_t)std::max(ctx->n_pi, 1) * ctx->n_grp * 4));
+    CK(ctx->d_p1g.ensure((size_t)std::max(ctx->n_pi, 1) * ctx->n_grp * (AVFS_PI_GMAJOR ? 8 : 4)));
     CK(ctx->d_p2g.ensure((size_t)std::max(ctx->n_pi, 1) * ctx->n_grp * 4));
     CK(ctx->d_act.ensure((size_t)S * V * sizeof(unsigned long long)));
     CK(ctx->d_latest.ensure((size_t)V * 4));

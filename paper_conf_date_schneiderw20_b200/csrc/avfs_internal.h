@@ -14,6 +14,10 @@ namespace avfs {
 #define AVFS_SWEEP_MINB (AVFS_SWEEP_THREADS > 768 ? 1 : (AVFS_SWEEP_THREADS > 512 ? 2 : 3))
 #endif
 
+#ifndef AVFS_PI_GMAJOR
+#define AVFS_PI_GMAJOR 1
+#endif
+
 constexpr int KMAX = 4;            // max cell inputs (truth table is 16 bits)
 constexpr int MAX_DEG = 7;         // max polynomial degree per variable
 
@@ -111,7 +115,9 @@ struct SweepParams {
     int32_t n_gates;
     const float* __restrict__ dtab;         // [n_gates][4][box.nk][2] delays, or null: evaluated in the sweep
     DelayParams dp;                         // delay model (used when dtab is null)
-    const uint32_t* __restrict__ p1g;       // [n_pi][n_grp] stimulus words per slot group (bit l: lane l's pair)
+    // stimulus words per slot group (bit l: lane l's pair): uint2 {p1, p2}
+    // [n_grp][n_pi] (AVFS_PI_GMAJOR), else p1g / p2g [n_pi][n_grp]
+    const uint32_t* __restrict__ p1g;
     const uint32_t* __restrict__ p2g;
     int64_t n_grp;                          // slot groups of the box
     SlotBox box;

@@ -415,8 +415,15 @@ __device__ __forceinline__ int phase_a(const SweepParams& p, const Grp& G, int g
         if ((uint32_t)q < K) {
             const uint32_t id = loc[q] & LOC_ID;
             if ((loc[q] & LOC_KIND) == LOC_PI) {       // reading C2: one event at t = 0 iff p1 != p2
+#if AVFS_PI_GMAJOR
+                // the group's (p1, p2) words of every PI are one contiguous
+                // block (L2-resident while the group is swept)
+                const uint2 pw = __ldg(reinterpret_cast<const uint2*>(p.p1g) + (grp_sw(G) * p.n_pi + id));
+                const uint32_t w1 = pw.x, w2 = pw.y;
+#else
                 const int64_t ix = (int64_t)id * p.n_grp + grp_sw(G);
                 const uint32_t w1 = __ldg(p.p1g + ix), w2 = __ldg(p.p2g + ix);
+#endif
                 X[q] = w1;
                 E[q] = AQ[q] = (w1 ^ w2) & grp_vmask(G);
                 M[q] = (uint32_t)__popc(E[q]);
@@ -1168,8 +1175,13 @@ __global__ void expand_groups_kernel(const uint32_t* __restrict__ p1, const uint
     }
     const int pi = b * 32 + lane;
     if (pi < n_pi) {
+#if AVFS_PI_GMAJOR
+        reinterpret_cast<uint2*>(p1g)[sw * n_pi + pi] = make_uint2(m1, m2);
+        (void)p2g;
+#else
         p1g[(int64_t)pi * n_grp + sw] = m1;
         p2g[(int64_t)pi * n_grp + sw] = m2;
+#endif
     }
 }
 
