@@ -32,6 +32,19 @@
 
 #include "avfs_internal.h"
 
+// Debug builds (-DAVFS_CHECKS): device asserts on the sweep's storage
+// invariants -- an observable input has an entry and at least one event in
+// the slot, a gate's outputs stay inside the extent reserved for it (region
+// or heap allocation), heap allocations inside the heap.  A failed assert
+// traps the kernel (sticky CUDA error).  scripts/gpu_checks.sh runs the GPU
+// test suite on such a build.
+#ifdef AVFS_CHECKS
+#include <cassert>
+#define AVFS_CHECK(c) assert(c)
+#else
+#define AVFS_CHECK(c) ((void)0)
+#endif
+
 
 namespace avfs {
 
@@ -226,7 +239,8 @@ enum : int {
     Q_X = 12, Q_E = 16, Q_AQ = 20,                  // per input: init, observable-event, entry masks
     Q_ENTB = 24,                                    // 4 x u64 entry bases of the inputs (PIs: the PI entry table)
     Q_ITB = 32,                                     // 4 x u64 time bases of the inputs
-    Q_OREG = 40                                     // u64 output region (its entries)
+    Q_OREG = 40,                                    // u64 output region (its entries)
+    Q_CAP = 42                                      // (AVFS_CHECKS) words reserved for the output's times
 };
 // Q_UNI: bits 0-3 the slots' input values, 4-7 their inputs with observable events
 constexpr uint32_t UNI_ALIKE = 0x100u;
@@ -515,6 +529,10 @@ __device__ __forceinline__ int phase_a(const SweepParams& p, const Grp& G, int g
             sts_u32(qe + 4 * Q_UNI, ub & UNI_ALIKE ? ub : 0u);
         }
         sts_u64(qe + 4 * Q_OREG, reinterpret_cast<unsigned long long>(oreg));
+#ifdef AVFS_CHECKS
+        AVFS_CHECK(!spilled || wb + need <= p.spill_words);
+        sts_u32(qe + 4 * Q_CAP, spilled ? need : ((uint32_t)p.region_bytes - times_off(A)) / 4u);
+#endif
         sts_u32x4(qe + 4 * Q_X, make_uint4(X[0], X[1], X[2], X[3]));
         sts_u32x4(qe + 4 * Q_E, make_uint4(O[0], O[1], O[2], O[3]));      // observable events
         sts_u32x4(qe + 4 * Q_AQ, make_uint4(AQ[0], AQ[1], AQ[2], AQ[3]));
@@ -728,6 +746,7 @@ __device__ __forceinline__ void gate_output(const SweepParams& p, const Grp& G, 
     const uint32_t A = lds_u32(qe + 4 * Q_A);
     const bool v = (A >> lane) & 1u;
     if (!v) n_out = 0;
+    AVFS_CHECK(!v || big || off + n_out <= lds_u32(qe + 4 * Q_CAP));
     if (v) {
         uint32_t* oent = reinterpret_cast<uint32_t*>(lds_u64(qe + 4 * Q_OREG));
         __stcg(oent + __popc(A & lmask), min(n_out, ENT_N) | (off << ENT_OFF_SHIFT));
@@ -793,11 +812,15 @@ __device__ __forceinline__ void phase_b(const SweepParams& p, const Grp& G, int 
         uint32_t e0 = 0, e1 = 0;
         if (use) {
             const uint32_t* eb = reinterpret_cast<const uint32_t*>(lds_u64(qe + 4 * Q_ENTB + 8 * p0));
+            AVFS_CHECK((lds_u32(qe + 4 * Q_AQ + 4 * p0) >> lane) & 1u);
             e0 = __ldcg(eb + __popc(lds_u32(qe + 4 * Q_AQ + 4 * p0) & lmask));
+            AVFS_CHECK((e0 & ENT_N) >= 1u);
         }
         if (rest) {
             const uint32_t* eb = reinterpret_cast<const uint32_t*>(lds_u64(qe + 4 * Q_ENTB + 8 * p1));
+            AVFS_CHECK((lds_u32(qe + 4 * Q_AQ + 4 * p1) >> lane) & 1u);
             e1 = __ldcg(eb + __popc(lds_u32(qe + 4 * Q_AQ + 4 * p1) & lmask));
+            AVFS_CHECK((e1 & ENT_N) >= 1u);
         }
         const uint32_t gate = lds_u32(qe + 4 * Q_GATE);
         float4 dl = make_float4(1.0f, 1.0f, 1.0f, 1.0f);
