@@ -224,6 +224,9 @@ __device__ unsigned long long g_phase_cycles[16];
 #ifndef AVFS_QN
 #define AVFS_QN 32
 #endif
+#ifndef AVFS_MIN_BATCH
+#define AVFS_MIN_BATCH 12          // smallest guided / tail batch (fewer bit-parallel phases per level)
+#endif
 #ifndef AVFS_TAIL_SPLIT
 #define AVFS_TAIL_SPLIT 1
 #endif
@@ -964,7 +967,7 @@ __global__ void __launch_bounds__(AVFS_SWEEP_THREADS, AVFS_SWEEP_MINB) sweep_ker
                         // gates, so that the level's last batches are small
                         if (lane == 0) {
                             const int rem = nlv - (int)lds_u32(cs);
-                            const int bs = max(1, min(QN, (rem + 2 * wpg - 1) / (2 * wpg)));
+                            const int bs = max(min(AVFS_MIN_BATCH, QN), min(QN, (rem + 2 * wpg - 1) / (2 * wpg)));
                             gb = atoms_add(cs, (uint32_t)bs) | ((uint32_t)bs << 24);
                         }
                         gb = __shfl_sync(FULL, gb, 0);
@@ -977,7 +980,7 @@ __global__ void __launch_bounds__(AVFS_SWEEP_THREADS, AVFS_SWEEP_MINB) sweep_ker
                         // evenly over the group's warps
                         if (lane == 0) {
                             const int rem = nlv - (int)lds_u32(cs);
-                            const int bs = rem >= QN * wpg ? QN : max(1, (rem + wpg - 1) / wpg);
+                            const int bs = rem >= QN * wpg ? QN : max(AVFS_MIN_BATCH, (rem + wpg - 1) / wpg);
                             gb = atoms_add(cs, (uint32_t)bs) | ((uint32_t)bs << 24);
                         }
                         gb = __shfl_sync(FULL, gb, 0);
