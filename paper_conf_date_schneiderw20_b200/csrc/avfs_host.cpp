@@ -246,13 +246,16 @@ avfs_status levelize(avfs_ctx* ctx) {
     for (int32_t g = 0; g < G; ++g) ctx->depth = std::max(ctx->depth, ctx->level[ctx->n_pi + g]);
     ctx->order.resize(G);
     for (int32_t g = 0; g < G; ++g) ctx->order[g] = g;
-    // by level; within a level, gates with <= 2 inputs first, so that most
-    // 32-gate batches evaluate the 2-input masks only (sweep phase A)
+    // by level; within a level, gates with > 2 inputs first, so that they
+    // fill the level's first (full, 32-gate) batches and most batches --
+    // among them all the small ones at the level's end -- evaluate the
+    // 2-input masks only (sweep phase A)
+    const bool wide_last = getenv("AVFS_WIDE_LAST") != nullptr && atoi(getenv("AVFS_WIDE_LAST")) != 0;
     std::stable_sort(ctx->order.begin(), ctx->order.end(), [&](int32_t a, int32_t b) {
         const int32_t la = ctx->level[ctx->n_pi + a], lb = ctx->level[ctx->n_pi + b];
         if (la != lb) return la < lb;
         const bool wa = ctx->fanin_ptr[a + 1] - ctx->fanin_ptr[a] > 2, wb = ctx->fanin_ptr[b + 1] - ctx->fanin_ptr[b] > 2;
-        return !wa && wb;
+        return wide_last ? (!wa && wb) : (wa && !wb);
     });
     ctx->level_ptr.assign(ctx->depth + 1, 0);
     for (int32_t g = 0; g < G; ++g) ctx->level_ptr[ctx->level[ctx->n_pi + g]]++;
