@@ -216,7 +216,11 @@ avfs_status avfs_default_options(avfs_options *opt);
  * call, and the next simulate, settle an outstanding simulate the same way.
  * Runs that need several slot batches settle each batch but the last
  * inside avfs_simulate.  Activity and latest arrival are accumulated over
- * the slot range and reset at the start of each call.                    */
+ * the slot range and reset at the start of each call.  Returns
+ * AVFS_ERR_STATE before netlist / stimuli / operating points are set, and
+ * AVFS_ERR_ARG when signals x operating points (or 4 x gates x points)
+ * reach 2^32 (the sweep forms its activity and delay-table rows as 32-bit
+ * element offsets).                                                       */
 avfs_status avfs_simulate(avfs_ctx *ctx, void *cuda_stream);
 avfs_status avfs_sync(avfs_ctx *ctx);
 
