@@ -39,8 +39,9 @@ constexpr uint32_t LOC_ID = ~LOC_KIND;
 //  region  in the round's arena [group][buffer]: popc(A) entry words, compact
 //          in the order of A's set bits (entry = n | off << ENT_OFF_SHIFT: the
 //          slot's count and the word offset of its first time), then the
-//          binary32 times right after them (byte 4 popc(A)), so a gate's
-//          output is one contiguous extent; when the record says REC_SPILL
+//          binary32 times from byte 128 (times_off: the line after 32
+//          entries; regions are line-aligned), so a gate's output is one
+//          extent; when the record says REC_SPILL
 //          the times live in the spill heap at the 64-bit address stored at
 //          byte REG_SPILLPTR.  Regions hold up to W times.
 constexpr uint32_t REC_NTOT = 0x0FFFFFFFu;
